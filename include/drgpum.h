@@ -1,0 +1,269 @@
+/*
+ * drgpum.h -- C ABI of the B200-native DrGPUM attribution library
+ * (libdrgpum.so, built from paper_conf_asplos_linzs23_b200/csrc for sm_100a).
+ *
+ * The library implements the data-parallel hot path of DrGPUM's object-centric
+ * analysis (Lin, Zhou, Su, ASPLOS '23).  "P:NNN" cites line NNN of the paper
+ * text (/root/reference/PAPER.md at build time; the text is not needed at run
+ * time).  Readings of the paper where it is silent or ambiguous are the
+ * numbered items R1..R18 of DESIGN.md §"Readings".
+ *
+ *   objects + GPU-API timeline  --drgpum_objects_load-->  memory map M as a
+ *       static segment index (§5.1)
+ *   access records              --drgpum_trace_attribute--> per-object bitmap
+ *       (§5.2), first/last use, accessing-API set (P:232,
+ *       Def 3.6/3.7 P:164-168)
+ *   per-object reductions       --drgpum_object_stats-->   accessed elements,
+ *       span, largest unaccessed chunk (Eq. (1)), liveness
+ *   patterns                    --drgpum_patterns-->       EA, LD, UA, ML, TI,
+ *       DW, OA (+Frag) (Defs 3.1-3.8 P:124-174, rules P:244-249)
+ *
+ * Conventions for every call
+ *   - Returns a drgpum_status; nothing throws across the ABI.  On failure the
+ *     context keeps a message for drgpum_last_error() (with the index of the
+ *     first offending object where relevant) and its state is unchanged.
+ *   - "stream" is a cudaStream_t passed as void* (0 = legacy default stream).
+ *     Device-side work is enqueued on it in call order; calls documented as
+ *     "synchronous" synchronise that stream before returning.
+ *   - Host input arrays are copied (or fully consumed) before the call
+ *     returns; the caller may free them afterwards.  Device record buffers are
+ *     BORROWED stream-ordered: keep them alive until the stream passes the call.
+ *   - The workspace is caller-owned device memory (the Python binding takes it
+ *     from torch.empty), bound once per trace; every device array the library
+ *     uses lives inside it.  The library never allocates device memory except
+ *     two tiny event/stream objects for drgpum_trace_attribute_host.
+ *   - One context per device (per rank).  A context is not thread-safe.
+ *   - Call order: create -> objects_load -> workspace_bind ->
+ *     { trace_attribute | trace_attribute_host }* -> [merge_or ...] ->
+ *     finalize / object_stats / patterns.  drgpum_reset starts a new trace on
+ *     the same objects.  Out-of-order calls return DRGPUM_ESTATE.
+ */
+#ifndef DRGPUM_H
+#define DRGPUM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define DRGPUM_API __attribute__((visibility("default")))
+#else
+#define DRGPUM_API
+#endif
+
+/* t_free of an object that is never freed (memory leak, Def 3.5);
+ * t_first of an object that is never accessed (unused, Def 3.4). */
+#define DRGPUM_NEVER 0xFFFFFFFFu
+
+/* GPU APIs of the timeline (footnote 1: allocation, deallocation, copy,
+ * set, kernel launch).  Allocation/deallocation never access an object
+ * (footnote 2). */
+typedef enum {
+  DRGPUM_API_ALLOC = 0, DRGPUM_API_FREE = 1, DRGPUM_API_MEMCPY = 2,
+  DRGPUM_API_MEMSET = 3, DRGPUM_API_KERNEL = 4
+} drgpum_api_kind;
+
+typedef enum {
+  DRGPUM_OK = 0,
+  DRGPUM_EINVAL = 1,    /* malformed argument / object / timeline (rules below) */
+  DRGPUM_EOVERLAP = 2,  /* two objects overlap in address AND in open lifetime [R5] */
+  DRGPUM_ESTATE = 3,    /* call out of order */
+  DRGPUM_ENOMEM = 4,    /* workspace too small / index would exceed limits */
+  DRGPUM_ECUDA = 5      /* CUDA runtime error (message has cudaGetErrorString) */
+} drgpum_status;
+
+/* A data object ("a data object's lifetime, start address, and size").
+ * 32 bytes.  Byte range [base, base+size); elements of elem_size bytes [R1];
+ * open lifetime (t_alloc, t_free): live at ts iff t_alloc < ts < t_free. */
+typedef struct {
+  uint64_t base;
+  uint64_t size;        /* > 0, multiple of elem_size, base+size must not overflow */
+  uint32_t elem_size;   /* 1, 2, 4, 8 or 16 */
+  uint32_t t_alloc;     /* timestamp of its ALLOC API */
+  uint32_t t_free;      /* timestamp of its FREE API, or DRGPUM_NEVER */
+  uint32_t user_id;     /* opaque, not interpreted */
+} drgpum_object_t;
+
+/* One instrumented access ("accessed memory range (i.e., start address
+ * and size)") stamped with the timestamp T of the GPU API that issued it
+ * (P:238).  16 bytes, little-endian; meta = ts | is_write << 31, ts < 2^31. */
+typedef struct {
+  uint64_t addr;
+  uint32_t size;
+  uint32_t meta;
+} drgpum_record_t;
+
+/* Per-object reductions, in the caller's load order.  56 bytes. */
+typedef struct {
+  uint64_t n_elems;                /* size / elem_size */
+  uint64_t accessed;               /* popcount of the bitmap */
+  uint64_t span_lo, span_hi;       /* lowest/highest accessed element; UINT64_MAX if none */
+  uint64_t largest_unaccessed_run; /* longest run of 0 bits in [0, n_elems) (Eq. (1)) */
+  uint32_t t_first, t_last;        /* T_first (DRGPUM_NEVER if unused), T_last (0 if unused) */
+  uint32_t n_access_apis;          /* number of distinct GPU APIs that access the object */
+  uint32_t _pad;
+} drgpum_object_stats_t;
+
+/* User-tunable thresholds.  Defaults {2, 80, 80}: TI X=2, OA 80%
+ * (P:268), Frag 80%. */
+typedef struct {
+  uint32_t ti_min_idle;      /* TI if >= this many APIs lie between consecutive accesses */
+  uint32_t oa_accessed_pct;  /* OA if 100*accessed < pct*n_elems (strict, [R10]) */
+  uint32_t oa_frag_pct;      /* OA_ACTIONABLE if also Frag < pct (Eq. (1), [R11]) */
+} drgpum_thresholds_t;
+
+enum {
+  DRGPUM_EA = 1,            /* early allocation      Def 3.1, rule P:244 */
+  DRGPUM_LD = 2,            /* late deallocation     Def 3.2, rule P:245, never for ML [R8] */
+  DRGPUM_UA = 4,            /* unused allocation     Def 3.4, rule P:246 */
+  DRGPUM_ML = 8,            /* memory leak           Def 3.5, rule P:247 */
+  DRGPUM_TI = 16,           /* temporary idleness    Def 3.6, rule P:248 */
+  DRGPUM_DW = 32,           /* dead write            Def 3.7, rule P:249 [R12] */
+  DRGPUM_OA = 64,           /* overallocation        Def 3.8, P:268 [R9] */
+  DRGPUM_OA_ACTIONABLE = 128/* OA and Frag below threshold (Table 2) */
+};
+
+/* Pattern report per object (load order).  32 bytes.  Distances are
+ * timestamp differences (inefficiency distance) and are 0 unless the
+ * pattern fires; "APIs between" = distance - 1 [R6]. */
+typedef struct {
+  uint32_t flags;
+  uint32_t ea_distance;     /* T_first - T_alloc when EA */
+  uint32_t ld_distance;     /* T_free - T_last when LD */
+  uint32_t ti_ranges;       /* number of idle gaps >= ti_min_idle */
+  uint32_t ti_max_idle;     /* longest such gap, in APIs */
+  uint32_t dw_pairs;        /* consecutive copy/set write pairs */
+  uint64_t ti_total_idle;   /* sum of those gaps */
+} drgpum_pattern_report_t;
+
+/* Trace counters.  records = attributed + unattributed +
+ * invalid; clipped <= attributed. */
+typedef struct {
+  uint64_t records;
+  uint64_t attributed;      /* found a live object containing addr */
+  uint64_t unattributed;    /* no live object contains addr [R4] */
+  uint64_t clipped;         /* attributed but ran past the object's end [R3] */
+  uint64_t invalid;         /* size 0, ts >= n_api, ts of ALLOC/FREE [R14], addr+size overflow */
+} drgpum_counters_t;
+
+/* Where the mergeable shadow state lives inside the workspace (byte offsets
+ * from the workspace base), for multi-GPU exchange.  The OR-
+ * mergeable words (bitmaps then hit rows) are ONE contiguous u32 array of
+ * or_words words at or_off.  first/last are u32[n_obj]; counters u64[5]. */
+typedef struct {
+  uint64_t or_off, or_words;
+  uint64_t bitmap_words, hit_words;   /* or_words = bitmap_words + hit_words */
+  uint64_t first_off, last_off, counters_off;
+  uint64_t n_obj;
+} drgpum_shadow_view_t;
+
+/* Per-object placement in the shadow (load order). */
+typedef struct {
+  uint64_t bitmap_word;   /* first u32 word of the object's bitmap (element e = bit e%32 of word bitmap_word + e/32) */
+  uint64_t hit_word;      /* first u32 word of its hit row, relative to bitmap_words */
+  uint32_t r_lo;          /* access-API rank of the first access API after t_alloc */
+  uint32_t n_hit_apis;    /* access APIs inside (t_alloc, t_free); hit bit 2*(rank-r_lo)+is_write */
+} drgpum_object_layout_t;
+
+typedef struct drgpum_ctx drgpum_ctx;
+
+/* Create a context on a CUDA device.  EINVAL if out is NULL; ECUDA if the
+ * device cannot be selected. */
+DRGPUM_API drgpum_status drgpum_create(int cuda_device, drgpum_ctx **out);
+
+/* Load the object table and the GPU-API timeline (host arrays, copied).
+ * Builds the memory map M as a static segment index valid for
+ * every timestamp, the bitmap/hit-row layout and the access-API rank tables.
+ * EINVAL: n_api >= 2^31; n_obj >= 2^32-1; an api kind > 4; per object: size
+ * 0, elem_size not in {1,2,4,8,16}, size % elem_size, base+size overflow,
+ * t_alloc >= n_api or not an ALLOC, t_free != NEVER and (>= n_api, <= t_alloc
+ * or not a FREE).  EOVERLAP: two objects overlap in address and in open
+ * lifetime [R5].  ENOMEM: the index would exceed 2^32-1 candidate entries.
+ * Allowed after create, or again after a previous load (discards it). */
+DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx *ctx,
+    const drgpum_object_t *h_objs, uint64_t n_obj,
+    const uint8_t *h_api_kinds, uint32_t n_api);
+
+/* Bytes of device workspace the loaded program needs (ESTATE before load). */
+DRGPUM_API drgpum_status drgpum_workspace_size(const drgpum_ctx *ctx, uint64_t *bytes);
+
+/* Bind caller-owned device memory (>= workspace_size bytes, 256-B aligned)
+ * and enqueue on stream: upload of the static tables and zero-initialisation
+ * of the shadow state (bitmaps/hit rows 0, first NEVER, last 0, counters 0).
+ * ENOMEM if bytes is too small; EINVAL if d_ws is NULL or misaligned. */
+DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx *ctx, void *d_ws,
+    uint64_t bytes, void *stream);
+
+/* Enqueue re-zeroing of the shadow state: start a new trace over the same
+ * objects and timeline (what one benchmark step does). */
+DRGPUM_API drgpum_status drgpum_reset(drgpum_ctx *ctx, void *stream);
+
+/* Attribute n device-resident records (d_recs 16-B aligned; n = 0 is a
+ * no-op).  Asynchronous.  For every record: find the object live at its
+ * timestamp that contains addr, set the bits of the touched elements, OR the
+ * (API, read/write) hit bit, fold ts into first/last, count it (SURVEY §8(a)
+ * A1-A5).  Records never fail the call; bad ones are counted as invalid.
+ * Order-free: any permutation / chunking of the records gives identical
+ * results.  EINVAL if d_recs is NULL (n > 0) or misaligned. */
+DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx *ctx,
+    const drgpum_record_t *d_recs, uint64_t n, void *stream);
+
+/* Same, from HOST memory: streams the records through two staging buffers
+ * inside the workspace, overlapping host-to-device copies with attribution.
+ * Synchronous w.r.t. the host buffer: returns once every record has been
+ * copied (the attribution may still be running on stream).  Pinned memory
+ * gives full PCIe/C2C bandwidth; pageable memory works but is slower. */
+DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx *ctx,
+    const drgpum_record_t *h_recs, uint64_t n, void *stream);
+
+/* Shadow-state locations inside the workspace (for merges), and per-object
+ * placement (h_out has n_obj entries, load order). */
+DRGPUM_API drgpum_status drgpum_shadow_view(const drgpum_ctx *ctx, drgpum_shadow_view_t *out);
+DRGPUM_API drgpum_status drgpum_object_layout(const drgpum_ctx *ctx, drgpum_object_layout_t *h_out);
+
+/* OR-merge: for w in [word_lo, word_hi) of the OR-mergeable
+ * words, or_words[w] |= OR_{s<n_src} d_in[s*src_stride + (w - word_lo)].
+ * d_in is device memory (e.g. the slices received by an all-to-all).
+ * Asynchronous.  EINVAL if the range exceeds or_words. */
+DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx *ctx, const uint32_t *d_in,
+    uint32_t n_src, uint64_t src_stride_words, uint64_t word_lo,
+    uint64_t word_hi, void *stream);
+
+/* Enqueue the per-object reductions and the pattern classification on the
+ * device (thresholds NULL = defaults).  Asynchronous; the results stay on
+ * the device until object_stats / patterns copy them out. */
+DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx *ctx,
+    const drgpum_thresholds_t *th, void *stream);
+
+/* Synchronous.  Runs finalize if the state changed since the last one, then
+ * copies n_obj stats (load order) and the counters to the host.  Either
+ * output pointer may be NULL. */
+DRGPUM_API drgpum_status drgpum_object_stats(drgpum_ctx *ctx,
+    drgpum_object_stats_t *h_out, drgpum_counters_t *h_ctr, void *stream);
+
+/* Synchronous.  Finalizes with th (NULL = defaults) if needed and copies n_obj
+ * pattern reports (load order) to the host. */
+DRGPUM_API drgpum_status drgpum_patterns(drgpum_ctx *ctx,
+    const drgpum_thresholds_t *th, drgpum_pattern_report_t *h_out, void *stream);
+
+/* Number of internal consistency violations found by the last finalize
+ * (first/last folded by atomics vs the hit rows; must be 0). */
+DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx *ctx,
+    uint64_t *h_errors, void *stream);
+
+/* Message for the last failed call on ctx (never NULL). */
+DRGPUM_API const char *drgpum_last_error(const drgpum_ctx *ctx);
+
+/* Release host-side state (the workspace belongs to the caller). */
+DRGPUM_API void drgpum_destroy(drgpum_ctx *ctx);
+
+/* Number of kernel launches the library has enqueued on this context since
+ * creation (evidence for benchmarks). */
+DRGPUM_API uint64_t drgpum_launch_count(const drgpum_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DRGPUM_H */

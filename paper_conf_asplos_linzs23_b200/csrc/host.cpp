@@ -1,0 +1,620 @@
+// Host side of libdrgpum.so: validation, the static segment index that
+// replaces DrGPUM's memory map M, workspace layout, and the C ABI.
+//
+// M (§5.1 l.238-240) maps the address range of every ACTIVE object
+// to the object and is updated at every alloc/free.  For a whole recorded
+// trace the library builds it once, for all timestamps at the same time: the
+// address line is cut at every object boundary into elementary segments, and
+// each segment lists the objects covering it sorted by t_alloc.  Because two
+// objects may not overlap in address and lifetime (reading R5), the object
+// live at ts in a segment is the last candidate with t_alloc < ts, provided
+// ts < its t_free.  With no address reuse every segment has at most one
+// candidate and the lookup is exactly the paper's binary search over M
+// (l.322, Fig. 5).  Validation of R5 falls out of the same structure: the
+// sorted candidates of every segment must have disjoint open lifetimes.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "../../include/drgpum.h"
+#include "internal.cuh"
+
+using namespace drgpum;
+
+namespace {
+enum State { S_CREATED = 0, S_LOADED = 1, S_BOUND = 2 };
+
+struct Layout {
+  uint64_t orw, first, last, ctr;           // dynamic (reset per trace)
+  uint64_t dyn_end;
+  uint64_t objs, seg_start, seg_cand_off, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
+  uint64_t tiles, tile_off, tile_part, stats, reports, rq, stage;
+  uint64_t total;
+};
+
+constexpr uint64_t kAlign = 256;
+inline uint64_t align_up(uint64_t x, uint64_t a = kAlign) { return (x + a - 1) / a * a; }
+}  // namespace
+
+struct drgpum_ctx {
+  int device = 0;
+  int num_sms = 148;
+  State state = S_CREATED;
+  std::string err;
+  uint64_t launches = 0;
+  // program
+  uint64_t n_obj = 0;
+  uint32_t n_api = 0, n_acc = 0;
+  std::vector<drgpum_object_t> objs;
+  std::vector<uint8_t> kinds;
+  // derived tables (uploaded at bind)
+  std::vector<DevObj> dobj;
+  std::vector<uint64_t> seg_start;
+  std::vector<uint32_t> seg_cand_off;
+  std::vector<CandEntry> cand;
+  std::vector<uint64_t> l1;
+  uint32_t l1_stride = 1;
+  std::vector<uint32_t> acc_rank, acc_ts, n_hit;
+  std::vector<uint8_t> acc_cs;
+  std::vector<Tile> tiles;
+  std::vector<uint32_t> tile_off;
+  std::vector<drgpum_object_layout_t> layout;
+  uint64_t bitmap_words = 0, hit_words = 0;
+  uint32_t rq_cap = 1u << 20;
+  Layout L{};
+  uint8_t* ws = nullptr;
+  uint64_t ws_bytes = 0;
+  // finalize cache
+  bool final_valid = false;
+  drgpum_thresholds_t final_th{2, 80, 80};
+  // host ingest
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
+};
+
+namespace {
+
+drgpum_status fail(drgpum_ctx* c, drgpum_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  if (c) c->err = buf;
+  return s;
+}
+
+drgpum_status cuda_check(drgpum_ctx* c, cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return DRGPUM_OK;
+  return fail(c, DRGPUM_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CK(expr)                                                     \
+  do {                                                               \
+    drgpum_status _s = cuda_check(ctx, (expr), #expr);               \
+    if (_s != DRGPUM_OK) return _s;                                  \
+  } while (0)
+
+template <typename T> T* at(drgpum_ctx* c, uint64_t off) { return reinterpret_cast<T*>(c->ws + off); }
+
+cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
+
+drgpum_status set_device(drgpum_ctx* ctx) { CK(cudaSetDevice(ctx->device)); return DRGPUM_OK; }
+
+uint32_t ilog2(uint32_t e) { uint32_t s = 0; while ((1u << s) < e) ++s; return s; }
+
+// Build everything derived from (objects, kinds) on the host.
+drgpum_status build_tables(drgpum_ctx* c) {
+  const uint64_t n = c->n_obj;
+  const uint32_t n_api = c->n_api;
+  // access-API ranks (footnote 2, l.178: ALLOC/FREE never access)
+  c->acc_rank.assign(n_api, kNone);
+  c->acc_ts.clear();
+  c->acc_cs.clear();
+  std::vector<uint32_t> acc_before(uint64_t(n_api) + 1, 0);
+  for (uint32_t t = 0; t < n_api; ++t) {
+    acc_before[t] = (uint32_t)c->acc_ts.size();
+    const uint8_t k = c->kinds[t];
+    if (k != DRGPUM_API_ALLOC && k != DRGPUM_API_FREE) {
+      c->acc_rank[t] = (uint32_t)c->acc_ts.size();
+      c->acc_ts.push_back(t);
+      c->acc_cs.push_back(k == DRGPUM_API_MEMCPY || k == DRGPUM_API_MEMSET);
+    }
+  }
+  acc_before[n_api] = (uint32_t)c->acc_ts.size();
+  c->n_acc = (uint32_t)c->acc_ts.size();
+
+  // segment index: elementary segments between consecutive object boundaries
+  std::vector<uint64_t>& pts = c->seg_start;
+  pts.clear();
+  pts.reserve(2 * n);
+  for (const auto& o : c->objs) { pts.push_back(o.base); pts.push_back(o.base + o.size); }
+  std::sort(pts.begin(), pts.end());
+  pts.erase(std::unique(pts.begin(), pts.end()), pts.end());
+  const uint64_t S = pts.size();
+  if (S >= 0xFFFFFFFFull) return fail(c, DRGPUM_ENOMEM, "too many segments (%llu)", (unsigned long long)S);
+  auto seg_of = [&](uint64_t a) { return (uint64_t)(std::lower_bound(pts.begin(), pts.end(), a) - pts.begin()); };
+  std::vector<uint64_t> j0(n), j1(n);
+  std::vector<uint64_t> cnt(S + 1, 0);
+  uint64_t total = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    j0[i] = seg_of(c->objs[i].base);
+    j1[i] = seg_of(c->objs[i].base + c->objs[i].size);
+    total += j1[i] - j0[i];
+    if (total >= 0xFFFFFFFFull)
+      return fail(c, DRGPUM_ENOMEM, "segment index exceeds 2^32 candidate entries (address reuse depth)");
+  }
+  // candidate counts by a difference array, offsets by prefix sum
+  std::vector<int64_t> diff(S + 1, 0);
+  for (uint64_t i = 0; i < n; ++i) { diff[j0[i]]++; diff[j1[i]]--; }
+  c->seg_cand_off.assign(S + 1, 0);
+  int64_t run = 0;
+  for (uint64_t j = 0; j < S; ++j) {
+    run += diff[j];
+    c->seg_cand_off[j + 1] = c->seg_cand_off[j] + (uint32_t)run;
+  }
+  c->cand.assign(total, CandEntry{0, 0});
+  std::vector<uint32_t> fillp(c->seg_cand_off.begin(), c->seg_cand_off.end() - 1);
+  std::vector<uint64_t> by_alloc(n);
+  std::iota(by_alloc.begin(), by_alloc.end(), 0);
+  std::stable_sort(by_alloc.begin(), by_alloc.end(), [&](uint64_t a, uint64_t b) {
+    return c->objs[a].t_alloc < c->objs[b].t_alloc;
+  });
+  for (uint64_t i : by_alloc)
+    for (uint64_t j = j0[i]; j < j1[i]; ++j) c->cand[fillp[j]++] = CandEntry{(uint32_t)i, c->objs[i].t_alloc};
+  // R5: within a segment, consecutive candidates (by t_alloc) must have
+  // disjoint open lifetimes: t_alloc(next) >= t_free(prev)
+  for (uint64_t j = 0; j < S; ++j) {
+    for (uint32_t k = c->seg_cand_off[j] + 1; k < c->seg_cand_off[j + 1]; ++k) {
+      const auto& pv = c->objs[c->cand[k - 1].obj];
+      const auto& nx = c->objs[c->cand[k].obj];
+      if (nx.t_alloc < pv.t_free)
+        return fail(c, DRGPUM_EOVERLAP, "objects %u and %u overlap in address and lifetime",
+                    c->cand[k - 1].obj, c->cand[k].obj);
+    }
+  }
+  // level-1 keys for shared memory
+  c->l1_stride = (uint32_t)std::max<uint64_t>(1, (S + kL1MaxKeys - 1) / kL1MaxKeys);
+  c->l1.clear();
+  for (uint64_t j = 0; j < S; j += c->l1_stride) c->l1.push_back(pts[j]);
+
+  // shadow layout: bitmaps (each 4-word aligned) then hit rows
+  c->layout.assign(n, drgpum_object_layout_t{});
+  c->dobj.assign(n, DevObj{});
+  c->n_hit.assign(n, 0);
+  c->tiles.clear();
+  c->tile_off.assign(n + 1, 0);
+  uint64_t bw = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    const auto& o = c->objs[i];
+    const uint64_t ne = o.size / o.elem_size;
+    const uint64_t words = (ne + 31) / 32;
+    c->layout[i].bitmap_word = bw;
+    c->tile_off[i] = (uint32_t)c->tiles.size();
+    for (uint64_t w = 0; w < words; w += kTileWords) {
+      Tile t;
+      t.word_lo = bw + w;
+      t.n_words = (uint32_t)std::min<uint64_t>(kTileWords, words - w);
+      t.obj = (uint32_t)i;
+      t.elem_lo = w * 32;
+      t.n_bits = std::min<uint64_t>(ne - w * 32, uint64_t(kTileWords) * 32);
+      c->tiles.push_back(t);
+    }
+    bw += align_up(words, 4);
+  }
+  if (c->tiles.size() >= 0xFFFFFFFFull) return fail(c, DRGPUM_ENOMEM, "too many reduction tiles");
+  c->tile_off[n] = (uint32_t)c->tiles.size();
+  c->bitmap_words = bw;
+  uint64_t hw = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    const auto& o = c->objs[i];
+    const uint32_t r_lo = acc_before[o.t_alloc];
+    const uint32_t r_hi = o.t_free == DRGPUM_NEVER ? c->n_acc : acc_before[o.t_free];
+    c->layout[i].r_lo = r_lo;
+    c->layout[i].n_hit_apis = r_hi - r_lo;
+    c->layout[i].hit_word = hw;
+    c->n_hit[i] = r_hi - r_lo;
+    DevObj d;
+    d.base = o.base;
+    d.end = o.base + o.size;
+    d.bm_bit = c->layout[i].bitmap_word * 32;
+    d.hit_word = bw + hw;
+    d.t_alloc = o.t_alloc;
+    d.t_free = o.t_free;
+    d.r_lo = r_lo;
+    d.shift = ilog2(o.elem_size);
+    c->dobj[i] = d;
+    hw += (2ull * (r_hi - r_lo) + 31) / 32;
+  }
+  c->hit_words = hw;
+
+  // workspace layout
+  Layout& L = c->L;
+  uint64_t off = 0;
+  auto put = [&](uint64_t bytes) { uint64_t o = off; off = align_up(off + bytes); return o; };
+  L.orw = put(4 * (c->bitmap_words + c->hit_words));
+  L.first = put(4 * n);
+  L.last = put(4 * n);
+  L.ctr = put(8 * C_SLOTS);
+  L.dyn_end = off;
+  L.objs = put(sizeof(DevObj) * n);
+  L.seg_start = put(8 * S);
+  L.seg_cand_off = put(4 * (S + 1));
+  L.cand = put(sizeof(CandEntry) * total);
+  L.l1 = put(8 * c->l1.size());
+  L.acc_rank = put(4ull * n_api);
+  L.acc_ts = put(4ull * c->n_acc);
+  L.acc_cs = put(c->n_acc);
+  L.n_hit = put(4 * n);
+  L.tiles = put(sizeof(Tile) * c->tiles.size());
+  L.tile_off = put(4 * (n + 1));
+  L.tile_part = put(sizeof(BitMonoid) * c->tiles.size());
+  L.stats = put(sizeof(drgpum_object_stats_t) * n);
+  L.reports = put(sizeof(drgpum_pattern_report_t) * n);
+  L.rq = put(sizeof(RangeEntry) * c->rq_cap);
+  L.stage = put(2 * kStageRecords * sizeof(drgpum_record_t));
+  L.total = off;
+  return DRGPUM_OK;
+}
+
+drgpum_status validate(drgpum_ctx* c, const drgpum_object_t* objs, uint64_t n_obj,
+                       const uint8_t* kinds, uint32_t n_api) {
+  if (n_api >= 0x80000000u) return fail(c, DRGPUM_EINVAL, "n_api >= 2^31");
+  if (n_obj >= 0xFFFFFFFFull) return fail(c, DRGPUM_EINVAL, "n_obj >= 2^32-1");
+  if (n_api && !kinds) return fail(c, DRGPUM_EINVAL, "api kinds is NULL");
+  if (n_obj && !objs) return fail(c, DRGPUM_EINVAL, "objects is NULL");
+  for (uint32_t t = 0; t < n_api; ++t)
+    if (kinds[t] > DRGPUM_API_KERNEL) return fail(c, DRGPUM_EINVAL, "api %u has kind %u", t, kinds[t]);
+  for (uint64_t i = 0; i < n_obj; ++i) {
+    const drgpum_object_t& o = objs[i];
+    const uint32_t E = o.elem_size;
+    const char* why = nullptr;
+    if (o.size == 0) why = "size 0";
+    else if (!(E == 1 || E == 2 || E == 4 || E == 8 || E == 16)) why = "elem_size not in {1,2,4,8,16}";
+    else if (o.size % E) why = "size not a multiple of elem_size";
+    else if (o.base > UINT64_MAX - o.size) why = "base+size overflows";
+    else if (o.t_alloc >= n_api || kinds[o.t_alloc] != DRGPUM_API_ALLOC) why = "t_alloc is not an ALLOC API";
+    else if (o.t_free != DRGPUM_NEVER &&
+             (o.t_free >= n_api || o.t_free <= o.t_alloc || kinds[o.t_free] != DRGPUM_API_FREE))
+      why = "t_free is not a FREE API after t_alloc";
+    if (why) return fail(c, DRGPUM_EINVAL, "object %llu: %s", (unsigned long long)i, why);
+  }
+  return DRGPUM_OK;
+}
+
+drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s) {
+  CK(cudaMemsetAsync(ctx->ws, 0, ctx->L.dyn_end, s));
+  ctx->launches += launch_fill_u32(at<uint32_t>(ctx, ctx->L.first), kNever, ctx->n_obj, s);
+  ctx->final_valid = false;
+  return DRGPUM_OK;
+}
+
+AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
+  AttrParams p;
+  p.recs = reinterpret_cast<const uint4*>(recs);
+  p.n = n;
+  p.objs = at<DevObj>(c, c->L.objs);
+  p.seg_start = at<uint64_t>(c, c->L.seg_start);
+  p.seg_cand_off = at<uint32_t>(c, c->L.seg_cand_off);
+  p.cand = at<CandEntry>(c, c->L.cand);
+  p.l1 = at<uint64_t>(c, c->L.l1);
+  p.n_seg = (uint32_t)c->seg_start.size();
+  p.n_l1 = (uint32_t)c->l1.size();
+  p.l1_stride = c->l1_stride;
+  p.n_api = c->n_api;
+  p.acc_rank = at<uint32_t>(c, c->L.acc_rank);
+  p.orw = at<uint32_t>(c, c->L.orw);
+  p.first = at<uint32_t>(c, c->L.first);
+  p.last = at<uint32_t>(c, c->L.last);
+  p.ctr = at<unsigned long long>(c, c->L.ctr);
+  p.rq = at<RangeEntry>(c, c->L.rq);
+  p.rq_cap = c->rq_cap;
+  return p;
+}
+
+}  // namespace
+
+extern "C" {
+
+DRGPUM_API drgpum_status drgpum_create(int cuda_device, drgpum_ctx** out) {
+  if (!out) return DRGPUM_EINVAL;
+  *out = nullptr;
+  drgpum_ctx* ctx = new drgpum_ctx();
+  ctx->device = cuda_device;
+  drgpum_status s = set_device(ctx);
+  if (s != DRGPUM_OK) { *out = ctx; return s; }
+  cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+  *out = ctx;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_object_t* h_objs,
+                                             uint64_t n_obj, const uint8_t* h_api_kinds,
+                                             uint32_t n_api) {
+  if (!ctx) return DRGPUM_EINVAL;
+  drgpum_status s = validate(ctx, h_objs, n_obj, h_api_kinds, n_api);
+  if (s != DRGPUM_OK) return s;
+  drgpum_ctx tmp;  // build into a scratch context so a failure leaves ctx unchanged
+  tmp.n_obj = n_obj;
+  tmp.n_api = n_api;
+  tmp.objs.assign(h_objs, h_objs + n_obj);
+  tmp.kinds.assign(h_api_kinds, h_api_kinds + n_api);
+  tmp.rq_cap = ctx->rq_cap;
+  s = build_tables(&tmp);
+  if (s != DRGPUM_OK) { ctx->err = tmp.err; return s; }
+  ctx->n_obj = tmp.n_obj; ctx->n_api = tmp.n_api; ctx->n_acc = tmp.n_acc;
+  ctx->objs.swap(tmp.objs); ctx->kinds.swap(tmp.kinds); ctx->dobj.swap(tmp.dobj);
+  ctx->seg_start.swap(tmp.seg_start); ctx->seg_cand_off.swap(tmp.seg_cand_off);
+  ctx->cand.swap(tmp.cand); ctx->l1.swap(tmp.l1); ctx->l1_stride = tmp.l1_stride;
+  ctx->acc_rank.swap(tmp.acc_rank); ctx->acc_ts.swap(tmp.acc_ts); ctx->acc_cs.swap(tmp.acc_cs);
+  ctx->n_hit.swap(tmp.n_hit); ctx->tiles.swap(tmp.tiles); ctx->tile_off.swap(tmp.tile_off);
+  ctx->layout.swap(tmp.layout);
+  ctx->bitmap_words = tmp.bitmap_words; ctx->hit_words = tmp.hit_words;
+  ctx->L = tmp.L;
+  ctx->ws = nullptr;
+  ctx->ws_bytes = 0;
+  ctx->state = S_LOADED;
+  ctx->final_valid = false;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_workspace_size(const drgpum_ctx* ctx, uint64_t* bytes) {
+  if (!ctx || !bytes) return DRGPUM_EINVAL;
+  if (ctx->state < S_LOADED) return DRGPUM_ESTATE;
+  *bytes = ctx->L.total;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint64_t bytes, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_LOADED) return fail(ctx, DRGPUM_ESTATE, "workspace_bind before objects_load");
+  if (!d_ws || (reinterpret_cast<uintptr_t>(d_ws) % kAlign))
+    return fail(ctx, DRGPUM_EINVAL, "workspace must be non-NULL and 256-B aligned");
+  if (bytes < ctx->L.total)
+    return fail(ctx, DRGPUM_ENOMEM, "workspace has %llu bytes, needs %llu",
+                (unsigned long long)bytes, (unsigned long long)ctx->L.total);
+  drgpum_status s = set_device(ctx);
+  if (s != DRGPUM_OK) return s;
+  cudaStream_t st = as_stream(stream);
+  ctx->ws = static_cast<uint8_t*>(d_ws);
+  ctx->ws_bytes = bytes;
+  const Layout& L = ctx->L;
+  auto up = [&](uint64_t off, const void* src, uint64_t n) -> drgpum_status {
+    if (!n) return DRGPUM_OK;
+    CK(cudaMemcpyAsync(ctx->ws + off, src, n, cudaMemcpyHostToDevice, st));
+    return DRGPUM_OK;
+  };
+  const uint64_t n = ctx->n_obj;
+  drgpum_status r;
+  if ((r = up(L.objs, ctx->dobj.data(), sizeof(DevObj) * n))) return r;
+  if ((r = up(L.seg_start, ctx->seg_start.data(), 8 * ctx->seg_start.size()))) return r;
+  if ((r = up(L.seg_cand_off, ctx->seg_cand_off.data(), 4 * ctx->seg_cand_off.size()))) return r;
+  if ((r = up(L.cand, ctx->cand.data(), sizeof(CandEntry) * ctx->cand.size()))) return r;
+  if ((r = up(L.l1, ctx->l1.data(), 8 * ctx->l1.size()))) return r;
+  if ((r = up(L.acc_rank, ctx->acc_rank.data(), 4 * ctx->acc_rank.size()))) return r;
+  if ((r = up(L.acc_ts, ctx->acc_ts.data(), 4 * ctx->acc_ts.size()))) return r;
+  if ((r = up(L.acc_cs, ctx->acc_cs.data(), ctx->acc_cs.size()))) return r;
+  if ((r = up(L.n_hit, ctx->n_hit.data(), 4 * n))) return r;
+  if ((r = up(L.tiles, ctx->tiles.data(), sizeof(Tile) * ctx->tiles.size()))) return r;
+  if ((r = up(L.tile_off, ctx->tile_off.data(), 4 * ctx->tile_off.size()))) return r;
+  if ((r = enqueue_reset(ctx, st))) return r;
+  // host vectors stay alive in ctx, so the async uploads are safe; make the
+  // bind synchronous anyway so callers may immediately reuse their stream
+  CK(cudaStreamSynchronize(st));
+  ctx->state = S_BOUND;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_reset(drgpum_ctx* ctx, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "reset before workspace_bind");
+  return enqueue_reset(ctx, as_stream(stream));
+}
+
+DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_record_t* d_recs,
+                                                uint64_t n, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "trace_attribute before workspace_bind");
+  if (n == 0) return DRGPUM_OK;
+  if (!d_recs || reinterpret_cast<uintptr_t>(d_recs) % 16)
+    return fail(ctx, DRGPUM_EINVAL, "records must be non-NULL and 16-B aligned");
+  AttrParams p = attr_params(ctx, d_recs, n);
+  ctx->launches += launch_attribute(p, ctx->num_sms, as_stream(stream));
+  ctx->final_valid = false;
+  CK(cudaGetLastError());
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgpum_record_t* h_recs,
+                                                     uint64_t n, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "trace_attribute_host before workspace_bind");
+  if (n == 0) return DRGPUM_OK;
+  if (!h_recs) return fail(ctx, DRGPUM_EINVAL, "records is NULL");
+  cudaStream_t st = as_stream(stream);
+  if (!ctx->copy_stream) {
+    CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      CK(cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&ctx->ev_used[i], cudaEventDisableTiming));
+    }
+  }
+  drgpum_record_t* stage[2] = {at<drgpum_record_t>(ctx, ctx->L.stage),
+                             at<drgpum_record_t>(ctx, ctx->L.stage) + kStageRecords};
+  // the copy stream must not overwrite a stage before prior work on `st` is done with it
+  CK(cudaEventRecord(ctx->ev_used[0], st));
+  CK(cudaEventRecord(ctx->ev_used[1], st));
+  uint64_t k = 0;
+  for (uint64_t off = 0; off < n; off += kStageRecords, ++k) {
+    const int b = int(k & 1);
+    const uint64_t m = std::min<uint64_t>(kStageRecords, n - off);
+    CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_used[b], 0));
+    CK(cudaMemcpyAsync(stage[b], h_recs + off, m * sizeof(drgpum_record_t), cudaMemcpyHostToDevice,
+                       ctx->copy_stream));
+    CK(cudaEventRecord(ctx->ev_copied[b], ctx->copy_stream));
+    CK(cudaStreamWaitEvent(st, ctx->ev_copied[b], 0));
+    AttrParams p = attr_params(ctx, stage[b], m);
+    ctx->launches += launch_attribute(p, ctx->num_sms, st);
+    CK(cudaEventRecord(ctx->ev_used[b], st));
+  }
+  CK(cudaStreamSynchronize(ctx->copy_stream));
+  ctx->final_valid = false;
+  CK(cudaGetLastError());
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_shadow_view(const drgpum_ctx* ctx, drgpum_shadow_view_t* out) {
+  if (!ctx || !out) return DRGPUM_EINVAL;
+  if (ctx->state < S_LOADED) return DRGPUM_ESTATE;
+  out->or_off = ctx->L.orw;
+  out->or_words = ctx->bitmap_words + ctx->hit_words;
+  out->bitmap_words = ctx->bitmap_words;
+  out->hit_words = ctx->hit_words;
+  out->first_off = ctx->L.first;
+  out->last_off = ctx->L.last;
+  out->counters_off = ctx->L.ctr;
+  out->n_obj = ctx->n_obj;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_object_layout(const drgpum_ctx* ctx, drgpum_object_layout_t* h_out) {
+  if (!ctx || (!h_out && ctx->n_obj)) return DRGPUM_EINVAL;
+  if (ctx->state < S_LOADED) return DRGPUM_ESTATE;
+  std::copy(ctx->layout.begin(), ctx->layout.end(), h_out);
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx* ctx, const uint32_t* d_in, uint32_t n_src,
+                                         uint64_t src_stride_words, uint64_t word_lo,
+                                         uint64_t word_hi, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_or before workspace_bind");
+  const uint64_t total = ctx->bitmap_words + ctx->hit_words;
+  ctx->final_valid = false;  // the caller is merging state into this shadow
+  if (word_lo > word_hi || word_hi > total)
+    return fail(ctx, DRGPUM_EINVAL, "merge range [%llu,%llu) exceeds %llu words",
+                (unsigned long long)word_lo, (unsigned long long)word_hi, (unsigned long long)total);
+  if (word_hi == word_lo || n_src == 0) return DRGPUM_OK;
+  if (!d_in) return fail(ctx, DRGPUM_EINVAL, "d_in is NULL");
+  if (n_src > 1 && src_stride_words < word_hi - word_lo)
+    return fail(ctx, DRGPUM_EINVAL, "src_stride_words smaller than the range");
+  ctx->launches += launch_merge_or(at<uint32_t>(ctx, ctx->L.orw) + word_lo, d_in, n_src,
+                                   src_stride_words, word_hi - word_lo, ctx->num_sms, as_stream(stream));
+  ctx->final_valid = false;
+  CK(cudaGetLastError());
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_thresholds_t* th, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "finalize before workspace_bind");
+  drgpum_thresholds_t t = th ? *th : drgpum_thresholds_t{2, 80, 80};
+  cudaStream_t st = as_stream(stream);
+  CK(cudaMemsetAsync(at<unsigned long long>(ctx, ctx->L.ctr) + C_CONSISTENCY, 0, 8, st));
+  FinalParams p;
+  p.orw = at<uint32_t>(ctx, ctx->L.orw);
+  p.tiles = at<Tile>(ctx, ctx->L.tiles);
+  p.tile_part = at<BitMonoid>(ctx, ctx->L.tile_part);
+  p.n_tiles = ctx->tiles.size();
+  p.tile_off = at<uint32_t>(ctx, ctx->L.tile_off);
+  p.objs = at<DevObj>(ctx, ctx->L.objs);
+  p.first = at<uint32_t>(ctx, ctx->L.first);
+  p.last = at<uint32_t>(ctx, ctx->L.last);
+  p.acc_ts = at<uint32_t>(ctx, ctx->L.acc_ts);
+  p.acc_cs = at<uint8_t>(ctx, ctx->L.acc_cs);
+  p.n_hit = at<uint32_t>(ctx, ctx->L.n_hit);
+  p.n_obj = ctx->n_obj;
+  p.ti_min_idle = t.ti_min_idle;
+  p.oa_pct = t.oa_accessed_pct;
+  p.frag_pct = t.oa_frag_pct;
+  p.stats = ctx->ws + ctx->L.stats;
+  p.reports = ctx->ws + ctx->L.reports;
+  p.ctr = at<unsigned long long>(ctx, ctx->L.ctr);
+  ctx->launches += launch_finalize(p, ctx->num_sms, st);
+  CK(cudaGetLastError());
+  ctx->final_valid = true;
+  ctx->final_th = t;
+  return DRGPUM_OK;
+}
+
+static bool same_th(const drgpum_thresholds_t& a, const drgpum_thresholds_t& b) {
+  return a.ti_min_idle == b.ti_min_idle && a.oa_accessed_pct == b.oa_accessed_pct &&
+         a.oa_frag_pct == b.oa_frag_pct;
+}
+
+DRGPUM_API drgpum_status drgpum_object_stats(drgpum_ctx* ctx, drgpum_object_stats_t* h_out,
+                                             drgpum_counters_t* h_ctr, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "object_stats before workspace_bind");
+  cudaStream_t st = as_stream(stream);
+  if (!ctx->final_valid) {
+    drgpum_status s = drgpum_finalize(ctx, &ctx->final_th, stream);
+    if (s != DRGPUM_OK) return s;
+  }
+  if (h_out && ctx->n_obj)
+    CK(cudaMemcpyAsync(h_out, ctx->ws + ctx->L.stats, sizeof(drgpum_object_stats_t) * ctx->n_obj,
+                       cudaMemcpyDeviceToHost, st));
+  unsigned long long c[C_SLOTS];
+  CK(cudaMemcpyAsync(c, ctx->ws + ctx->L.ctr, sizeof c, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (h_ctr) {
+    h_ctr->records = c[C_RECORDS];
+    h_ctr->attributed = c[C_ATTRIBUTED];
+    h_ctr->unattributed = c[C_UNATTRIBUTED];
+    h_ctr->clipped = c[C_CLIPPED];
+    h_ctr->invalid = c[C_INVALID];
+  }
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_patterns(drgpum_ctx* ctx, const drgpum_thresholds_t* th,
+                                         drgpum_pattern_report_t* h_out, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "patterns before workspace_bind");
+  drgpum_thresholds_t t = th ? *th : drgpum_thresholds_t{2, 80, 80};
+  cudaStream_t st = as_stream(stream);
+  if (!ctx->final_valid || !same_th(t, ctx->final_th)) {
+    drgpum_status s = drgpum_finalize(ctx, &t, stream);
+    if (s != DRGPUM_OK) return s;
+  }
+  if (h_out && ctx->n_obj)
+    CK(cudaMemcpyAsync(h_out, ctx->ws + ctx->L.reports, sizeof(drgpum_pattern_report_t) * ctx->n_obj,
+                       cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx* ctx, uint64_t* h_errors, void* stream) {
+  if (!ctx || !h_errors) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return DRGPUM_ESTATE;
+  cudaStream_t st = as_stream(stream);
+  unsigned long long c[C_SLOTS];
+  CK(cudaMemcpyAsync(c, ctx->ws + ctx->L.ctr, sizeof c, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  *h_errors = c[C_CONSISTENCY];
+  return DRGPUM_OK;
+}
+
+DRGPUM_API const char* drgpum_last_error(const drgpum_ctx* ctx) {
+  if (!ctx) return "null context";
+  return ctx->err.c_str();
+}
+
+DRGPUM_API void drgpum_destroy(drgpum_ctx* ctx) {
+  if (!ctx) return;
+  if (ctx->copy_stream) {
+    cudaStreamDestroy(ctx->copy_stream);
+    for (int i = 0; i < 2; ++i) { cudaEventDestroy(ctx->ev_copied[i]); cudaEventDestroy(ctx->ev_used[i]); }
+  }
+  delete ctx;
+}
+
+DRGPUM_API uint64_t drgpum_launch_count(const drgpum_ctx* ctx) { return ctx ? ctx->launches : 0; }
+
+}  // extern "C"

@@ -1,0 +1,92 @@
+// Internal types shared by the host library and the sm_100a kernels.
+// (Nothing here is shared with oracle/ -- the oracle has its own code.)
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace drgpum {
+
+constexpr uint32_t kNever = 0xFFFFFFFFu;
+constexpr uint32_t kNone = 0xFFFFFFFFu;        // "no object" / invalid rank
+constexpr int kL1MaxKeys = 2048;               // level-1 keys staged in shared memory (16 KB)
+constexpr uint32_t kRangeChunkWords = 4096;    // range-expansion work item (16 KB of bitmap)
+constexpr uint32_t kTileWords = 8192;          // bitmap reduction tile (32 KB)
+constexpr uint64_t kStageRecords = 1ull << 22; // host-ingest staging chunk (64 MB)
+
+// Object as the attribution kernel sees it: 48 bytes, three 16-B loads.
+struct alignas(16) DevObj {
+  uint64_t base, end;       // [base, end)
+  uint64_t bm_bit;          // global bit index of element 0 (word aligned: multiple of 32)
+  uint64_t hit_word;        // global u32 word index of the hit row (inside the OR array)
+  uint32_t t_alloc, t_free; // live iff t_alloc < ts < t_free
+  uint32_t r_lo;            // access-API rank of the first access API after t_alloc
+  uint32_t shift;           // log2(elem_size)
+};
+static_assert(sizeof(DevObj) == 48, "DevObj layout");
+
+// Segment-index candidate: object id + its t_alloc (candidates of a segment
+// are sorted by t_alloc and have disjoint lifetimes).
+struct CandEntry { uint32_t obj, t_alloc; };
+
+// Range-expansion queue entry: inclusive global bit range, <= kRangeChunkWords words.
+struct RangeEntry { uint64_t bit_lo, bit_hi; };
+
+// Bitmap reduction tile: a run of <= kTileWords words of ONE object.
+struct Tile { uint64_t word_lo; uint32_t n_words; uint32_t obj; uint64_t elem_lo; uint64_t n_bits; };
+
+// Bitmap run monoid over a bit sequence.  Positions are
+// relative to the start of the sequence; kNoPos when the sequence has no 1.
+constexpr uint64_t kNoPos = ~0ull;
+struct BitMonoid {
+  uint64_t len, pop, lo, hi, pre, suf, best;
+};
+
+// Counter slots (u64) at the start of the counters block.
+enum : int { C_RECORDS = 0, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID,
+             C_RQ_OVERFLOW, C_CONSISTENCY, C_RQ_COUNT, C_SLOTS = 16 };
+
+struct AttrParams {
+  const uint4* recs;
+  uint64_t n;
+  const DevObj* objs;
+  const uint64_t* seg_start;
+  const uint32_t* seg_cand_off;
+  const CandEntry* cand;
+  const uint64_t* l1;        // every l1_stride-th segment start
+  uint32_t n_seg, n_l1, l1_stride, n_api;
+  const uint32_t* acc_rank;  // [n_api], kNone for ALLOC/FREE
+  uint32_t* orw;             // OR-mergeable words: bitmaps then hit rows
+  uint32_t* first;
+  uint32_t* last;
+  unsigned long long* ctr;
+  RangeEntry* rq;
+  uint32_t rq_cap;
+};
+
+struct FinalParams {
+  const uint32_t* orw;
+  const Tile* tiles;
+  BitMonoid* tile_part;
+  uint64_t n_tiles;
+  const uint32_t* tile_off;  // [n_obj+1]
+  const DevObj* objs;
+  const uint32_t* first;
+  const uint32_t* last;
+  const uint32_t* acc_ts;    // [n_acc]
+  const uint8_t* acc_cs;     // [n_acc] 1 if MEMCPY/MEMSET
+  const uint32_t* n_hit;     // [n_obj] number of access APIs in the hit row
+  uint64_t n_obj;
+  uint32_t ti_min_idle, oa_pct, frag_pct;
+  void* stats;               // drgpum_object_stats[n_obj]
+  void* reports;             // drgpum_pattern_report[n_obj]
+  unsigned long long* ctr;
+};
+
+// Launchers (return the number of kernels enqueued).
+int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);
+int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
+int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
+int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src,
+                    uint64_t src_stride, uint64_t n_words, int num_sms, cudaStream_t s);
+
+}  // namespace drgpum

@@ -1,0 +1,174 @@
+"""Session: one DrGPUM attribution context on one CUDA device.
+
+PyTorch supplies device memory (the workspace), streams and -- for multi-GPU
+merges (parallel.py) -- process groups.  Everything else is a call into
+libdrgpum.so.
+"""
+import ctypes
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import (OBJECT_DTYPE, RECORD_DTYPE, STATS_DTYPE, REPORT_DTYPE, COUNTERS_DTYPE,
+                   LAYOUT_DTYPE, Thresholds, ShadowView, Counters, check)
+
+
+def _np_ptr(a):
+    return ctypes.c_void_p(a.ctypes.data)
+
+
+def _stream_handle(stream):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _thresholds(th):
+    if th is None:
+        return Thresholds(2, 80, 80)
+    if isinstance(th, Thresholds):
+        return th
+    return Thresholds(*th)
+
+
+class Session:
+    """Attribute an access trace to the objects of one program.
+
+    objects: array of OBJECT_DTYPE (32-B drgpum_object_t) records.
+    kinds:   uint8 array, the GPU-API kind of every timestamp.
+    """
+
+    def __init__(self, objects, kinds, device=None):
+        if not torch.cuda.is_available():
+            raise RuntimeError("drgpum Session needs a CUDA device (there is no CPU fallback)")
+        self.L = _lib.load()
+        self.device = torch.device("cuda", torch.cuda.current_device() if device is None
+                                   else torch.device(device).index or 0)
+        objs = np.asarray(objects)
+        self.objects = np.ascontiguousarray(objs if objs.dtype == OBJECT_DTYPE
+                                            else objs.view(OBJECT_DTYPE))
+        self.kinds = np.ascontiguousarray(kinds, dtype=np.uint8)
+        self.n_obj = int(self.objects.shape[0])
+        h = ctypes.c_void_p()
+        st = self.L.drgpum_create(self.device.index, ctypes.byref(h))
+        self._h = h
+        check(self._h, st)
+        check(self._h, self.L.drgpum_objects_load(self._h, _np_ptr(self.objects), self.n_obj,
+                                                  _np_ptr(self.kinds), self.kinds.shape[0]))
+        nbytes = ctypes.c_uint64()
+        check(self._h, self.L.drgpum_workspace_size(self._h, ctypes.byref(nbytes)))
+        self.workspace = torch.empty(max(int(nbytes.value), 256), dtype=torch.uint8,
+                                     device=self.device)
+        with torch.cuda.device(self.device):
+            check(self._h, self.L.drgpum_workspace_bind(
+                self._h, ctypes.c_void_p(self.workspace.data_ptr()), self.workspace.numel(),
+                _stream_handle(None)))
+        v = ShadowView()
+        check(self._h, self.L.drgpum_shadow_view(self._h, ctypes.byref(v)))
+        self.view = v
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            self.L.drgpum_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ------------------------------------------------------------ attribution
+    def reset(self, stream=None):
+        check(self._h, self.L.drgpum_reset(self._h, _stream_handle(stream)))
+
+    def attribute(self, records, stream=None):
+        """records: a CUDA tensor holding 16-B records (any dtype, contiguous,
+        nbytes % 16 == 0) -> drgpum_trace_attribute; or a host numpy array /
+        CPU tensor -> drgpum_trace_attribute_host (pipelined H2D staging)."""
+        if isinstance(records, torch.Tensor):
+            if not records.is_contiguous():
+                raise ValueError("records tensor must be contiguous")
+            nbytes = records.numel() * records.element_size()
+            if nbytes % 16:
+                raise ValueError("records tensor size is not a multiple of 16 bytes")
+            n = nbytes // 16
+            if records.is_cuda:
+                check(self._h, self.L.drgpum_trace_attribute(
+                    self._h, ctypes.c_void_p(records.data_ptr()), n, _stream_handle(stream)))
+            else:
+                check(self._h, self.L.drgpum_trace_attribute_host(
+                    self._h, ctypes.c_void_p(records.data_ptr()), n, _stream_handle(stream)))
+            return
+        a = np.ascontiguousarray(records)
+        if a.dtype != RECORD_DTYPE:
+            a = a.view(RECORD_DTYPE)
+        check(self._h, self.L.drgpum_trace_attribute_host(self._h, _np_ptr(a), a.shape[0],
+                                                          _stream_handle(stream)))
+
+    # ------------------------------------------------------------ results
+    def finalize(self, thresholds=None, stream=None):
+        th = _thresholds(thresholds)
+        check(self._h, self.L.drgpum_finalize(self._h, ctypes.byref(th), _stream_handle(stream)))
+
+    def object_stats(self, stream=None):
+        out = np.zeros(self.n_obj, dtype=STATS_DTYPE)
+        c = Counters()
+        check(self._h, self.L.drgpum_object_stats(self._h, _np_ptr(out), ctypes.byref(c),
+                                                  _stream_handle(stream)))
+        ctr = np.zeros((), dtype=COUNTERS_DTYPE)
+        for k in COUNTERS_DTYPE.names:
+            ctr[k] = getattr(c, k)
+        return out, ctr
+
+    def patterns(self, thresholds=None, stream=None):
+        out = np.zeros(self.n_obj, dtype=REPORT_DTYPE)
+        th = _thresholds(thresholds)
+        check(self._h, self.L.drgpum_patterns(self._h, ctypes.byref(th), _np_ptr(out),
+                                              _stream_handle(stream)))
+        return out
+
+    def consistency_errors(self, stream=None):
+        e = ctypes.c_uint64()
+        check(self._h, self.L.drgpum_consistency_errors(self._h, ctypes.byref(e),
+                                                        _stream_handle(stream)))
+        return int(e.value)
+
+    def layout(self):
+        out = np.zeros(self.n_obj, dtype=LAYOUT_DTYPE)
+        check(self._h, self.L.drgpum_object_layout(self._h, _np_ptr(out)))
+        return out
+
+    def launch_count(self):
+        return int(self.L.drgpum_launch_count(self._h))
+
+    # ------------------------------------------------------------ shadow views
+    def or_words(self):
+        """The OR-mergeable shadow (bitmaps then hit rows) as an int32 CUDA
+        tensor aliasing the workspace."""
+        v = self.view
+        return self.workspace[v.or_off: v.or_off + 4 * v.or_words].view(torch.int32)
+
+    def first_last(self):
+        v = self.view
+        f = self.workspace[v.first_off: v.first_off + 4 * v.n_obj].view(torch.int32)
+        l = self.workspace[v.last_off: v.last_off + 4 * v.n_obj].view(torch.int32)
+        return f, l
+
+    def counters_tensor(self):
+        v = self.view
+        return self.workspace[v.counters_off: v.counters_off + 8 * 5].view(torch.int64)
+
+    def merge_or(self, src, n_src, src_stride_words, word_lo, word_hi, stream=None):
+        check(self._h, self.L.drgpum_merge_or(self._h, ctypes.c_void_p(src.data_ptr()), n_src,
+                                              src_stride_words, word_lo, word_hi,
+                                              _stream_handle(stream)))
+
+    def bitmap(self, o):
+        """Object o's bitmap as a bool numpy array (copies from the device)."""
+        lay = self.layout()[o]
+        ne = int(self.objects["size"][o] // self.objects["elem_size"][o])
+        nw = (ne + 31) // 32
+        w0 = int(lay["bitmap_word"])
+        words = self.or_words()[w0: w0 + nw].cpu().numpy().view(np.uint32)
+        return np.unpackbits(words.view(np.uint8), bitorder="little")[:ne].astype(bool)

@@ -1,0 +1,213 @@
+"""Bit-exact parity of the CUDA path (through the C ABI) with the CPU oracle.
+
+Everything the library produces is an integer function of (objects,
+timeline, records), so every comparison is exact: the whole OR-mergeable
+shadow (every bitmap word and hit-row word, padding included), first/last,
+stats, pattern reports and counters.  Inputs are seeded synthetic programs
+(tracegen) and the paper's worked examples (tests/golden).
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from oracle import Oracle  # noqa: E402
+from tracegen import (build_config, build_tiny, gen_all_records, gen_records, OBJ_DTYPE,  # noqa: E402
+                      REC_DTYPE, NEVER)
+from tests.golden_util import golden_names, load, to_arrays  # noqa: E402
+
+
+def _session(objs, kinds):
+    from paper_conf_asplos_linzs23_b200 import Session
+    return Session(objs, kinds)
+
+
+def _acc_rank(kinds):
+    k = np.asarray(kinds)
+    is_acc = (k != 0) & (k != 1)
+    before = np.concatenate(([0], np.cumsum(is_acc)))   # access APIs strictly before t
+    return before, is_acc
+
+
+def expected_or_words(s, orc, objs, kinds):
+    """The shadow the oracle implies, placed with the library's layout."""
+    lay = s.layout()
+    v = s.view
+    exp = np.zeros(v.or_words, dtype=np.uint32)
+    eb = exp.view(np.uint8)
+    before, _ = _acc_rank(kinds)
+    for o in range(len(objs)):
+        pk = orc.bitmap_packed(o)
+        off = int(lay["bitmap_word"][o]) * 4
+        eb[off: off + pk.size] = pk
+        r_lo = int(before[objs["t_alloc"][o]])
+        assert lay["r_lo"][o] == r_lo
+        tf = int(objs["t_free"][o])
+        r_hi = int(before[-1]) if tf == NEVER else int(before[tf])
+        assert lay["n_hit_apis"][o] == r_hi - r_lo
+        ts, rw = orc.accesses(o)
+        for t, f in zip(ts, rw):
+            slot = 2 * (int(before[t]) - r_lo)
+            for bit, on in ((slot, f & 1), (slot + 1, f & 2)):
+                if on:
+                    w = int(v.bitmap_words) + int(lay["hit_word"][o]) + (bit >> 5)
+                    exp[w] |= np.uint32(1 << (bit & 31))
+    return exp
+
+
+def run_gpu(objs, kinds, recs, chunks=1, host=False, th=None, shuffle_seed=None):
+    s = _session(objs, kinds)
+    r = recs
+    if shuffle_seed is not None:
+        r = recs[np.random.default_rng(shuffle_seed).permutation(len(recs))]
+    if host:
+        for part in np.array_split(r, chunks):
+            s.attribute(part)
+    else:
+        d = torch.from_numpy(np.ascontiguousarray(r).view(np.uint8)).cuda()
+        bounds = np.linspace(0, len(r), chunks + 1).astype(np.int64)
+        for a, b in zip(bounds, bounds[1:]):
+            s.attribute(d[a * 16: b * 16])
+    st, ctr = s.object_stats()
+    rep = s.patterns(th)
+    orw = s.or_words().cpu().numpy().view(np.uint32).copy()
+    f, l = s.first_last()
+    return s, st, ctr, rep, orw, f.cpu().numpy().view(np.uint32), l.cpu().numpy().view(np.uint32)
+
+
+def check_parity(objs, kinds, recs, th=(2, 80, 80), **kw):
+    orc = Oracle(objs, kinds)
+    orc.attribute(recs)
+    ost, octr = orc.stats()
+    orep = orc.patterns(th)
+    s, st, ctr, rep, orw, first, last = run_gpu(objs, kinds, recs, th=th, **kw)
+    assert s.consistency_errors() == 0
+    for name in octr.dtype.names:
+        assert int(ctr[name]) == int(octr[name]), name
+    for name in ost.dtype.names:
+        if name == "_pad":
+            continue
+        bad = np.flatnonzero(st[name] != ost[name])
+        assert bad.size == 0, (name, bad[:5], st[name][bad[:5]], ost[name][bad[:5]])
+    for name in orep.dtype.names:
+        bad = np.flatnonzero(rep[name] != orep[name])
+        assert bad.size == 0, (name, bad[:5], rep[name][bad[:5]], orep[name][bad[:5]])
+    assert np.array_equal(first, ost["t_first"]) and np.array_equal(last, ost["t_last"])
+    exp = expected_or_words(s, orc, objs, kinds)
+    bad = np.flatnonzero(orw != exp)
+    assert bad.size == 0, ("shadow words differ", bad[:8], orw[bad[:8]], exp[bad[:8]])
+    return s
+
+
+@pytest.mark.parametrize("name", golden_names())
+def test_golden_fixtures(name):
+    objs, kinds, recs, _ = to_arrays(load(name))
+    check_parity(objs, kinds, recs)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_tiny_programs(seed):
+    p = build_tiny(2000 + seed)
+    check_parity(p.objects, p.kinds, gen_all_records(p))
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_tiny_programs_no_reuse_chunked(seed):
+    p = build_tiny(3000 + seed, reuse=False)
+    check_parity(p.objects, p.kinds, gen_all_records(p), chunks=3)
+
+
+@pytest.fixture(scope="module")
+def c1():
+    p = build_config("C1")
+    return p, gen_all_records(p)
+
+
+def test_c1_full(c1):
+    p, r = c1
+    check_parity(p.objects, p.kinds, r)
+
+
+def test_c1_shuffled_and_chunked(c1):
+    p, r = c1
+    check_parity(p.objects, p.kinds, r, chunks=7, shuffle_seed=1)
+
+
+def test_c1_host_ingest(c1):
+    p, r = c1
+    check_parity(p.objects, p.kinds, r, host=True, chunks=2)
+
+
+@pytest.mark.parametrize("th", [(0, 100, 100), (1, 50, 20), (5, 90, 99), (100, 1, 1)])
+def test_c1_thresholds(c1, th):
+    p, r = c1
+    check_parity(p.objects, p.kinds, r, th=th)
+
+
+def test_reset_gives_a_fresh_trace(c1):
+    p, r = c1
+    s = _session(p.objects, p.kinds)
+    d = torch.from_numpy(r.view(np.uint8)).cuda()
+    s.attribute(d)
+    st1, c1_ = s.object_stats()
+    s.attribute(d[: 16 * 1000])       # more records, then start over
+    s.reset()
+    s.attribute(d)
+    st2, c2_ = s.object_stats()
+    assert np.array_equal(st1, st2) and c1_ == c2_
+
+
+def test_empty_and_degenerate():
+    # no records at all: every object unused
+    p = build_tiny(7)
+    check_parity(p.objects, p.kinds, np.zeros(0, dtype=REC_DTYPE))
+    # every record invalid or unattributed
+    recs = np.zeros(3, dtype=REC_DTYPE)
+    recs[0] = (1, 0, 1)
+    recs[1] = (2**64 - 8, 16, 1)
+    recs[2] = (0x10, 4, 1)
+    check_parity(p.objects, p.kinds, recs)
+
+
+def test_no_objects():
+    kinds = np.array([4, 4], dtype=np.uint8)
+    recs = np.zeros(2, dtype=REC_DTYPE)
+    recs[0] = (4096, 4, 0)
+    recs[1] = (4096, 4, 1)
+    s = _session(np.zeros(0, dtype=OBJ_DTYPE), kinds)
+    s.attribute(torch.from_numpy(recs.view(np.uint8)).cuda())
+    _, ctr = s.object_stats()
+    assert int(ctr["unattributed"]) == 2 and int(ctr["records"]) == 2
+
+
+def test_max_range_record():
+    """A memset of 2^30 one-byte elements: one record expands to 2^25 words
+    through the range queue (A3b), split into 4096-word work items."""
+    kinds = np.array([0, 3, 4, 1], dtype=np.uint8)
+    objs = np.zeros(1, dtype=OBJ_DTYPE)
+    objs[0] = (1 << 40, 1 << 30, 1, 0, 3, 0)
+    recs = np.zeros(3, dtype=REC_DTYPE)
+    recs[0] = ((1 << 40) + 5, (1 << 30) - 7, 1 | (1 << 31))    # ragged both ends
+    recs[1] = ((1 << 40), 0xFFFFFFFF, 2)                        # clipped at the end
+    recs[2] = ((1 << 40) + 3, 1, 2)
+    check_parity(objs, kinds, recs)
+
+
+def test_uint32_size_boundary():
+    """Largest record (size 2^32-1) over 16-byte elements."""
+    kinds = np.array([0, 2, 1], dtype=np.uint8)
+    objs = np.zeros(1, dtype=OBJ_DTYPE)
+    objs[0] = (1 << 44, 1 << 33, 16, 0, 2, 0)
+    recs = np.zeros(1, dtype=REC_DTYPE)
+    recs[0] = ((1 << 44) + 16 * 3 + 1, 0xFFFFFFFF, 1 | (1 << 31))
+    check_parity(objs, kinds, recs)
+
+
+@pytest.mark.slow
+def test_c2_full_size():
+    """BASELINE.json configs[1] at full size (1e8 records), in the launch
+    configuration bench.py times: every word of the ~115 MiB shadow compared."""
+    p = build_config("C2")
+    r = gen_records(p, 0, p.n_records)
+    check_parity(p.objects, p.kinds, r)
