@@ -229,6 +229,7 @@ def main():
     # touched shadow words of the last step (algorithmic write-back of A3/A4)
     touched = int(torch.count_nonzero(s.or_words()).item())
     stats, ctr = s.object_stats()
+    paths = s.path_stats()
 
     # ---------------- end-to-end through the public API with HOST buffers
     e2e_steps = a.e2e_steps or min(a.steps, 10)
@@ -304,6 +305,7 @@ def main():
         "gpu_launches": launches,
         "clocks": clocks,
         "counters": {k: int(ctr[k]) for k in ctr.dtype.names},
+        "attribution_paths_tiles": paths,
         "wall_s_device_region": wall_dev,
     }
     print(json.dumps(line), flush=True)

@@ -253,6 +253,12 @@ DRGPUM_API drgpum_status drgpum_patterns(drgpum_ctx *ctx,
 DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx *ctx,
     uint64_t *h_errors, void *stream);
 
+/* Diagnostics (not part of the method): how many 32-record tiles took each
+ * attribution path since the last reset -- out[0] affine run with one union
+ * range, out[1] affine run with per-record words, out[2] per-tile fast path
+ * (cached object and API), out[3] full per-lane path.  Synchronous. */
+DRGPUM_API drgpum_status drgpum_path_stats(drgpum_ctx *ctx, uint64_t out[4], void *stream);
+
 /* Message for the last failed call on ctx (never NULL). */
 DRGPUM_API const char *drgpum_last_error(const drgpum_ctx *ctx);
 

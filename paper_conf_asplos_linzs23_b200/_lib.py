@@ -61,7 +61,7 @@ EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_workspace_size",
            "drgpum_workspace_bind", "drgpum_reset", "drgpum_trace_attribute",
            "drgpum_trace_attribute_host", "drgpum_shadow_view", "drgpum_object_layout",
            "drgpum_merge_or", "drgpum_finalize", "drgpum_object_stats", "drgpum_patterns",
-           "drgpum_consistency_errors", "drgpum_last_error", "drgpum_destroy",
+           "drgpum_consistency_errors", "drgpum_path_stats", "drgpum_last_error", "drgpum_destroy",
            "drgpum_launch_count"]
 
 _lib = None
@@ -93,6 +93,7 @@ def load():
         "drgpum_object_stats": ([P, P, ctypes.POINTER(Counters), P], I),
         "drgpum_patterns": ([P, ctypes.POINTER(Thresholds), P, P], I),
         "drgpum_consistency_errors": ([P, ctypes.POINTER(U64), P], I),
+        "drgpum_path_stats": ([P, P, P], I),
         "drgpum_last_error": ([P], ctypes.c_char_p),
         "drgpum_destroy": ([P], None),
         "drgpum_launch_count": ([P], U64),

@@ -1,22 +1,28 @@
 // B1 attribute_kernel + B2 range_expand_kernel (sm_100a).
 //
 // Per record (§5.1 l.238-240, §5.2 l.264-268):
-//   A1  stream the 16-B record (ld.global.nc.L1::no_allocate, 128-bit),
-//       reject invalid ones (size 0, ts >= n_api, ts of an ALLOC/FREE API --
-//       footnote 2 l.178 --, addr+size overflow);
-//   A2  find the object live at ts that contains addr: per-lane cache of the
-//       last object (bursts are warp-coalesced), else a two-level search of
-//       the static segment index (level-1 keys in shared memory, leaves in
-//       L2) and a search of the segment's candidates by t_alloc (address
-//       reuse, reading R5);
-//   A3  clip to the object (R3), turn the byte range into element bits
-//       (partial elements count, R2) and OR them into the object's bitmap:
-//       lanes hitting the same u32 word are merged by a warp segmented scan
-//       (or one REDUX when the whole warp hits one word) and a single RED.OR
-//       per word run; ranges spanning > 2 words go to the range queue (A3b);
+//   A1  stream the 16-B records: each block owns one contiguous record range
+//       and a producer lane streams it through a 4-stage shared-memory ring
+//       with cp.async.bulk (TMA bulk copy, L2 evict-first), mbarrier-paced;
+//       reject invalid records (size 0, ts >= n_api, ts of an ALLOC/FREE API
+//       -- footnote 2 l.178 --, addr+size overflow);
+//   A2  find the object live at ts that contains addr: each lane caches the
+//       last (object, API) it validated; bursts are warp-coalesced, so almost
+//       every 32-record tile takes the uniform FAST path (all lanes inside
+//       their cached object and API: no search, no liveness/hit work).
+//       Otherwise the SLOW path runs the full per-lane algorithm: two-level
+//       search of the static segment index (level-1 keys in shared memory,
+//       leaves in L2), candidate search by t_alloc (address reuse, R5);
+//   A3  clip to the object (R3), element bits (partial elements count, R2),
+//       OR into the object's bitmap.  Fast path: when the 32 lanes' bit
+//       ranges chain into one contiguous range (sequential sweeps of any
+//       access size) the warp writes that union directly, one RED.OR per
+//       word; otherwise runs of equal words are merged by a shuffle
+//       segmented scan (or not at all when every lane has its own word).
+//       Records spanning > 2 words go to the range queue (A3b);
 //   A4  fold ts into first (RED.MIN) / last (RED.MAX) and OR the (access API,
-//       read|write) bit into the object's hit row -- both skipped when this
-//       lane already knows the global value covers it (values are monotone);
+//       read|write) bit into the object's hit row -- once per lane per
+//       (object, API, rw), in the slow path;
 //   A5  count records / attributed / unattributed / clipped / invalid.
 #include "internal.cuh"
 
@@ -24,10 +30,67 @@ namespace drgpum {
 
 #define FULL_MASK 0xFFFFFFFFu
 
-__device__ __forceinline__ uint4 ld_stream(const uint4* p) {
+constexpr int kConsumerWarps = 8;
+constexpr int kAttrThreads = kConsumerWarps * 32;
+constexpr int kStages = 4;                                   // per-warp ring depth
+constexpr int kTilesPerWarp = 4;                             // 32-record tiles per stage
+constexpr int kWarpRecords = kTilesPerWarp * 32;             // 128 records = 2 KB per stage
+// 8 warps x 4 x 2 KB ring + 16 KB level-1 keys + barriers = 80 KB: two blocks
+// per SM leave ~66 KB of L1 for the index / object-table loads
+constexpr size_t kAttrSmem = size_t(kConsumerWarps) * kStages * kWarpRecords * 16 + kL1MaxKeys * 8 +
+                             size_t(kConsumerWarps) * kStages * (8 + 4);
+constexpr uint64_t kChunkRecords = 2048;                     // dynamic work unit (16 stages)
+
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done;
+  do {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  } while (!done);
+}
+// producer-side wait: back off so the spinning lane does not steal issue slots
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+  uint32_t done;
+  asm volatile(
+      "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+      : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  while (!done) {
+    __nanosleep(256);
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  }
+}
+__device__ __forceinline__ void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes,
+                                            uint64_t* bar, uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+      ::"r"(smem_u32(smem_dst)), "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)), "l"(policy) : "memory");
+}
+__device__ __forceinline__ uint64_t evict_first_policy() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint4 lds128(uint32_t saddr) {
   uint4 r;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.u32 {%0,%1,%2,%3}, [%4];"
-               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(saddr));
   return r;
 }
 
@@ -35,6 +98,7 @@ __device__ __forceinline__ uint32_t bits_mask(uint32_t b0, uint32_t b1) {  // bi
   return (0xFFFFFFFFu >> (31 - b1)) & (0xFFFFFFFFu << b0);
 }
 
+// ------------------------------------------------------------------ warp helpers
 // Warp segmented inclusive scan over runs of adjacent lanes with equal keys.
 // Returns the run-reduced value in the run's last lane (tail = true there).
 template <typename Op>
@@ -58,12 +122,18 @@ struct OpMax { __device__ uint32_t operator()(uint32_t a, uint32_t b) const { re
 
 constexpr uint64_t kNoKey = ~0ull;
 
-// OR masks into words, one RED per run of lanes sharing a word.
+// OR masks into words: one RED per run of adjacent lanes sharing a word when
+// runs are long, one RED per lane when (almost) every lane has its own word.
 __device__ __forceinline__ void warp_or_words(uint32_t* words, uint64_t key, uint32_t m, int lane) {
-  const uint64_t k0 = __shfl_sync(FULL_MASK, key, 0);
-  if (__all_sync(FULL_MASK, key == k0)) {
+  const uint64_t pk = __shfl_up_sync(FULL_MASK, key, 1);
+  const uint32_t heads = __ballot_sync(FULL_MASK, lane == 0 || pk != key);
+  if (heads == 1u) {  // one word for the whole warp
     const uint32_t v = __reduce_or_sync(FULL_MASK, m);
-    if (lane == 0 && k0 != kNoKey && v) atomicOr(words + k0, v);
+    if (lane == 0 && key != kNoKey && v) atomicOr(words + key, v);
+    return;
+  }
+  if (__popc(heads) > 16) {  // mostly distinct words: OR is idempotent, just RED
+    if (key != kNoKey && m) atomicOr(words + key, m);
     return;
   }
   bool tail;
@@ -71,9 +141,12 @@ __device__ __forceinline__ void warp_or_words(uint32_t* words, uint64_t key, uin
   if (tail && key != kNoKey && v) atomicOr(words + key, v);
 }
 
+// ------------------------------------------------------------------ lane state
 struct LaneCache {
-  uint64_t base, end, bm_bit, hit_word;
+  uint64_t base, size;        // cached object: [base, base+size)
+  uint64_t bm_word, hit_word;  // object's first bitmap word; hit-row word
   uint32_t t_alloc, t_free, r_lo, shift, obj;
+  uint32_t meta;              // ts|w<<31 whose first/last/hit work is done (fast-path key)
   uint32_t ts, rank;          // last timestamp -> access-API rank
   uint32_t first_known;       // first[obj] <= first_known is known
   uint32_t last_known;        // last[obj]  >= last_known  is known
@@ -86,14 +159,12 @@ struct LaneCounts { uint32_t rec, attr, unattr, clip, inval, ovf; };
 __device__ __forceinline__ uint32_t find_object(const AttrParams& p, const uint64_t* s_l1,
                                                 uint64_t addr, uint32_t ts) {
   if (p.n_seg == 0 || addr < s_l1[0]) return kNone;
-  // level 1 (shared memory): last key <= addr
-  uint32_t lo = 0, hi = p.n_l1;
+  uint32_t lo = 0, hi = p.n_l1;       // level 1 (shared memory): last key <= addr
   while (hi - lo > 1) {
     const uint32_t mid = (lo + hi) >> 1;
     if (s_l1[mid] <= addr) lo = mid; else hi = mid;
   }
-  // level 2 (global/L2): last segment start <= addr within the level-1 block
-  uint32_t a = lo * p.l1_stride;
+  uint32_t a = lo * p.l1_stride;      // level 2 (L2): last segment start <= addr
   uint32_t b = min(a + p.l1_stride, p.n_seg);
   while (b - a > 1) {
     const uint32_t mid = (a + b) >> 1;
@@ -101,8 +172,8 @@ __device__ __forceinline__ uint32_t find_object(const AttrParams& p, const uint6
   }
   const uint32_t c0 = __ldg(p.seg_cand_off + a), c1 = __ldg(p.seg_cand_off + a + 1);
   if (c0 == c1) return kNone;
-  // candidates sorted by t_alloc, lifetimes disjoint: the last one allocated
-  // before ts is the only one that can be live at ts
+  // candidates sorted by t_alloc with disjoint lifetimes: only the last one
+  // allocated before ts can be live at ts
   uint32_t l = c0, h = c1;
   const uint2* cand = reinterpret_cast<const uint2*>(p.cand);
   while (l < h) {
@@ -113,30 +184,35 @@ __device__ __forceinline__ uint32_t find_object(const AttrParams& p, const uint6
   return __ldg(&cand[l - 1].x);
 }
 
-__device__ __noinline__ void enqueue_range(const AttrParams& p, uint64_t gb0, uint64_t gb1, LaneCounts& k) {
+__device__ __noinline__ void enqueue_range(RangeEntry* rq, uint32_t rq_cap, unsigned long long* ctr,
+                                           uint32_t* orw, uint64_t gb0, uint64_t gb1, uint32_t& ovf) {
   const uint64_t wlo = gb0 >> 5, whi = gb1 >> 5;
   const uint64_t nch = (whi - wlo) / kRangeChunkWords + 1;
-  const unsigned long long slot = atomicAdd(&p.ctr[C_RQ_COUNT], (unsigned long long)nch);
+  const unsigned long long slot = atomicAdd(&ctr[C_RQ_COUNT], (unsigned long long)nch);
   for (uint64_t c = 0; c < nch; ++c) {
     const uint64_t cw0 = wlo + c * kRangeChunkWords;
     const uint64_t bl = c == 0 ? gb0 : cw0 * 32;
     const uint64_t bh = min(gb1, (cw0 + kRangeChunkWords) * 32 - 1);
-    if (slot + c < p.rq_cap) {
-      p.rq[slot + c] = RangeEntry{bl, bh};
+    if (slot + c < rq_cap) {
+      rq[slot + c] = RangeEntry{bl, bh};
     } else {  // queue full: expand this chunk in place (slow but exact)
-      k.ovf++;
+      ovf++;
       for (uint64_t w = bl >> 5; w <= (bh >> 5); ++w) {
         uint32_t m = 0xFFFFFFFFu;
         if (w == (bl >> 5)) m &= 0xFFFFFFFFu << (bl & 31);
         if (w == (bh >> 5)) m &= 0xFFFFFFFFu >> (31 - (bh & 31));
-        atomicOr(p.orw + w, m);
+        atomicOr(orw + w, m);
       }
     }
   }
 }
 
-__device__ __forceinline__ void process(const AttrParams& p, const uint64_t* s_l1, uint4 r,
-                                        bool present, int lane, LaneCache& c, LaneCounts& k) {
+// ------------------------------------------------------------------ slow path
+// The complete per-lane algorithm (every lane, any record).  Leaves each lane
+// with c.meta = the record's meta when the record was attributed, so that
+// following records of the same (object, API, rw) take the fast path.
+__device__ __noinline__ void process_slow(const AttrParams& p, const uint64_t* s_l1, uint4 r,
+                                          bool present, int lane, LaneCache& c, LaneCounts& k) {
   const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
   const uint32_t size = r.z;
   const uint32_t ts = r.w & 0x7FFFFFFFu;
@@ -150,7 +226,7 @@ __device__ __forceinline__ void process(const AttrParams& p, const uint64_t* s_l
   // ---- A2: object lookup
   bool att = false;
   if (ok) {
-    att = addr >= c.base && addr < c.end && ts > c.t_alloc && ts < c.t_free;
+    att = addr - c.base < c.size && ts > c.t_alloc && ts < c.t_free;
     if (!att) {
       const uint32_t o = find_object(p, s_l1, addr, ts);
       if (o != kNone) {
@@ -158,8 +234,8 @@ __device__ __forceinline__ void process(const AttrParams& p, const uint64_t* s_l
         const uint4 a = __ldg(q), b = __ldg(q + 1), d = __ldg(q + 2);
         if (ts < d.y) {
           c.base = (uint64_t(a.y) << 32) | a.x;
-          c.end = (uint64_t(a.w) << 32) | a.z;
-          c.bm_bit = (uint64_t(b.y) << 32) | b.x;
+          c.size = ((uint64_t(a.w) << 32) | a.z) - c.base;
+          c.bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
           c.hit_word = (uint64_t(b.w) << 32) | b.z;
           c.t_alloc = d.x; c.t_free = d.y; c.r_lo = d.z; c.shift = d.w;
           c.obj = o;
@@ -176,13 +252,13 @@ __device__ __forceinline__ void process(const AttrParams& p, const uint64_t* s_l
   uint64_t key0 = kNoKey, key1 = kNoKey;
   uint32_t m0 = 0, m1 = 0;
   if (att) {
-    uint64_t end = addr + size;
-    if (end > c.end) { end = c.end; k.clip++; }
-    const uint64_t gb0 = c.bm_bit + ((addr - c.base) >> c.shift);
-    const uint64_t gb1 = c.bm_bit + ((end - 1 - c.base) >> c.shift);
+    uint64_t off_end = addr - c.base + size;   // no overflow: addr+size validated
+    if (off_end > c.size) { off_end = c.size; k.clip++; }
+    const uint64_t gb0 = c.bm_word * 32 + ((addr - c.base) >> c.shift);
+    const uint64_t gb1 = c.bm_word * 32 + ((off_end - 1) >> c.shift);
     const uint64_t w0 = gb0 >> 5, w1 = gb1 >> 5;
     if (w1 - w0 >= 2) {
-      enqueue_range(p, gb0, gb1, k);
+      enqueue_range(p.rq, p.rq_cap, p.ctr, p.orw, gb0, gb1, k.ovf);
     } else if (w1 == w0) {
       key0 = w0; m0 = bits_mask(gb0 & 31, gb1 & 31);
     } else {
@@ -192,7 +268,7 @@ __device__ __forceinline__ void process(const AttrParams& p, const uint64_t* s_l
   }
   warp_or_words(p.orw, key0, m0, lane);
   if (__any_sync(FULL_MASK, key1 != kNoKey)) warp_or_words(p.orw, key1, m1, lane);
-  // ---- A4: liveness fold
+  // ---- A4: liveness fold (skipped where this lane already knows it holds)
   const bool need_min = att && ts < c.first_known;
   if (__any_sync(FULL_MASK, need_min)) {
     bool tail;
@@ -224,43 +300,283 @@ __device__ __forceinline__ void process(const AttrParams& p, const uint64_t* s_l
       if (hkey == c.hw) c.hbits |= hm; else { c.hw = hkey; c.hbits = hm; }
     }
   }
+  // first/last/hit for (c.obj, ts, is_w) are now ensured by this lane
+  c.meta = att ? r.w : kNever;
 }
 
-constexpr int kAttrThreads = 256;
-constexpr int kAttrUnroll = 4;
+// ------------------------------------------------------------------ fast path
+// Preconditions (checked by the caller): every lane's cache holds the SAME
+// object (< 4 GiB) and the same (API, rw) whose first/last/hit work is done,
+// and every lane's record lies inside that object, unclipped, <= 2 words.
+// e0/e1 are element indices relative to the object; bm_word its first word.
+// Only the bitmap OR remains.
+__device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_t e0, uint32_t e1, int lane) {
+  // contiguous union: intervals chain (start within or right after the
+  // previous interval, monotone ends) -> union = [e0 of lane 0, e1 of lane 31]
+  const uint32_t pe0 = __shfl_up_sync(FULL_MASK, e0, 1);
+  const uint32_t pe1 = __shfl_up_sync(FULL_MASK, e1, 1);
+  const bool chain = lane == 0 || (e0 >= pe0 && e0 <= pe1 + 1 && e1 >= pe1);
+  if (__all_sync(FULL_MASK, chain)) {
+    const uint32_t lo = __shfl_sync(FULL_MASK, e0, 0);
+    const uint32_t hi = __shfl_sync(FULL_MASK, e1, 31);
+    const uint32_t wlo = lo >> 5, nw = (hi >> 5) - wlo;   // words wlo .. wlo+nw
+    uint32_t* base = orw + bm_word + wlo;
+    for (uint32_t w = lane; w <= nw; w += 32) {
+      uint32_t m = 0xFFFFFFFFu;
+      if (w == 0) m &= 0xFFFFFFFFu << (lo & 31);
+      if (w == nw) m &= 0xFFFFFFFFu >> (31 - (hi & 31));
+      atomicOr(base + w, m);
+    }
+    return;
+  }
+  const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
+  const bool two = w1 != w0;
+  warp_or_words(orw, bm_word + w0, two ? (0xFFFFFFFFu << (e0 & 31)) : bits_mask(e0 & 31, e1 & 31), lane);
+  if (__any_sync(FULL_MASK, two))
+    warp_or_words(orw, two ? bm_word + w1 : kNoKey, 0xFFFFFFFFu >> (31 - (e1 & 31)), lane);
+}
+
+// Affine tier: the warp's 128 consecutive records (4 tiles, lane l holds
+// records l, 32+l, 64+l, 96+l) are one constant-stride run of one size and one
+// (API, rw) inside the warp's cached object: addr_j = a0 + j*st.  This is
+// what warp-coalesced instrumentation emits for a[i] sweeps and strided
+// loops.  Validity, liveness, first/last and the hit bit are then settled by
+// the cache; when consecutive records overlap or touch adjacent elements
+// (st <= size or st <= elem_size) the union is ONE element range, written
+// with one RED.OR per word; otherwise each record ORs its own word(s).
+// Returns false (no side effect) when the precondition does not hold.
+__device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const LaneCache& c,
+                                           uint32_t* orw, int lane) {
+  const uint64_t my0 = (uint64_t(r[0].y) << 32) | r[0].x;
+  const uint64_t a0 = __shfl_sync(FULL_MASK, my0, 0);
+  const uint64_t st = __shfl_sync(FULL_MASK, my0, 1) - a0;
+  const uint32_t sz = __shfl_sync(FULL_MASK, r[0].z, 0);
+  bool ok = true;
+#pragma unroll
+  for (int k = 0; k < kTilesPerWarp; ++k) {
+    const uint64_t ak = (uint64_t(r[k].y) << 32) | r[k].x;
+    ok = ok && ak == a0 + uint64_t(32 * k + lane) * st && r[k].z == sz && r[k].w == c.meta;
+  }
+  if (!__all_sync(FULL_MASK, ok)) return 0;
+  // uniform from here on: every lane holds the same values
+  constexpr uint32_t kN = 32 * kTilesPerWarp;
+  const uint64_t off0 = a0 - c.base;
+  if (st == 0 || st >= (1ull << 32) || sz == 0 || off0 >= c.size) return 0;
+  const uint64_t off_end = off0 + uint64_t(kN - 1) * st + sz;       // one past the last byte
+  if (off_end > c.size) return 0;
+  const uint32_t o0 = uint32_t(off0);                                // c.size < 2^32 (uni)
+  const uint32_t st32 = uint32_t(st);
+  if (st32 <= sz || st32 <= (1u << c.shift)) {
+    const uint32_t lo = o0 >> c.shift, hi = uint32_t(off_end - 1) >> c.shift;
+    const uint32_t wlo = lo >> 5, nw = (hi >> 5) - wlo;
+    uint32_t* base = orw + c.bm_word + wlo;
+    for (uint32_t w = lane; w <= nw; w += 32) {
+      uint32_t m = 0xFFFFFFFFu;
+      if (w == 0) m &= 0xFFFFFFFFu << (lo & 31);
+      if (w == nw) m &= 0xFFFFFFFFu >> (31 - (hi & 31));
+      atomicOr(base + w, m);
+    }
+    return 1;
+  }
+  if (((sz - 1) >> c.shift) >= 32) return 0;   // records wider than a word: tile path
+#pragma unroll
+  for (int k = 0; k < kTilesPerWarp; ++k) {
+    const uint32_t off = o0 + (32 * k + lane) * st32;
+    const uint32_t e0 = off >> c.shift, e1 = (off + sz - 1) >> c.shift;
+    const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
+    const bool two = w1 != w0;
+    warp_or_words(orw, c.bm_word + w0, two ? (0xFFFFFFFFu << (e0 & 31)) : bits_mask(e0 & 31, e1 & 31), lane);
+    if (__any_sync(FULL_MASK, two))
+      warp_or_words(orw, two ? c.bm_word + w1 : kNoKey, 0xFFFFFFFFu >> (31 - (e1 & 31)), lane);
+  }
+  return 2;
+}
+
+// Warp-uniform slow path: all 32 records share one (API, rw) and land in one
+// object (the first tile of every burst).  One lane resolves the object and
+// folds first/last/hit once for the warp; the lanes adopt the object into
+// their caches.  Returns false (no side effect) when the precondition fails.
+__device__ __forceinline__ bool try_uniform_slow(const AttrParams& p, const uint64_t* s_l1, uint4 r,
+                                                 bool present, int lane, LaneCache& c, LaneCounts& k) {
+  const uint32_t meta = r.w;
+  const uint32_t meta0 = __shfl_sync(FULL_MASK, meta, 0);   // all lanes: never inside && / ||
+  if (!__all_sync(FULL_MASK, present && meta == meta0)) return false;
+  const uint32_t ts = meta & 0x7FFFFFFFu, is_w = meta >> 31;
+  if (ts >= p.n_api) return false;
+  const uint32_t rank = __ldg(p.acc_rank + ts);
+  if (rank == kNone) return false;
+  const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
+  uint32_t o = kNone;
+  if (lane == 0) o = find_object(p, s_l1, addr, ts);
+  o = __shfl_sync(FULL_MASK, o, 0);
+  if (o == kNone) return false;
+  const uint4* q = reinterpret_cast<const uint4*>(p.objs + o);
+  const uint4 a = __ldg(q), b = __ldg(q + 1), d = __ldg(q + 2);
+  if (ts >= d.y) return false;
+  const uint64_t base = (uint64_t(a.y) << 32) | a.x;
+  const uint64_t osz = ((uint64_t(a.w) << 32) | a.z) - base;
+  if (osz > 0xFFFFFFFFull) return false;
+  const uint64_t off = addr - base;
+  const uint32_t size = r.z;
+  const uint32_t off32 = uint32_t(off), e0 = off32 >> d.w, e1 = (off32 + size - 1) >> d.w;
+  const bool ok = off < osz && size != 0 && size <= uint32_t(osz) - off32 && (e1 >> 5) - (e0 >> 5) < 2;
+  if (!__all_sync(FULL_MASK, ok)) return false;
+  c.base = base; c.size = osz;
+  c.bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
+  c.hit_word = (uint64_t(b.w) << 32) | b.z;
+  c.t_alloc = d.x; c.t_free = d.y; c.r_lo = d.z; c.shift = d.w; c.obj = o;
+  c.ts = ts; c.rank = rank;
+  const uint32_t hb = 2 * (rank - d.z) + is_w;
+  c.hw = c.hit_word + (hb >> 5);
+  c.hbits = 1u << (hb & 31);
+  if (lane == 0) {
+    atomicMin(p.first + o, ts);
+    atomicMax(p.last + o, ts);
+    atomicOr(p.orw + c.hw, c.hbits);
+  }
+  c.first_known = ts; c.last_known = ts; c.meta = meta;
+  k.rec += 1; k.attr += 1;
+  fast_or(p.orw, c.bm_word, e0, e1, lane);
+  return true;
+}
 
 __global__ void __launch_bounds__(kAttrThreads, 2) attribute_kernel(const AttrParams p) {
-  __shared__ uint64_t s_l1[kL1MaxKeys];
+  extern __shared__ __align__(128) uint8_t smem[];
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  // per-warp ring: kStages slots of kWarpRecords records, one mbarrier and one
+  // record count per slot
+  uint4* ring = reinterpret_cast<uint4*>(smem) + size_t(warp) * kStages * kWarpRecords;
+  uint64_t* s_l1 = reinterpret_cast<uint64_t*>(smem + size_t(kConsumerWarps) * kStages * kWarpRecords * 16);
+  uint64_t* full = s_l1 + kL1MaxKeys + warp * kStages;
+  uint32_t* slot_cnt = reinterpret_cast<uint32_t*>(s_l1 + kL1MaxKeys + kConsumerWarps * kStages) + warp * kStages;
+
+  // Work distribution: warps take contiguous chunks of kChunkRecords records
+  // from a global cursor (dynamic, so slow warps do not set the kernel's end).
+  // Only lane 0 touches the fetch state.
+  const uint64_t policy = evict_first_policy();
+  uint64_t f_pos = 0, f_hi = 0;
+  auto fetch = [&](int s) {   // lane 0: fill slot s with the next <= 128 records, or mark the end
+    if (f_pos == f_hi) {
+      f_pos = atomicAdd(&p.ctr[C_WORK], (unsigned long long)kChunkRecords);
+      f_hi = min(f_pos + kChunkRecords, p.n);
+      if (f_pos >= p.n) f_pos = f_hi = p.n;
+    }
+    const uint32_t cnt = uint32_t(min(uint64_t(kWarpRecords), f_hi - f_pos));
+    slot_cnt[s] = cnt;
+    if (cnt) {
+      mbar_arrive_expect_tx(&full[s], cnt * 16);
+      tma_load_1d(ring + size_t(s) * kWarpRecords, p.recs + f_pos, cnt * 16, &full[s], policy);
+      f_pos += cnt;
+    } else {
+      mbar_arrive(&full[s]);   // end of work: complete the phase with cnt = 0
+    }
+  };
+
+  if (lane == 0) {
+    for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    for (int s = 0; s < kStages; ++s) fetch(s);
+  }
   for (uint32_t i = threadIdx.x; i < p.n_l1; i += blockDim.x) s_l1[i] = p.l1[i];
   __syncthreads();
-  const int lane = threadIdx.x & 31;
-  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+
   LaneCache c;
-  c.base = 1; c.end = 0; c.bm_bit = 0; c.hit_word = 0;
+  c.base = 0; c.size = 0; c.bm_word = 0; c.hit_word = 0;
   c.t_alloc = 0; c.t_free = 0; c.r_lo = 0; c.shift = 0; c.obj = kNone;
-  c.ts = kNone; c.rank = kNone; c.first_known = kNever; c.last_known = 0;
+  c.meta = kNever; c.ts = kNone; c.rank = kNone; c.first_known = kNever; c.last_known = 0;
   c.hw = kNoKey; c.hbits = 0;
   LaneCounts k = {0, 0, 0, 0, 0, 0};
-  constexpr uint64_t per_iter = 32 * kAttrUnroll;
-  for (uint64_t base = gwarp * per_iter; base < p.n; base += nwarps * per_iter) {
-    uint4 r[kAttrUnroll];
+  uint32_t fast_rec = 0;
+  uint32_t n_aff_u = 0, n_aff_w = 0, n_fast = 0, n_slow = 0;   // diagnostics (warp-uniform)
+  bool uni = false;  // warp-uniform: all lanes cache one object (< 4 GiB) and one (API, rw)
+  const uint32_t wfirst = 0;
+  for (uint32_t st = 0;; ++st) {
+    const int s = int(st % kStages);
+    mbar_wait(&full[s], (st / kStages) & 1);
+    const uint32_t cnt = slot_cnt[s];
+    if (cnt == 0) break;                                   // warp-uniform
+    const int ntiles = int((cnt + 31) / 32);
+    // copy the stage to registers (lane l: records l, 32+l, 64+l, 96+l) and refill the slot
+    const uint32_t sbuf = smem_u32(ring + size_t(s) * kWarpRecords) + lane * 16;
+    uint4 r4[kTilesPerWarp];
 #pragma unroll
-    for (int u = 0; u < kAttrUnroll; ++u) {
-      const uint64_t i = base + u * 32 + lane;
-      r[u] = i < p.n ? ld_stream(p.recs + i) : make_uint4(0, 0, 0, 0);
+    for (int t = 0; t < kTilesPerWarp; ++t)
+      r4[t] = t * 32 + lane < cnt ? lds128(sbuf + t * 512) : make_uint4(0, 0, 0, 0);
+    // The vote consumes every lane's loaded registers, so all of this warp's
+    // reads of the slot have completed before lane 0 refills it (no memory
+    // fence: that would also wait for this lane's outstanding global REDs).
+    uint32_t dep = 0;
+#pragma unroll
+    for (int t = 0; t < kTilesPerWarp; ++t) dep ^= r4[t].x ^ r4[t].w;
+    const bool never = __any_sync(FULL_MASK, dep == 0x9E3779B9u && lane == 32);
+    if (lane == 0 && !never) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      fetch(s);
     }
+    __syncwarp();
+    if (uni && ntiles == kTilesPerWarp) {
+      const int how = try_affine(r4, c, p.orw, lane);
+      if (how) {
+        fast_rec += kTilesPerWarp;
+        if (how == 1) n_aff_u += kTilesPerWarp; else n_aff_w += kTilesPerWarp;
+        continue;
+      }
+    }
+#pragma unroll 1
+    for (int t = 0; t < ntiles; ++t) {
+      const bool present = wfirst + t * 32 + lane < cnt;
+      uint4 r = r4[0];                       // register select, no local-memory indexing
 #pragma unroll
-    for (int u = 0; u < kAttrUnroll; ++u)
-      process(p, s_l1, r[u], base + u * 32 + lane < p.n, lane, c, k);
+      for (int j = 1; j < kTilesPerWarp; ++j) if (t == j) r = r4[j];
+      if (uni) {
+        // fast check in 32-bit object-relative arithmetic
+        const uint64_t off = ((uint64_t(r.y) << 32) | r.x) - c.base;
+        const uint32_t off32 = uint32_t(off), size = r.z, osz = uint32_t(c.size);
+        const uint32_t e0 = off32 >> c.shift;
+        const uint32_t e1 = (off32 + size - 1) >> c.shift;
+        const bool ok = present && r.w == c.meta && (off >> 32) == 0 && off32 < osz &&
+                        size != 0 && size <= osz - off32 && (e1 >> 5) - (e0 >> 5) < 2;
+        if (__all_sync(FULL_MASK, ok)) {
+          fast_or(p.orw, c.bm_word, e0, e1, lane);
+          ++fast_rec;
+          ++n_fast;
+          continue;
+        }
+      }
+      if (try_uniform_slow(p, s_l1, r, present, lane, c, k)) {
+        ++n_slow;
+        uni = true;
+        continue;
+      }
+      {  // rare: out of line, through copies so c and k stay in registers elsewhere
+        LaneCache c2 = c;
+        LaneCounts k2 = k;
+        process_slow(p, s_l1, r, present, lane, c2, k2);
+        c = c2;
+        k = k2;
+      }
+      ++n_slow;
+      const uint32_t m0 = __shfl_sync(FULL_MASK, c.meta, 0);
+      const uint32_t o0 = __shfl_sync(FULL_MASK, c.obj, 0);
+      uni = __all_sync(FULL_MASK, c.meta == m0 && c.obj == o0 && m0 != kNever && c.size <= 0xFFFFFFFFull);
+    }
+  }
+  k.rec += fast_rec;
+  k.attr += fast_rec;
+  if (lane == 0) {
+    atomicAdd(&p.ctr[C_TILES_AFFINE_UNION], (unsigned long long)n_aff_u);
+    atomicAdd(&p.ctr[C_TILES_AFFINE_WORDS], (unsigned long long)n_aff_w);
+    atomicAdd(&p.ctr[C_TILES_FAST], (unsigned long long)n_fast);
+    atomicAdd(&p.ctr[C_TILES_SLOW], (unsigned long long)n_slow);
   }
   // A5: warp-reduce the counters, one atomic per warp and counter
   const uint32_t v[6] = {k.rec, k.attr, k.unattr, k.clip, k.inval, k.ovf};
   const int slot[6] = {C_RECORDS, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID, C_RQ_OVERFLOW};
 #pragma unroll
   for (int i = 0; i < 6; ++i) {
-    const uint32_t s = __reduce_add_sync(FULL_MASK, v[i]);
-    if (lane == 0 && s) atomicAdd(&p.ctr[slot[i]], (unsigned long long)s);
+    const uint32_t sum = __reduce_add_sync(FULL_MASK, v[i]);
+    if (lane == 0 && sum) atomicAdd(&p.ctr[slot[i]], (unsigned long long)sum);
   }
 }
 
@@ -289,16 +605,19 @@ __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
 int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s) {
   if (p.n == 0) return 0;
   cudaMemsetAsync(p.ctr + C_RQ_COUNT, 0, sizeof(unsigned long long), s);
+  cudaMemsetAsync(p.ctr + C_WORK, 0, sizeof(unsigned long long), s);
   static int occ = 0;
   if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, attribute_kernel, kAttrThreads, 0);
+    cudaFuncSetAttribute(attribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kAttrSmem));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, attribute_kernel, kAttrThreads, kAttrSmem);
     if (occ < 1) occ = 1;
   }
-  const uint64_t per_block = uint64_t(kAttrThreads / 32) * 32 * kAttrUnroll;
-  uint64_t blocks = (p.n + per_block - 1) / per_block;
+  // enough stages per block to keep the ring busy, at most one wave
+  uint64_t blocks = (p.n + 4ull * kConsumerWarps * kWarpRecords - 1) / (4ull * kConsumerWarps * kWarpRecords);
   const uint64_t full = uint64_t(num_sms) * occ;
   if (blocks > full) blocks = full;
-  attribute_kernel<<<(unsigned)blocks, kAttrThreads, 0, s>>>(p);
+  if (blocks < 1) blocks = 1;
+  attribute_kernel<<<(unsigned)blocks, kAttrThreads, kAttrSmem, s>>>(p);
   range_expand_kernel<<<num_sms * 4, 256, 0, s>>>(p.rq, p.ctr, p.rq_cap, p.orw);
   return 2;
 }

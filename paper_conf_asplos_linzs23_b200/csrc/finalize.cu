@@ -51,8 +51,8 @@ __device__ __forceinline__ M32 m32_cat(const M32& a, const M32& b) {
   r.pop = a.pop + b.pop;
   r.lo = a.pop ? a.lo : (b.pop ? a.len + b.lo : kNoPos32);
   r.hi = b.pop ? a.len + b.hi : a.hi;
-  r.pre = a.pop ? a.pre : a.len + b.pre;
-  r.suf = b.pop ? b.suf : b.len + a.suf;
+  r.pre = a.pre == a.len ? a.len + b.pre : a.pre;   // a has no 1 in the run view
+  r.suf = b.suf == b.len ? b.len + a.suf : b.suf;
   r.best = max(max(a.best, b.best), a.suf + b.pre);
   return r;
 }
@@ -72,8 +72,8 @@ __device__ __forceinline__ BitMonoid bm_cat(const BitMonoid& a, const BitMonoid&
   r.pop = a.pop + b.pop;
   r.lo = a.pop ? a.lo : (b.pop ? a.len + b.lo : kNoPos);
   r.hi = b.pop ? a.len + b.hi : a.hi;
-  r.pre = a.pop ? a.pre : a.len + b.pre;
-  r.suf = b.pop ? b.suf : b.len + a.suf;
+  r.pre = a.pre == a.len ? a.len + b.pre : a.pre;   // a has no 1 in the run view
+  r.suf = b.suf == b.len ? b.len + a.suf : b.suf;
   r.best = max(max(a.best, b.best), a.suf + b.pre);
   return r;
 }
@@ -85,62 +85,118 @@ __device__ __forceinline__ BitMonoid bm_shfl_down(const BitMonoid& m, int d) {
                    __shfl_down_sync(FULL_MASK, m.best, d)};
 }
 
-// B4: one warp per tile.  Each step covers 128 words (lane l: words 4l..4l+3
-// via one 16-B load; object bitmaps and tiles start 4-word aligned).
+// B4: one warp per tile (<= kTileWords = 1024 words of one object), read with
+// eight coalesced 16-B loads per lane issued up front.  Each 128-word block
+// (lane l holds words 4l..4l+3) is reduced without shuffle trees: lane runs
+// by sequential folds, then popcount by REDUX.SUM, lowest/highest accessed
+// bit by ballot + one shuffle, and the longest zero run by joining every
+// lane's leading zeros to the trailing zeros of the previous non-empty lane
+// (ballot + one indexed shuffle + REDUX.MAX).  Bits past the object's last
+// element are treated as 1 ("sentinels") for the run view so no zero run
+// extends past n_elems; they never count as accessed.
 __global__ void __launch_bounds__(256) tile_reduce_kernel(const uint32_t* __restrict__ orw,
     const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out) {
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  constexpr int kBlocks = kTileWords / 128;
   for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
     const Tile tl = tiles[t];
-    M32 acc = m32_identity();  // meaningful in lane 0
-    for (uint32_t w0 = 0; w0 < tl.n_words; w0 += 128) {
-      const uint32_t my = w0 + 4 * lane;
-      uint4 v = make_uint4(0, 0, 0, 0);
-      if (my < tl.n_words) v = *reinterpret_cast<const uint4*>(orw + tl.word_lo + my);
-      // bits of this tile covered by word j: clamp(n_bits - 32*j, 0, 32)
-      const uint64_t bit0 = uint64_t(my) * 32;
-      const bool in = my < tl.n_words;
-      const bool zero = (v.x | v.y | v.z | v.w) == 0;
-      const bool ones = (v.x & v.y & v.z & v.w) == 0xFFFFFFFFu;
-      const uint64_t chunk_bits = 128ull * 32;
-      const bool full_chunk = uint64_t(w0) * 32 + chunk_bits <= tl.n_bits;
-      M32 m;
-      if (full_chunk && __all_sync(FULL_MASK, zero)) {
-        m = M32{4096, 0, kNoPos32, kNoPos32, 4096, 4096, 4096};
-        if (lane == 0) acc = m32_cat(acc, m);
-        continue;
-      }
-      if (full_chunk && __all_sync(FULL_MASK, ones)) {
-        m = M32{4096, 4096, 0, 4095, 0, 0, 0};
-        if (lane == 0) acc = m32_cat(acc, m);
-        continue;
-      }
-      auto nv = [&](uint64_t b) -> uint32_t {
-        if (!in || b >= tl.n_bits) return 0;
-        const uint64_t r = tl.n_bits - b;
-        return r >= 32 ? 32u : uint32_t(r);
-      };
-      m = m32_word(v.x, nv(bit0));
-      m = m32_cat(m, m32_word(v.y, nv(bit0 + 32)));
-      m = m32_cat(m, m32_word(v.z, nv(bit0 + 64)));
-      m = m32_cat(m, m32_word(v.w, nv(bit0 + 96)));
+    const uint32_t nbits = uint32_t(tl.n_bits);
+    uint4 v[kBlocks];
 #pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const M32 o = m32_shfl_down(m, d);
-        m = m32_cat(m, o);
+    for (int b = 0; b < kBlocks; ++b) {
+      const uint32_t w = b * 128 + 4 * lane;
+      v[b] = w < tl.n_words ? __ldg(reinterpret_cast<const uint4*>(orw + tl.word_lo + w))
+                            : make_uint4(0, 0, 0, 0);
+    }
+    M32 acc = m32_identity();   // identical in every lane
+#pragma unroll
+    for (int b = 0; b < kBlocks; ++b) {
+      const uint32_t wb = b * 128 + 4 * lane;   // tile-relative word of v[b].x
+      uint32_t real[4] = {v[b].x, v[b].y, v[b].z, v[b].w};
+      uint32_t run[4] = {v[b].x, v[b].y, v[b].z, v[b].w};
+      if (uint32_t(b + 1) * 128 * 32 > nbits) {   // block reaches past the tile's last bit
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t bj = (wb + j) * 32;
+          const uint32_t nv = bj >= nbits ? 0u : min(32u, nbits - bj);
+          const uint32_t vm = nv == 32 ? 0xFFFFFFFFu : ((1u << nv) - 1u);
+          real[j] &= vm;
+          run[j] = real[j] | ~vm;
+        }
       }
-      if (lane == 0) acc = m32_cat(acc, m);
+      // lane: real popcount / first / last accessed bit; run-view fold
+      uint32_t pop = 0, lo = kNoPos32, hi = kNoPos32;
+      M32 r = m32_identity();
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        pop += __popc(real[j]);
+        if (real[j]) {
+          if (lo == kNoPos32) lo = 32 * j + __ffs(real[j]) - 1;
+          hi = 32 * j + 31 - __clz(real[j]);
+        }
+        r = m32_cat(r, m32_word(run[j], 32));
+      }
+      // block (128 words): combine the 32 lanes in order
+      M32 blk;
+      blk.len = 4096;
+      blk.pop = __reduce_add_sync(FULL_MASK, pop);
+      const uint32_t nzp = __ballot_sync(FULL_MASK, pop != 0);
+      if (nzp) {
+        const int fl = __ffs(nzp) - 1, ll = 31 - __clz(nzp);
+        blk.lo = 128 * fl + __shfl_sync(FULL_MASK, lo, fl);
+        blk.hi = 128 * ll + __shfl_sync(FULL_MASK, hi, ll);
+      } else {
+        __shfl_sync(FULL_MASK, lo, 0);   // keep the shuffles convergent
+        __shfl_sync(FULL_MASK, hi, 0);
+        blk.lo = blk.hi = kNoPos32;
+      }
+      const uint32_t nz = __ballot_sync(FULL_MASK, r.pop != 0);   // lanes with a 1 in the run view
+      const uint32_t below = nz & ((1u << lane) - 1u);
+      const int i = below ? 31 - __clz(below) : -1;
+      const uint32_t suf_i = __shfl_sync(FULL_MASK, r.suf, i < 0 ? 0 : i);
+      const uint32_t run_j = (i < 0 ? 0u : suf_i + 128u * uint32_t(lane - i - 1)) +
+                             (i < 0 ? 128u * lane : 0u) + r.pre;
+      const uint32_t cand = r.pop ? max(r.best, run_j) : 0u;
+      uint32_t best = __reduce_max_sync(FULL_MASK, cand);
+      if (nz == 0) {
+        blk.pre = blk.suf = blk.best = 4096;
+        __shfl_sync(FULL_MASK, r.pre, 0);
+        __shfl_sync(FULL_MASK, r.suf, 0);
+      } else {
+        const int f = __ffs(nz) - 1, l = 31 - __clz(nz);
+        blk.pre = 128 * f + __shfl_sync(FULL_MASK, r.pre, f);
+        blk.suf = 128 * (31 - l) + __shfl_sync(FULL_MASK, r.suf, l);
+        blk.best = max(best, blk.suf);
+      }
+      acc = m32_cat(acc, blk);
     }
     if (lane == 0) {
       BitMonoid r;
-      r.len = acc.len; r.pop = acc.pop;
+      r.len = acc.len;   // run-view length (sentinel bits only after an object's end)
+      r.pop = acc.pop;
       r.lo = acc.lo == kNoPos32 ? kNoPos : acc.lo;
       r.hi = acc.hi == kNoPos32 ? kNoPos : acc.hi;
       r.pre = acc.pre; r.suf = acc.suf; r.best = acc.best;
       out[t] = r;
     }
+  }
+}
+
+// B4b: one warp per group (<= 32 consecutive tiles of one object): ordered
+// shuffle tree over the tile monoids.
+__global__ void __launch_bounds__(256) group_reduce_kernel(const Group* __restrict__ groups,
+    uint64_t n_groups, const BitMonoid* __restrict__ tile_part, BitMonoid* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  for (uint64_t g = gwarp; g < n_groups; g += nwarps) {
+    const Group gr = groups[g];
+    BitMonoid m = uint32_t(lane) < gr.n_tiles ? tile_part[gr.tile_lo + lane] : bm_identity();
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) m = bm_cat(m, bm_shfl_down(m, d));
+    if (lane == 0) out[g] = m;
   }
 }
 
@@ -193,11 +249,11 @@ __global__ void __launch_bounds__(256) object_finalize_kernel(const FinalParams 
   drgpum_object_stats_t* stats = static_cast<drgpum_object_stats_t*>(p.stats);
   drgpum_pattern_report_t* reps = static_cast<drgpum_pattern_report_t*>(p.reports);
   for (uint64_t o = gwarp; o < p.n_obj; o += nwarps) {
-    // ---- bitmap tiles of o, in order
-    const uint32_t t0 = p.tile_off[o], t1 = p.tile_off[o + 1];
+    // ---- bitmap groups of o, in order
+    const uint32_t t0 = p.group_off[o], t1 = p.group_off[o + 1];
     BitMonoid bm = bm_identity();
     for (uint32_t tb = t0; tb < t1; tb += 32) {
-      BitMonoid m = (tb + lane < t1) ? p.tile_part[tb + lane] : bm_identity();
+      BitMonoid m = (tb + lane < t1) ? p.group_part[tb + lane] : bm_identity();
 #pragma unroll
       for (int d = 1; d < 32; d <<= 1) m = bm_cat(m, bm_shfl_down(m, d));
       if (lane == 0) bm = bm_cat(bm, m);
@@ -246,7 +302,7 @@ __global__ void __launch_bounds__(256) object_finalize_kernel(const FinalParams 
     stats[o] = st;
     // cross-check of the two liveness folds (atomics vs hit rows), and of
     // bitmap vs hit row (an object with accessed elements has accessing APIs)
-    const bool consistent = bm.len == n &&
+    const bool consistent = bm.len >= n && (bm.pop == 0 || bm.hi < n) &&
         (hm.cnt ? (first == hm.first_ts && last == hm.last_ts && bm.pop > 0)
                 : (first == kNever && last == 0 && bm.pop == 0));
     if (!consistent) atomicAdd(&p.ctr[C_CONSISTENCY], 1ull);
@@ -282,10 +338,13 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   const uint64_t tb = (p.n_tiles + 7) / 8;
   const unsigned g1 = (unsigned)(tb < uint64_t(num_sms) * 16 ? tb : uint64_t(num_sms) * 16);
   tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles, p.n_tiles, p.tile_part);
+  const uint64_t gb = (p.n_groups + 7) / 8;
+  const unsigned g3 = (unsigned)(gb < uint64_t(num_sms) * 16 ? gb : uint64_t(num_sms) * 16);
+  group_reduce_kernel<<<g3 ? g3 : 1, 256, 0, s>>>(p.groups, p.n_groups, p.tile_part, p.group_part);
   const uint64_t ob = (p.n_obj + 7) / 8;
   const unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
   object_finalize_kernel<<<g2, 256, 0, s>>>(p);
-  return 2;
+  return 3;
 }
 
 // ---------------------------------------------------------------- utilities

@@ -34,7 +34,7 @@ struct Layout {
   uint64_t orw, first, last, ctr;           // dynamic (reset per trace)
   uint64_t dyn_end;
   uint64_t objs, seg_start, seg_cand_off, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
-  uint64_t tiles, tile_off, tile_part, stats, reports, rq, stage;
+  uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage;
   uint64_t total;
 };
 
@@ -64,6 +64,8 @@ struct drgpum_ctx {
   std::vector<uint8_t> acc_cs;
   std::vector<Tile> tiles;
   std::vector<uint32_t> tile_off;
+  std::vector<Group> groups;
+  std::vector<uint32_t> group_off;
   std::vector<drgpum_object_layout_t> layout;
   uint64_t bitmap_words = 0, hit_words = 0;
   uint32_t rq_cap = 1u << 20;
@@ -210,6 +212,14 @@ drgpum_status build_tables(drgpum_ctx* c) {
   }
   if (c->tiles.size() >= 0xFFFFFFFFull) return fail(c, DRGPUM_ENOMEM, "too many reduction tiles");
   c->tile_off[n] = (uint32_t)c->tiles.size();
+  c->groups.clear();
+  c->group_off.assign(n + 1, 0);
+  for (uint64_t i = 0; i < n; ++i) {
+    c->group_off[i] = (uint32_t)c->groups.size();
+    for (uint32_t t = c->tile_off[i]; t < c->tile_off[i + 1]; t += kGroupTiles)
+      c->groups.push_back(Group{t, std::min<uint32_t>(kGroupTiles, c->tile_off[i + 1] - t)});
+  }
+  c->group_off[n] = (uint32_t)c->groups.size();
   c->bitmap_words = bw;
   uint64_t hw = 0;
   for (uint64_t i = 0; i < n; ++i) {
@@ -253,8 +263,10 @@ drgpum_status build_tables(drgpum_ctx* c) {
   L.acc_cs = put(c->n_acc);
   L.n_hit = put(4 * n);
   L.tiles = put(sizeof(Tile) * c->tiles.size());
-  L.tile_off = put(4 * (n + 1));
   L.tile_part = put(sizeof(BitMonoid) * c->tiles.size());
+  L.groups = put(sizeof(Group) * c->groups.size());
+  L.group_off = put(4 * (n + 1));
+  L.group_part = put(sizeof(BitMonoid) * c->groups.size());
   L.stats = put(sizeof(drgpum_object_stats_t) * n);
   L.reports = put(sizeof(drgpum_pattern_report_t) * n);
   L.rq = put(sizeof(RangeEntry) * c->rq_cap);
@@ -354,6 +366,7 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   ctx->cand.swap(tmp.cand); ctx->l1.swap(tmp.l1); ctx->l1_stride = tmp.l1_stride;
   ctx->acc_rank.swap(tmp.acc_rank); ctx->acc_ts.swap(tmp.acc_ts); ctx->acc_cs.swap(tmp.acc_cs);
   ctx->n_hit.swap(tmp.n_hit); ctx->tiles.swap(tmp.tiles); ctx->tile_off.swap(tmp.tile_off);
+  ctx->groups.swap(tmp.groups); ctx->group_off.swap(tmp.group_off);
   ctx->layout.swap(tmp.layout);
   ctx->bitmap_words = tmp.bitmap_words; ctx->hit_words = tmp.hit_words;
   ctx->L = tmp.L;
@@ -402,7 +415,8 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
   if ((r = up(L.acc_cs, ctx->acc_cs.data(), ctx->acc_cs.size()))) return r;
   if ((r = up(L.n_hit, ctx->n_hit.data(), 4 * n))) return r;
   if ((r = up(L.tiles, ctx->tiles.data(), sizeof(Tile) * ctx->tiles.size()))) return r;
-  if ((r = up(L.tile_off, ctx->tile_off.data(), 4 * ctx->tile_off.size()))) return r;
+  if ((r = up(L.groups, ctx->groups.data(), sizeof(Group) * ctx->groups.size()))) return r;
+  if ((r = up(L.group_off, ctx->group_off.data(), 4 * ctx->group_off.size()))) return r;
   if ((r = enqueue_reset(ctx, st))) return r;
   // host vectors stay alive in ctx, so the async uploads are safe; make the
   // bind synchronous anyway so callers may immediately reuse their stream
@@ -522,7 +536,10 @@ DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_threshold
   p.tiles = at<Tile>(ctx, ctx->L.tiles);
   p.tile_part = at<BitMonoid>(ctx, ctx->L.tile_part);
   p.n_tiles = ctx->tiles.size();
-  p.tile_off = at<uint32_t>(ctx, ctx->L.tile_off);
+  p.groups = at<Group>(ctx, ctx->L.groups);
+  p.group_part = at<BitMonoid>(ctx, ctx->L.group_part);
+  p.n_groups = ctx->groups.size();
+  p.group_off = at<uint32_t>(ctx, ctx->L.group_off);
   p.objs = at<DevObj>(ctx, ctx->L.objs);
   p.first = at<uint32_t>(ctx, ctx->L.first);
   p.last = at<uint32_t>(ctx, ctx->L.last);
@@ -598,6 +615,20 @@ DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx* ctx, uint64_t* h_
   CK(cudaMemcpyAsync(c, ctx->ws + ctx->L.ctr, sizeof c, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   *h_errors = c[C_CONSISTENCY];
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_path_stats(drgpum_ctx* ctx, uint64_t out[4], void* stream) {
+  if (!ctx || !out) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return DRGPUM_ESTATE;
+  cudaStream_t st = as_stream(stream);
+  unsigned long long c[C_SLOTS];
+  CK(cudaMemcpyAsync(c, ctx->ws + ctx->L.ctr, sizeof c, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  out[0] = c[C_TILES_AFFINE_UNION];
+  out[1] = c[C_TILES_AFFINE_WORDS];
+  out[2] = c[C_TILES_FAST];
+  out[3] = c[C_TILES_SLOW];
   return DRGPUM_OK;
 }
 

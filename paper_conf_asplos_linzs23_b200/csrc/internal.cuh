@@ -10,7 +10,8 @@ constexpr uint32_t kNever = 0xFFFFFFFFu;
 constexpr uint32_t kNone = 0xFFFFFFFFu;        // "no object" / invalid rank
 constexpr int kL1MaxKeys = 2048;               // level-1 keys staged in shared memory (16 KB)
 constexpr uint32_t kRangeChunkWords = 4096;    // range-expansion work item (16 KB of bitmap)
-constexpr uint32_t kTileWords = 8192;          // bitmap reduction tile (32 KB)
+constexpr uint32_t kTileWords = 1024;          // bitmap reduction tile (4 KB)
+constexpr uint32_t kGroupTiles = 32;           // tiles per reduction group
 constexpr uint64_t kStageRecords = 1ull << 22; // host-ingest staging chunk (64 MB)
 
 // Object as the attribution kernel sees it: 48 bytes, three 16-B loads.
@@ -33,6 +34,8 @@ struct RangeEntry { uint64_t bit_lo, bit_hi; };
 
 // Bitmap reduction tile: a run of <= kTileWords words of ONE object.
 struct Tile { uint64_t word_lo; uint32_t n_words; uint32_t obj; uint64_t elem_lo; uint64_t n_bits; };
+// Reduction group: <= kGroupTiles consecutive tiles of ONE object.
+struct Group { uint32_t tile_lo, n_tiles; };
 
 // Bitmap run monoid over a bit sequence.  Positions are
 // relative to the start of the sequence; kNoPos when the sequence has no 1.
@@ -43,7 +46,11 @@ struct BitMonoid {
 
 // Counter slots (u64) at the start of the counters block.
 enum : int { C_RECORDS = 0, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID,
-             C_RQ_OVERFLOW, C_CONSISTENCY, C_RQ_COUNT, C_SLOTS = 16 };
+             C_RQ_OVERFLOW, C_CONSISTENCY, C_RQ_COUNT,
+             // diagnostics: 32-record tiles by attribution path
+             C_TILES_AFFINE_UNION, C_TILES_AFFINE_WORDS, C_TILES_FAST, C_TILES_SLOW,
+             C_WORK,   // attribution work cursor (records handed out)
+             C_SLOTS = 16 };
 
 struct AttrParams {
   const uint4* recs;
@@ -68,7 +75,10 @@ struct FinalParams {
   const Tile* tiles;
   BitMonoid* tile_part;
   uint64_t n_tiles;
-  const uint32_t* tile_off;  // [n_obj+1]
+  const Group* groups;
+  BitMonoid* group_part;
+  uint64_t n_groups;
+  const uint32_t* group_off;  // [n_obj+1]
   const DevObj* objs;
   const uint32_t* first;
   const uint32_t* last;

@@ -134,6 +134,12 @@ class Session:
                                                         _stream_handle(stream)))
         return int(e.value)
 
+    def path_stats(self, stream=None):
+        """Diagnostics: 32-record tiles per attribution path since the last reset."""
+        out = np.zeros(4, dtype=np.uint64)
+        check(self._h, self.L.drgpum_path_stats(self._h, _np_ptr(out), _stream_handle(stream)))
+        return dict(zip(("affine_union", "affine_words", "tile_fast", "slow"), (int(x) for x in out)))
+
     def layout(self):
         out = np.zeros(self.n_obj, dtype=LAYOUT_DTYPE)
         check(self._h, self.L.drgpum_object_layout(self._h, _np_ptr(out)))
