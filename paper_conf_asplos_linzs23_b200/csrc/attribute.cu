@@ -98,6 +98,18 @@ __device__ __forceinline__ uint32_t bits_mask(uint32_t b0, uint32_t b1) {  // bi
   return (0xFFFFFFFFu >> (31 - b1)) & (0xFFFFFFFFu << b0);
 }
 
+// Fire-and-forget global reductions (SASS REDG): OR/MIN/MAX are idempotent and
+// commutative, results are only read after the kernel, so relaxed gpu scope.
+__device__ __forceinline__ void red_or(uint32_t* a, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_min(uint32_t* a, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.min.u32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_max(uint32_t* a, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.max.u32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
+}
+
 // ------------------------------------------------------------------ warp helpers
 // Warp segmented inclusive scan over runs of adjacent lanes with equal keys.
 // Returns the run-reduced value in the run's last lane (tail = true there).
@@ -129,16 +141,16 @@ __device__ __forceinline__ void warp_or_words(uint32_t* words, uint64_t key, uin
   const uint32_t heads = __ballot_sync(FULL_MASK, lane == 0 || pk != key);
   if (heads == 1u) {  // one word for the whole warp
     const uint32_t v = __reduce_or_sync(FULL_MASK, m);
-    if (lane == 0 && key != kNoKey && v) atomicOr(words + key, v);
+    if (lane == 0 && key != kNoKey && v) red_or(words + key, v);
     return;
   }
   if (__popc(heads) > 16) {  // mostly distinct words: OR is idempotent, just RED
-    if (key != kNoKey && m) atomicOr(words + key, m);
+    if (key != kNoKey && m) red_or(words + key, m);
     return;
   }
   bool tail;
   const uint32_t v = seg_scan(key, m, lane, tail, OpOr());
-  if (tail && key != kNoKey && v) atomicOr(words + key, v);
+  if (tail && key != kNoKey && v) red_or(words + key, v);
 }
 
 // ------------------------------------------------------------------ lane state
@@ -201,7 +213,7 @@ __device__ __noinline__ void enqueue_range(RangeEntry* rq, uint32_t rq_cap, unsi
         uint32_t m = 0xFFFFFFFFu;
         if (w == (bl >> 5)) m &= 0xFFFFFFFFu << (bl & 31);
         if (w == (bh >> 5)) m &= 0xFFFFFFFFu >> (31 - (bh & 31));
-        atomicOr(orw + w, m);
+        red_or(orw + w, m);
       }
     }
   }
@@ -274,7 +286,7 @@ __device__ __noinline__ void process_slow(const AttrParams& p, const uint64_t* s
     bool tail;
     const uint64_t key = need_min ? c.obj : kNoKey;
     const uint32_t v = seg_scan(key, ts, lane, tail, OpMin());
-    if (tail && need_min) atomicMin(p.first + c.obj, v);
+    if (tail && need_min) red_min(p.first + c.obj, v);
     if (need_min) c.first_known = ts;
   }
   const bool need_max = att && ts > c.last_known;
@@ -282,7 +294,7 @@ __device__ __noinline__ void process_slow(const AttrParams& p, const uint64_t* s
     bool tail;
     const uint64_t key = need_max ? c.obj : kNoKey;
     const uint32_t v = seg_scan(key, ts, lane, tail, OpMax());
-    if (tail && need_max) atomicMax(p.last + c.obj, v);
+    if (tail && need_max) red_max(p.last + c.obj, v);
     if (need_max) c.last_known = ts;
   }
   // hit row: bit 2*(rank - r_lo) + is_write of the object's row
@@ -325,7 +337,7 @@ __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_
       uint32_t m = 0xFFFFFFFFu;
       if (w == 0) m &= 0xFFFFFFFFu << (lo & 31);
       if (w == nw) m &= 0xFFFFFFFFu >> (31 - (hi & 31));
-      atomicOr(base + w, m);
+      red_or(base + w, m);
     }
     return;
   }
@@ -347,25 +359,33 @@ __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_
 // Returns false (no side effect) when the precondition does not hold.
 __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const LaneCache& c,
                                            uint32_t* orw, int lane) {
-  const uint64_t my0 = (uint64_t(r[0].y) << 32) | r[0].x;
-  const uint64_t a0 = __shfl_sync(FULL_MASK, my0, 0);
-  const uint64_t st = __shfl_sync(FULL_MASK, my0, 1) - a0;
+  // predicted record j = 32k + lane: {lo(a0) + j*st, hi(a0), sz, meta}; the
+  // mismatch bits of all four words of all records are ORed with 3-input
+  // LOP3s (about 5 instructions per record)
+  const uint32_t a0lo = __shfl_sync(FULL_MASK, r[0].x, 0);
+  const uint32_t a0hi = __shfl_sync(FULL_MASK, r[0].y, 0);
+  const uint32_t st32 = __shfl_sync(FULL_MASK, r[0].x, 1) - a0lo;
   const uint32_t sz = __shfl_sync(FULL_MASK, r[0].z, 0);
-  bool ok = true;
+  uint32_t exp = a0lo + uint32_t(lane) * st32;
+  uint32_t bad = 0;
 #pragma unroll
   for (int k = 0; k < kTilesPerWarp; ++k) {
-    const uint64_t ak = (uint64_t(r[k].y) << 32) | r[k].x;
-    ok = ok && ak == a0 + uint64_t(32 * k + lane) * st && r[k].z == sz && r[k].w == c.meta;
+    bad |= (r[k].x ^ exp) | (r[k].y ^ a0hi);
+    bad |= (r[k].z ^ sz) | (r[k].w ^ c.meta);
+    exp += 32u * st32;
   }
-  if (!__all_sync(FULL_MASK, ok)) return 0;
+  if (!__all_sync(FULL_MASK, bad == 0)) return 0;
   // uniform from here on: every lane holds the same values
   constexpr uint32_t kN = 32 * kTilesPerWarp;
+  // the prediction is exact only if the low word never wrapped: then record j
+  // is at a0 + j*st in 64 bits
+  const uint64_t a0 = (uint64_t(a0hi) << 32) | a0lo;
+  if (st32 == 0 || sz == 0 || uint64_t(a0lo) + uint64_t(kN - 1) * st32 + sz > (1ull << 32)) return 0;
   const uint64_t off0 = a0 - c.base;
-  if (st == 0 || st >= (1ull << 32) || sz == 0 || off0 >= c.size) return 0;
-  const uint64_t off_end = off0 + uint64_t(kN - 1) * st + sz;       // one past the last byte
+  if (off0 >= c.size) return 0;
+  const uint64_t off_end = off0 + uint64_t(kN - 1) * st32 + sz;     // one past the last byte
   if (off_end > c.size) return 0;
   const uint32_t o0 = uint32_t(off0);                                // c.size < 2^32 (uni)
-  const uint32_t st32 = uint32_t(st);
   if (st32 <= sz || st32 <= (1u << c.shift)) {
     const uint32_t lo = o0 >> c.shift, hi = uint32_t(off_end - 1) >> c.shift;
     const uint32_t wlo = lo >> 5, nw = (hi >> 5) - wlo;
@@ -374,11 +394,27 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
       uint32_t m = 0xFFFFFFFFu;
       if (w == 0) m &= 0xFFFFFFFFu << (lo & 31);
       if (w == nw) m &= 0xFFFFFFFFu >> (31 - (hi & 31));
-      atomicOr(base + w, m);
+      red_or(base + w, m);
     }
     return 1;
   }
   if (((sz - 1) >> c.shift) >= 32) return 0;   // records wider than a word: tile path
+  if ((st32 >> c.shift) >= 32) {
+    // stride >= 32 elements: every record owns its word(s), nothing to merge
+#pragma unroll
+    for (int k = 0; k < kTilesPerWarp; ++k) {
+      const uint32_t off = o0 + (32 * k + lane) * st32;
+      const uint32_t e0 = off >> c.shift, e1 = (off + sz - 1) >> c.shift;
+      const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
+      if (w1 == w0) {
+        red_or(orw + c.bm_word + w0, bits_mask(e0 & 31, e1 & 31));
+      } else {
+        red_or(orw + c.bm_word + w0, 0xFFFFFFFFu << (e0 & 31));
+        red_or(orw + c.bm_word + w1, 0xFFFFFFFFu >> (31 - (e1 & 31)));
+      }
+    }
+    return 2;
+  }
 #pragma unroll
   for (int k = 0; k < kTilesPerWarp; ++k) {
     const uint32_t off = o0 + (32 * k + lane) * st32;
@@ -430,9 +466,9 @@ __device__ __forceinline__ bool try_uniform_slow(const AttrParams& p, const uint
   c.hw = c.hit_word + (hb >> 5);
   c.hbits = 1u << (hb & 31);
   if (lane == 0) {
-    atomicMin(p.first + o, ts);
-    atomicMax(p.last + o, ts);
-    atomicOr(p.orw + c.hw, c.hbits);
+    red_min(p.first + o, ts);
+    red_max(p.last + o, ts);
+    red_or(p.orw + c.hw, c.hbits);
   }
   c.first_known = ts; c.last_known = ts; c.meta = meta;
   k.rec += 1; k.attr += 1;
@@ -500,9 +536,14 @@ __global__ void __launch_bounds__(kAttrThreads, 2) attribute_kernel(const AttrPa
     // copy the stage to registers (lane l: records l, 32+l, 64+l, 96+l) and refill the slot
     const uint32_t sbuf = smem_u32(ring + size_t(s) * kWarpRecords) + lane * 16;
     uint4 r4[kTilesPerWarp];
+    if (cnt == kWarpRecords) {                             // full stage (all but a chunk's tail)
 #pragma unroll
-    for (int t = 0; t < kTilesPerWarp; ++t)
-      r4[t] = t * 32 + lane < cnt ? lds128(sbuf + t * 512) : make_uint4(0, 0, 0, 0);
+      for (int t = 0; t < kTilesPerWarp; ++t) r4[t] = lds128(sbuf + t * 512);
+    } else {
+#pragma unroll
+      for (int t = 0; t < kTilesPerWarp; ++t)
+        r4[t] = t * 32 + lane < cnt ? lds128(sbuf + t * 512) : make_uint4(0, 0, 0, 0);
+    }
     // The vote consumes every lane's loaded registers, so all of this warp's
     // reads of the slot have completed before lane 0 refills it (no memory
     // fence: that would also wait for this lane's outstanding global REDs).
@@ -597,7 +638,7 @@ __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
       uint32_t m = 0xFFFFFFFFu;
       if (w == w0) m &= 0xFFFFFFFFu << (r.bit_lo & 31);
       if (w == w1) m &= 0xFFFFFFFFu >> (31 - (r.bit_hi & 31));
-      if (m == 0xFFFFFFFFu) orw[w] = m; else atomicOr(orw + w, m);
+      if (m == 0xFFFFFFFFu) orw[w] = m; else red_or(orw + w, m);
     }
   }
 }

@@ -8,7 +8,7 @@ namespace drgpum {
 
 constexpr uint32_t kNever = 0xFFFFFFFFu;
 constexpr uint32_t kNone = 0xFFFFFFFFu;        // "no object" / invalid rank
-constexpr int kL1MaxKeys = 2048;               // level-1 keys staged in shared memory (16 KB)
+constexpr int kL1MaxKeys = 512;                // level-1 keys staged in shared memory (4 KB)
 constexpr uint32_t kRangeChunkWords = 4096;    // range-expansion work item (16 KB of bitmap)
 constexpr uint32_t kTileWords = 1024;          // bitmap reduction tile (4 KB)
 constexpr uint32_t kGroupTiles = 32;           // tiles per reduction group
