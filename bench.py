@@ -266,7 +266,8 @@ def main():
     tfile = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tfile):
         try:
-            traffic = json.load(open(tfile)).get(a.config)
+            t = json.load(open(tfile)).get(a.config)
+            traffic = None if t is None else int(t["bytes_per_launch"])
         except Exception:
             traffic = None
 

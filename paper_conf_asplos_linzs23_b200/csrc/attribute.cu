@@ -634,12 +634,24 @@ __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
   for (uint64_t e = gwarp; e < cnt; e += nwarps) {
     const RangeEntry r = rq[e];
     const uint64_t w0 = r.bit_lo >> 5, w1 = r.bit_hi >> 5;
-    for (uint64_t w = w0 + lane; w <= w1; w += 32) {
-      uint32_t m = 0xFFFFFFFFu;
-      if (w == w0) m &= 0xFFFFFFFFu << (r.bit_lo & 31);
-      if (w == w1) m &= 0xFFFFFFFFu >> (31 - (r.bit_hi & 31));
-      if (m == 0xFFFFFFFFu) orw[w] = m; else red_or(orw + w, m);
+    // edge words: masked RED; interior: all-ones, 16-B stores on the
+    // 4-word-aligned middle and scalar stores around it
+    if (lane == 0) red_or(orw + w0, w0 == w1 ? (0xFFFFFFFFu << (r.bit_lo & 31)) &
+                                                 (0xFFFFFFFFu >> (31 - (r.bit_hi & 31)))
+                                               : 0xFFFFFFFFu << (r.bit_lo & 31));
+    if (lane == 1 && w1 != w0) red_or(orw + w1, 0xFFFFFFFFu >> (31 - (r.bit_hi & 31)));
+    if (w1 <= w0 + 1) continue;
+    const uint64_t i0 = w0 + 1, i1 = w1;                 // interior [i0, i1)
+    const uint64_t a0 = (i0 + 3) & ~3ull, a1 = i1 & ~3ull;
+    if (a0 >= a1) {
+      for (uint64_t w = i0 + lane; w < i1; w += 32) orw[w] = 0xFFFFFFFFu;
+      continue;
     }
+    if (i0 + lane < a0) orw[i0 + lane] = 0xFFFFFFFFu;
+    if (a1 + lane < i1) orw[a1 + lane] = 0xFFFFFFFFu;
+    uint4* v = reinterpret_cast<uint4*>(orw + a0);
+    const uint64_t nv = (a1 - a0) >> 2;
+    for (uint64_t k = lane; k < nv; k += 32) v[k] = make_uint4(~0u, ~0u, ~0u, ~0u);
   }
 }
 

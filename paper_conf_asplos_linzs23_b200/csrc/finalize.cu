@@ -39,8 +39,19 @@ __device__ __forceinline__ M32 m32_word(uint32_t w, uint32_t nvalid) {
   m.suf = nvalid - 1 - m.hi;
   // zeros strictly between lo and hi: longest run of ones in y
   uint32_t y = ~w & ((1u << m.hi) - 1u) & ~((2u << m.lo) - 1u);
-  uint32_t run = 0;
-  while (y) { y &= y >> 1; ++run; }
+  // longest run of ones in y (y != ~0 here: it excludes bits lo and hi), by
+  // binary lifting: A_j marks starts of runs >= 2^j (A_{j+1} = A_j & A_j >> 2^j);
+  // cur marks starts of runs >= run; extend run by 2^j, j = 4..0, whenever a
+  // run continues for another 2^j bits.  Branch-free, about 30 instructions.
+  const uint32_t a1 = y & (y >> 1), a2 = a1 & (a1 >> 2), a3 = a2 & (a2 >> 4), a4 = a3 & (a3 >> 8);
+  const uint32_t A[5] = {y, a1, a2, a3, a4};
+  uint32_t cur = 0xFFFFFFFFu, run = 0;
+#pragma unroll
+  for (int j = 4; j >= 0; --j) {
+    const uint32_t t = cur & (A[j] >> run);
+    run += t ? (1u << j) : 0u;
+    cur = t ? t : cur;
+  }
   m.best = max(max(m.pre, m.suf), run);
   return m;
 }
@@ -116,7 +127,14 @@ __global__ void __launch_bounds__(256) tile_reduce_kernel(const uint32_t* __rest
       const uint32_t wb = b * 128 + 4 * lane;   // tile-relative word of v[b].x
       uint32_t real[4] = {v[b].x, v[b].y, v[b].z, v[b].w};
       uint32_t run[4] = {v[b].x, v[b].y, v[b].z, v[b].w};
-      if (uint32_t(b + 1) * 128 * 32 > nbits) {   // block reaches past the tile's last bit
+      const bool partial = uint32_t(b + 1) * 128 * 32 > nbits;   // warp-uniform
+      const bool lz = (v[b].x | v[b].y | v[b].z | v[b].w) == 0u;
+      const bool lo1 = (v[b].x & v[b].y & v[b].z & v[b].w) == 0xFFFFFFFFu;
+      if (!partial) {                                 // whole block untouched / fully accessed
+        if (__all_sync(FULL_MASK, lz)) { acc = m32_cat(acc, M32{4096, 0, kNoPos32, kNoPos32, 4096, 4096, 4096}); continue; }
+        if (__all_sync(FULL_MASK, lo1)) { acc = m32_cat(acc, M32{4096, 4096, 0, 4095, 0, 0, 0}); continue; }
+      }
+      if (partial) {   // block reaches past the tile's last bit
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
           const uint32_t bj = (wb + j) * 32;
@@ -128,15 +146,23 @@ __global__ void __launch_bounds__(256) tile_reduce_kernel(const uint32_t* __rest
       }
       // lane: real popcount / first / last accessed bit; run-view fold
       uint32_t pop = 0, lo = kNoPos32, hi = kNoPos32;
-      M32 r = m32_identity();
+      M32 r;
+      if (!partial && lz) {
+        r = M32{128, 0, kNoPos32, kNoPos32, 128, 128, 128};
+      } else if (!partial && lo1) {
+        r = M32{128, 128, 0, 127, 0, 0, 0};
+        pop = 128; lo = 0; hi = 127;
+      } else {
+        r = m32_identity();
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        pop += __popc(real[j]);
-        if (real[j]) {
-          if (lo == kNoPos32) lo = 32 * j + __ffs(real[j]) - 1;
-          hi = 32 * j + 31 - __clz(real[j]);
+        for (int j = 0; j < 4; ++j) {
+          pop += __popc(real[j]);
+          if (real[j]) {
+            if (lo == kNoPos32) lo = 32 * j + __ffs(real[j]) - 1;
+            hi = 32 * j + 31 - __clz(real[j]);
+          }
+          r = m32_cat(r, m32_word(run[j], 32));
         }
-        r = m32_cat(r, m32_word(run[j], 32));
       }
       // block (128 words): combine the 32 lanes in order
       M32 blk;
@@ -242,7 +268,22 @@ __device__ __forceinline__ HitM hit_shfl_down(const HitM& m, int d) {
 }
 
 // B5 + B6: one warp per object.
-__global__ void __launch_bounds__(256) object_finalize_kernel(const FinalParams p) {
+// acc_ts / acc_cs are staged in shared memory when they fit (the hit-row scan
+// looks them up once per accessing API, on a dependent chain).
+constexpr uint32_t kSmemAcc = 8192;
+
+template <bool kStaged>
+__global__ void __launch_bounds__(128) object_finalize_kernel(const FinalParams p) {
+  extern __shared__ uint32_t s_acc[];   // [n_acc] ts, then [n_acc] cs bytes
+  const uint32_t* acc_ts = p.acc_ts;
+  const uint8_t* acc_cs = p.acc_cs;
+  if (kStaged) {
+    uint8_t* s_cs = reinterpret_cast<uint8_t*>(s_acc + p.n_acc);
+    for (uint32_t i = threadIdx.x; i < p.n_acc; i += blockDim.x) { s_acc[i] = p.acc_ts[i]; s_cs[i] = p.acc_cs[i]; }
+    __syncthreads();
+    acc_ts = s_acc;
+    acc_cs = s_cs;
+  }
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
@@ -262,29 +303,27 @@ __global__ void __launch_bounds__(256) object_finalize_kernel(const FinalParams 
     const DevObj ob = p.objs[o];
     const uint32_t nh = p.n_hit[o];
     const uint32_t nwords = (2 * nh + 31) / 32;
+    // each lane folds a contiguous run of hit words, then one ordered tree
+    const uint32_t per = (nwords + 31) / 32;
+    const uint32_t wlo = min(nwords, lane * per), whi = min(nwords, wlo + per);
     HitM hm = hit_identity();
-    for (uint32_t wb = 0; wb < nwords; wb += 32) {
-      HitM m = hit_identity();
-      const uint32_t wi = wb + lane;
-      if (wi < nwords) {
-        uint32_t w = p.orw[ob.hit_word + wi];
-        while (w) {
-          const uint32_t b = __ffs(w) - 1;
-          const uint32_t j = b >> 1;                  // API slot inside this word
-          const uint32_t pair = (w >> (2 * j)) & 3u;  // bit0 read, bit1 write
-          w &= ~(3u << (2 * j));
-          const uint32_t rank = ob.r_lo + wi * 16 + j;
-          const uint32_t ts = __ldg(p.acc_ts + rank);
-          const uint32_t cs = __ldg(p.acc_cs + rank);
-          const uint32_t wr = (pair >> 1) & 1u;
-          const HitM one{1, ts, ts, wr | (cs << 1) | (wr << 2) | (cs << 3), 0, 0, 0, 0};
-          m = hit_cat(m, one, p.ti_min_idle);
-        }
+    for (uint32_t wi = wlo; wi < whi; ++wi) {
+      uint32_t w = p.orw[ob.hit_word + wi];
+      while (w) {
+        const uint32_t b = __ffs(w) - 1;
+        const uint32_t j = b >> 1;                  // API slot inside this word
+        const uint32_t pair = (w >> (2 * j)) & 3u;  // bit0 read, bit1 write
+        w &= ~(3u << (2 * j));
+        const uint32_t rank = ob.r_lo + wi * 16 + j;
+        const uint32_t ts = acc_ts[rank];
+        const uint32_t cs = acc_cs[rank];
+        const uint32_t wr = (pair >> 1) & 1u;
+        const HitM one{1, ts, ts, wr | (cs << 1) | (wr << 2) | (cs << 3), 0, 0, 0, 0};
+        hm = hit_cat(hm, one, p.ti_min_idle);
       }
-#pragma unroll
-      for (int d = 1; d < 32; d <<= 1) m = hit_cat(m, hit_shfl_down(m, d), p.ti_min_idle);
-      if (lane == 0) hm = hit_cat(hm, m, p.ti_min_idle);
     }
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) hm = hit_cat(hm, hit_shfl_down(hm, d), p.ti_min_idle);
     if (lane != 0) continue;
     // ---- stats (A6)
     const uint64_t n = (ob.end - ob.base) >> ob.shift;
@@ -341,9 +380,12 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   const uint64_t gb = (p.n_groups + 7) / 8;
   const unsigned g3 = (unsigned)(gb < uint64_t(num_sms) * 16 ? gb : uint64_t(num_sms) * 16);
   group_reduce_kernel<<<g3 ? g3 : 1, 256, 0, s>>>(p.groups, p.n_groups, p.tile_part, p.group_part);
-  const uint64_t ob = (p.n_obj + 7) / 8;
-  const unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
-  object_finalize_kernel<<<g2, 256, 0, s>>>(p);
+  const uint64_t ob = (p.n_obj + 3) / 4;   // one warp per object, 4 warps per block
+  const unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 32 ? ob : uint64_t(num_sms) * 32);
+  if (p.n_acc <= kSmemAcc)
+    object_finalize_kernel<true><<<g2, 128, p.n_acc * 5 + 16, s>>>(p);
+  else
+    object_finalize_kernel<false><<<g2, 128, 0, s>>>(p);
   return 3;
 }
 

@@ -546,6 +546,7 @@ DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_threshold
   p.acc_ts = at<uint32_t>(ctx, ctx->L.acc_ts);
   p.acc_cs = at<uint8_t>(ctx, ctx->L.acc_cs);
   p.n_hit = at<uint32_t>(ctx, ctx->L.n_hit);
+  p.n_acc = ctx->n_acc;
   p.n_obj = ctx->n_obj;
   p.ti_min_idle = t.ti_min_idle;
   p.oa_pct = t.oa_accessed_pct;

@@ -85,6 +85,7 @@ struct FinalParams {
   const uint32_t* acc_ts;    // [n_acc]
   const uint8_t* acc_cs;     // [n_acc] 1 if MEMCPY/MEMSET
   const uint32_t* n_hit;     // [n_obj] number of access APIs in the hit row
+  uint32_t n_acc;
   uint64_t n_obj;
   uint32_t ti_min_idle, oa_pct, frag_pct;
   void* stats;               // drgpum_object_stats[n_obj]
