@@ -32,13 +32,14 @@ namespace drgpum {
 
 constexpr int kConsumerWarps = 8;
 constexpr int kAttrThreads = kConsumerWarps * 32;
-constexpr int kStages = 4;                                   // per-warp ring depth
+constexpr int kStages = 3;                                   // per-warp ring depth
 constexpr int kTilesPerWarp = 4;                             // 32-record tiles per stage
 constexpr int kWarpRecords = kTilesPerWarp * 32;             // 128 records = 2 KB per stage
-// 8 warps x 4 x 2 KB ring + 16 KB level-1 keys + barriers = 80 KB: two blocks
-// per SM leave ~66 KB of L1 for the index / object-table loads
+// per block: 8 warps x 3 x 2 KB rings + 4 KB level-1 keys + barriers + 256 x 56 B
+// lane caches + counters = ~66 KB: three blocks (24 warps) per SM with ~26 KB of L1
 constexpr size_t kAttrSmem = size_t(kConsumerWarps) * kStages * kWarpRecords * 16 + kL1MaxKeys * 8 +
-                             size_t(kConsumerWarps) * kStages * (8 + 4);
+                             size_t(kConsumerWarps) * kStages * 16 + size_t(kAttrThreads) * 56 +
+                             size_t(kConsumerWarps) * 24;
 // Dynamic work units: chunk k of a launch covers records [chunk_start(k),
 // chunk_start(k+1)): big chunks (fewer cache warm-ups at chunk starts) for
 // the first ~80% of the records, small ones at the end (balance).
@@ -69,19 +70,6 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
         : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
   } while (!done);
-}
-// producer-side wait: back off so the spinning lane does not steal issue slots
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
-  uint32_t done;
-  asm volatile(
-      "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-      : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-  while (!done) {
-    __nanosleep(256);
-    asm volatile(
-        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-        : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-  }
 }
 __device__ __forceinline__ void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes,
                                             uint64_t* bar, uint64_t policy) {
@@ -161,19 +149,23 @@ __device__ __forceinline__ void warp_or_words(uint32_t* words, uint64_t key, uin
 }
 
 // ------------------------------------------------------------------ lane state
-struct LaneCache {
-  uint64_t base, size;        // cached object: [base, base+size)
-  uint64_t bm_word, hit_word;  // object's first bitmap word; hit-row word
+// Per-lane object cache.  The authoritative copy lives in SHARED memory (one
+// per thread) and only the out-of-line slow paths touch it; the fast paths run
+// on a register mirror of the five fields they need, so the slow-path state
+// costs no registers (this is what lets three blocks share an SM).
+struct SlowCache {                       // 56 B
+  uint64_t base, size;                   // cached object: [base, base+size)
+  uint64_t bm_word, hit_word;            // its first bitmap word; its hit-row word
   uint32_t t_alloc, t_free, r_lo, shift, obj;
-  uint32_t meta;              // ts|w<<31 whose first/last/hit work is done (fast-path key)
-  uint32_t ts, rank;          // last timestamp -> access-API rank
-  uint32_t first_known;       // first[obj] <= first_known is known
-  uint32_t last_known;        // last[obj]  >= last_known  is known
-  uint64_t hw;                // hit word whose bits hbits are known set
-  uint32_t hbits;
+  uint32_t meta;                         // ts|w<<31 whose first/last/hit work is done
 };
+struct FastCache { uint64_t base, size, bm_word; uint32_t shift, meta; };
 
-struct LaneCounts { uint32_t rec, attr, unattr, clip, inval, ovf; };
+struct WarpCounts { uint32_t rec, attr, unattr, clip, inval, ovf; };   // per warp, shared memory
+
+__device__ __forceinline__ FastCache mirror(const SlowCache* c) {
+  return FastCache{c->base, c->size, c->bm_word, c->shift, c->meta};
+}
 
 __device__ __forceinline__ uint32_t find_object(const AttrParams& p, const uint64_t* s_l1,
                                                 uint64_t addr, uint32_t ts) {
@@ -226,58 +218,68 @@ __device__ __noinline__ void enqueue_range(RangeEntry* rq, uint32_t rq_cap, unsi
   }
 }
 
+__device__ __forceinline__ void add_counts(WarpCounts* wc, int lane, uint32_t rec, uint32_t attr,
+                                           uint32_t unattr, uint32_t clip, uint32_t inval, uint32_t ovf) {
+  rec = __reduce_add_sync(FULL_MASK, rec);
+  attr = __reduce_add_sync(FULL_MASK, attr);
+  unattr = __reduce_add_sync(FULL_MASK, unattr);
+  clip = __reduce_add_sync(FULL_MASK, clip);
+  inval = __reduce_add_sync(FULL_MASK, inval);
+  ovf = __reduce_add_sync(FULL_MASK, ovf);
+  if (lane == 0) {
+    wc->rec += rec; wc->attr += attr; wc->unattr += unattr;
+    wc->clip += clip; wc->inval += inval; wc->ovf += ovf;
+  }
+}
+
 // ------------------------------------------------------------------ slow path
 // The complete per-lane algorithm (every lane, any record).  Leaves each lane
-// with c.meta = the record's meta when the record was attributed, so that
-// following records of the same (object, API, rw) take the fast path.
+// with c->meta = the record's meta when the record was attributed, so that
+// following records of the same (object, API, rw) take the fast paths.
 __device__ __noinline__ void process_slow(const AttrParams& p, const uint64_t* s_l1, uint4 r,
-                                          bool present, int lane, LaneCache& c, LaneCounts& k) {
+                                          bool present, int lane, SlowCache* c, WarpCounts* wc) {
   const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
   const uint32_t size = r.z;
   const uint32_t ts = r.w & 0x7FFFFFFFu;
   const uint32_t is_w = r.w >> 31;
-  // ---- A1: validity
+  // ---- A1: validity (footnote 2: ALLOC/FREE timestamps access nothing)
   bool ok = present && size != 0 && ts < p.n_api && addr <= ~0ull - size;
-  if (ok && ts != c.ts) { c.rank = __ldg(p.acc_rank + ts); c.ts = ts; }
-  ok = ok && c.rank != kNone;
-  k.rec += present;
-  k.inval += present && !ok;
+  const uint32_t rank = ok ? __ldg(p.acc_rank + ts) : kNone;
+  ok = ok && rank != kNone;
   // ---- A2: object lookup
   bool att = false;
+  uint32_t clip = 0, ovf = 0;
   if (ok) {
-    att = addr - c.base < c.size && ts > c.t_alloc && ts < c.t_free;
+    att = addr - c->base < c->size && ts > c->t_alloc && ts < c->t_free;
     if (!att) {
       const uint32_t o = find_object(p, s_l1, addr, ts);
       if (o != kNone) {
         const uint4* q = reinterpret_cast<const uint4*>(p.objs + o);
         const uint4 a = __ldg(q), b = __ldg(q + 1), d = __ldg(q + 2);
         if (ts < d.y) {
-          c.base = (uint64_t(a.y) << 32) | a.x;
-          c.size = ((uint64_t(a.w) << 32) | a.z) - c.base;
-          c.bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
-          c.hit_word = (uint64_t(b.w) << 32) | b.z;
-          c.t_alloc = d.x; c.t_free = d.y; c.r_lo = d.z; c.shift = d.w;
-          c.obj = o;
-          c.first_known = kNever; c.last_known = 0;
-          c.hw = kNoKey; c.hbits = 0;
+          c->base = (uint64_t(a.y) << 32) | a.x;
+          c->size = ((uint64_t(a.w) << 32) | a.z) - c->base;
+          c->bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
+          c->hit_word = (uint64_t(b.w) << 32) | b.z;
+          c->t_alloc = d.x; c->t_free = d.y; c->r_lo = d.z; c->shift = d.w;
+          c->obj = o;
           att = true;
         }
       }
     }
-    k.attr += att;
-    k.unattr += !att;
   }
   // ---- A3: element bits
   uint64_t key0 = kNoKey, key1 = kNoKey;
   uint32_t m0 = 0, m1 = 0;
+  const uint32_t obj = c->obj;
   if (att) {
-    uint64_t off_end = addr - c.base + size;   // no overflow: addr+size validated
-    if (off_end > c.size) { off_end = c.size; k.clip++; }
-    const uint64_t gb0 = c.bm_word * 32 + ((addr - c.base) >> c.shift);
-    const uint64_t gb1 = c.bm_word * 32 + ((off_end - 1) >> c.shift);
+    uint64_t off_end = addr - c->base + size;   // no overflow: addr+size validated
+    if (off_end > c->size) { off_end = c->size; clip = 1; }
+    const uint64_t gb0 = c->bm_word * 32 + ((addr - c->base) >> c->shift);
+    const uint64_t gb1 = c->bm_word * 32 + ((off_end - 1) >> c->shift);
     const uint64_t w0 = gb0 >> 5, w1 = gb1 >> 5;
     if (w1 - w0 >= 2) {
-      enqueue_range(p.rq, p.rq_cap, p.ctr, p.orw, gb0, gb1, k.ovf);
+      enqueue_range(p.rq, p.rq_cap, p.ctr, p.orw, gb0, gb1, ovf);
     } else if (w1 == w0) {
       key0 = w0; m0 = bits_mask(gb0 & 31, gb1 & 31);
     } else {
@@ -287,40 +289,25 @@ __device__ __noinline__ void process_slow(const AttrParams& p, const uint64_t* s
   }
   warp_or_words(p.orw, key0, m0, lane);
   if (__any_sync(FULL_MASK, key1 != kNoKey)) warp_or_words(p.orw, key1, m1, lane);
-  // ---- A4: liveness fold (skipped where this lane already knows it holds)
-  const bool need_min = att && ts < c.first_known;
-  if (__any_sync(FULL_MASK, need_min)) {
+  // ---- A4: liveness fold and hit row, one RED per run of equal objects / words
+  if (__any_sync(FULL_MASK, att)) {
     bool tail;
-    const uint64_t key = need_min ? c.obj : kNoKey;
-    const uint32_t v = seg_scan(key, ts, lane, tail, OpMin());
-    if (tail && need_min) red_min(p.first + c.obj, v);
-    if (need_min) c.first_known = ts;
-  }
-  const bool need_max = att && ts > c.last_known;
-  if (__any_sync(FULL_MASK, need_max)) {
-    bool tail;
-    const uint64_t key = need_max ? c.obj : kNoKey;
-    const uint32_t v = seg_scan(key, ts, lane, tail, OpMax());
-    if (tail && need_max) red_max(p.last + c.obj, v);
-    if (need_max) c.last_known = ts;
-  }
-  // hit row: bit 2*(rank - r_lo) + is_write of the object's row
-  uint64_t hkey = kNoKey;
-  uint32_t hm = 0;
-  if (att) {
-    const uint32_t hb = 2 * (c.rank - c.r_lo) + is_w;
-    const uint64_t hw = c.hit_word + (hb >> 5);
-    const uint32_t bit = 1u << (hb & 31);
-    if (!(hw == c.hw && (c.hbits & bit))) { hkey = hw; hm = bit; }
-  }
-  if (__any_sync(FULL_MASK, hkey != kNoKey)) {
-    warp_or_words(p.orw, hkey, hm, lane);
-    if (hkey != kNoKey) {
-      if (hkey == c.hw) c.hbits |= hm; else { c.hw = hkey; c.hbits = hm; }
+    const uint64_t key = att ? obj : kNoKey;
+    const uint32_t vmin = seg_scan(key, ts, lane, tail, OpMin());
+    if (tail && att) red_min(p.first + obj, vmin);
+    const uint32_t vmax = seg_scan(key, ts, lane, tail, OpMax());
+    if (tail && att) red_max(p.last + obj, vmax);
+    uint64_t hkey = kNoKey;
+    uint32_t hm = 0;
+    if (att) {
+      const uint32_t hb = 2 * (rank - c->r_lo) + is_w;
+      hkey = c->hit_word + (hb >> 5);
+      hm = 1u << (hb & 31);
     }
+    warp_or_words(p.orw, hkey, hm, lane);
   }
-  // first/last/hit for (c.obj, ts, is_w) are now ensured by this lane
-  c.meta = att ? r.w : kNever;
+  c->meta = att ? r.w : kNever;
+  add_counts(wc, lane, present, att, ok && !att, clip, present && !ok, ovf);
 }
 
 // ------------------------------------------------------------------ fast path
@@ -329,6 +316,19 @@ __device__ __noinline__ void process_slow(const AttrParams& p, const uint64_t* s
 // and every lane's record lies inside that object, unclipped, <= 2 words.
 // e0/e1 are element indices relative to the object; bm_word its first word.
 // Only the bitmap OR remains.
+// OR the element range [e0, e1] (at most two words) of an object's bitmap.
+// OR is idempotent, so records sharing a word need no warp-level merge; the
+// L2 atomic units have the headroom (ncu: ~15% busy), the issue slots do not.
+__device__ __forceinline__ void red_record(uint32_t* orw, uint64_t bm_word, uint32_t e0, uint32_t e1) {
+  const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
+  if (w1 == w0) {
+    red_or(orw + bm_word + w0, bits_mask(e0 & 31, e1 & 31));
+  } else {
+    red_or(orw + bm_word + w0, 0xFFFFFFFFu << (e0 & 31));
+    red_or(orw + bm_word + w1, 0xFFFFFFFFu >> (31 - (e1 & 31)));
+  }
+}
+
 __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_t e0, uint32_t e1, int lane) {
   // contiguous union: intervals chain (start within or right after the
   // previous interval, monotone ends) -> union = [e0 of lane 0, e1 of lane 31]
@@ -348,11 +348,7 @@ __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_
     }
     return;
   }
-  const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
-  const bool two = w1 != w0;
-  warp_or_words(orw, bm_word + w0, two ? (0xFFFFFFFFu << (e0 & 31)) : bits_mask(e0 & 31, e1 & 31), lane);
-  if (__any_sync(FULL_MASK, two))
-    warp_or_words(orw, two ? bm_word + w1 : kNoKey, 0xFFFFFFFFu >> (31 - (e1 & 31)), lane);
+  red_record(orw, bm_word, e0, e1);   // irregular: each record ORs its own word(s)
 }
 
 // Affine tier: the warp's 128 consecutive records (4 tiles, lane l holds
@@ -364,7 +360,7 @@ __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_
 // (st <= size or st <= elem_size) the union is ONE element range, written
 // with one RED.OR per word; otherwise each record ORs its own word(s).
 // Returns false (no side effect) when the precondition does not hold.
-__device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const LaneCache& c,
+__device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const FastCache& c,
                                            uint32_t* orw, int lane) {
   // predicted record j = 32k + lane: {lo(a0) + j*st, hi(a0), sz, meta}; the
   // mismatch bits of all four words of all records are ORed with 3-input
@@ -406,41 +402,47 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
     return 1;
   }
   if (((sz - 1) >> c.shift) >= 32) return 0;   // records wider than a word: tile path
-  if ((st32 >> c.shift) >= 32) {
-    // stride >= 32 elements: every record owns its word(s), nothing to merge
-#pragma unroll
-    for (int k = 0; k < kTilesPerWarp; ++k) {
-      const uint32_t off = o0 + (32 * k + lane) * st32;
-      const uint32_t e0 = off >> c.shift, e1 = (off + sz - 1) >> c.shift;
-      const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
-      if (w1 == w0) {
-        red_or(orw + c.bm_word + w0, bits_mask(e0 & 31, e1 & 31));
-      } else {
-        red_or(orw + c.bm_word + w0, 0xFFFFFFFFu << (e0 & 31));
-        red_or(orw + c.bm_word + w1, 0xFFFFFFFFu >> (31 - (e1 & 31)));
-      }
-    }
-    return 2;
-  }
+  // not one range: every record ORs its own word(s) (offsets in 32 bits)
+  uint32_t off = o0 + uint32_t(lane) * st32;
 #pragma unroll
   for (int k = 0; k < kTilesPerWarp; ++k) {
-    const uint32_t off = o0 + (32 * k + lane) * st32;
-    const uint32_t e0 = off >> c.shift, e1 = (off + sz - 1) >> c.shift;
-    const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
-    const bool two = w1 != w0;
-    warp_or_words(orw, c.bm_word + w0, two ? (0xFFFFFFFFu << (e0 & 31)) : bits_mask(e0 & 31, e1 & 31), lane);
-    if (__any_sync(FULL_MASK, two))
-      warp_or_words(orw, two ? c.bm_word + w1 : kNoKey, 0xFFFFFFFFu >> (31 - (e1 & 31)), lane);
+    red_record(orw, c.bm_word, off >> c.shift, (off + sz - 1) >> c.shift);
+    off += 32u * st32;
   }
   return 2;
+}
+
+// In-object tier: the warp's 128 records all carry the cached (API, rw) and
+// fall inside the cached object (< 4 GiB), unclipped, <= 2 words each, in any
+// order (random gathers, strided sweeps that wrap).  Each record ORs its own
+// word(s): no warp analysis, OR is idempotent.  Returns false without side
+// effects otherwise.
+__device__ __forceinline__ bool try_in_object(const uint4 (&r)[kTilesPerWarp], const FastCache& c,
+                                              uint32_t* orw) {
+  const uint32_t osz = uint32_t(c.size);
+  uint32_t e0[kTilesPerWarp], e1[kTilesPerWarp];
+  bool ok = true;
+#pragma unroll
+  for (int k = 0; k < kTilesPerWarp; ++k) {
+    const uint64_t off = ((uint64_t(r[k].y) << 32) | r[k].x) - c.base;
+    const uint32_t off32 = uint32_t(off), size = r[k].z;
+    e0[k] = off32 >> c.shift;
+    e1[k] = (off32 + size - 1) >> c.shift;
+    ok = ok && r[k].w == c.meta && (off >> 32) == 0 && off32 < osz && size != 0 &&
+         size <= osz - off32 && (e1[k] >> 5) - (e0[k] >> 5) < 2;
+  }
+  if (!__all_sync(FULL_MASK, ok)) return false;
+#pragma unroll
+  for (int k = 0; k < kTilesPerWarp; ++k) red_record(orw, c.bm_word, e0[k], e1[k]);
+  return true;
 }
 
 // Warp-uniform slow path: all 32 records share one (API, rw) and land in one
 // object (the first tile of every burst).  One lane resolves the object and
 // folds first/last/hit once for the warp; the lanes adopt the object into
 // their caches.  Returns false (no side effect) when the precondition fails.
-__device__ __forceinline__ bool try_uniform_slow(const AttrParams& p, const uint64_t* s_l1, uint4 r,
-                                                 bool present, int lane, LaneCache& c, LaneCounts& k) {
+__device__ __noinline__ bool try_uniform_slow(const AttrParams& p, const uint64_t* s_l1, uint4 r,
+                                              bool present, int lane, SlowCache* c, WarpCounts* wc) {
   const uint32_t meta = r.w;
   const uint32_t meta0 = __shfl_sync(FULL_MASK, meta, 0);   // all lanes: never inside && / ||
   if (!__all_sync(FULL_MASK, present && meta == meta0)) return false;
@@ -464,35 +466,39 @@ __device__ __forceinline__ bool try_uniform_slow(const AttrParams& p, const uint
   const uint32_t off32 = uint32_t(off), e0 = off32 >> d.w, e1 = (off32 + size - 1) >> d.w;
   const bool ok = off < osz && size != 0 && size <= uint32_t(osz) - off32 && (e1 >> 5) - (e0 >> 5) < 2;
   if (!__all_sync(FULL_MASK, ok)) return false;
-  c.base = base; c.size = osz;
-  c.bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
-  c.hit_word = (uint64_t(b.w) << 32) | b.z;
-  c.t_alloc = d.x; c.t_free = d.y; c.r_lo = d.z; c.shift = d.w; c.obj = o;
-  c.ts = ts; c.rank = rank;
-  const uint32_t hb = 2 * (rank - d.z) + is_w;
-  c.hw = c.hit_word + (hb >> 5);
-  c.hbits = 1u << (hb & 31);
+  c->base = base; c->size = osz;
+  c->bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
+  c->hit_word = (uint64_t(b.w) << 32) | b.z;
+  c->t_alloc = d.x; c->t_free = d.y; c->r_lo = d.z; c->shift = d.w; c->obj = o;
+  c->meta = meta;
   if (lane == 0) {
+    const uint32_t hb = 2 * (rank - d.z) + is_w;
     red_min(p.first + o, ts);
     red_max(p.last + o, ts);
-    red_or(p.orw + c.hw, c.hbits);
+    red_or(p.orw + c->hit_word + (hb >> 5), 1u << (hb & 31));
+    wc->rec += 32;
+    wc->attr += 32;
   }
-  c.first_known = ts; c.last_known = ts; c.meta = meta;
-  k.rec += 1; k.attr += 1;
-  fast_or(p.orw, c.bm_word, e0, e1, lane);
+  fast_or(p.orw, c->bm_word, e0, e1, lane);
   return true;
 }
 
-__global__ void __launch_bounds__(kAttrThreads, 2) attribute_kernel(const AttrParams p) {
+__global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid_constant__ AttrParams p) {
   extern __shared__ __align__(128) uint8_t smem[];
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  // per-warp ring: kStages slots of kWarpRecords records, one mbarrier and one
-  // record count per slot
+  // shared memory: per-warp rings | level-1 keys | barriers, slot counts |
+  // per-lane slow caches | per-warp counters
   uint4* ring = reinterpret_cast<uint4*>(smem) + size_t(warp) * kStages * kWarpRecords;
-  uint64_t* s_l1 = reinterpret_cast<uint64_t*>(smem + size_t(kConsumerWarps) * kStages * kWarpRecords * 16);
+  uint8_t* tail = smem + size_t(kConsumerWarps) * kStages * kWarpRecords * 16;
+  uint64_t* s_l1 = reinterpret_cast<uint64_t*>(tail);
   uint64_t* full = s_l1 + kL1MaxKeys + warp * kStages;
   uint32_t* slot_cnt = reinterpret_cast<uint32_t*>(s_l1 + kL1MaxKeys + kConsumerWarps * kStages) + warp * kStages;
+  SlowCache* caches = reinterpret_cast<SlowCache*>(
+      tail + kL1MaxKeys * 8 + kConsumerWarps * kStages * 16);
+  WarpCounts* wcounts = reinterpret_cast<WarpCounts*>(caches + kAttrThreads);
+  SlowCache* my = caches + threadIdx.x;
+  WarpCounts* wc = wcounts + warp;
 
   // Work distribution: warps take contiguous chunks (chunk_start) of records
   // from a global cursor (dynamic, so slow warps do not set the kernel's end).
@@ -517,7 +523,10 @@ __global__ void __launch_bounds__(kAttrThreads, 2) attribute_kernel(const AttrPa
     }
   };
 
+  my->base = 0; my->size = 0; my->bm_word = 0; my->hit_word = 0;
+  my->t_alloc = 0; my->t_free = 0; my->r_lo = 0; my->shift = 0; my->obj = kNone; my->meta = kNever;
   if (lane == 0) {
+    *wc = WarpCounts{0, 0, 0, 0, 0, 0};
     for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     for (int s = 0; s < kStages; ++s) fetch(s);
@@ -525,16 +534,10 @@ __global__ void __launch_bounds__(kAttrThreads, 2) attribute_kernel(const AttrPa
   for (uint32_t i = threadIdx.x; i < p.n_l1; i += blockDim.x) s_l1[i] = p.l1[i];
   __syncthreads();
 
-  LaneCache c;
-  c.base = 0; c.size = 0; c.bm_word = 0; c.hit_word = 0;
-  c.t_alloc = 0; c.t_free = 0; c.r_lo = 0; c.shift = 0; c.obj = kNone;
-  c.meta = kNever; c.ts = kNone; c.rank = kNone; c.first_known = kNever; c.last_known = 0;
-  c.hw = kNoKey; c.hbits = 0;
-  LaneCounts k = {0, 0, 0, 0, 0, 0};
+  FastCache c = mirror(my);
   uint32_t fast_rec = 0;
   uint32_t n_aff_u = 0, n_aff_w = 0, n_fast = 0, n_slow = 0;   // diagnostics (warp-uniform)
   bool uni = false;  // warp-uniform: all lanes cache one object (< 4 GiB) and one (API, rw)
-  const uint32_t wfirst = 0;
   for (uint32_t st = 0;; ++st) {
     const int s = int(st % kStages);
     mbar_wait(&full[s], (st / kStages) & 1);
@@ -571,10 +574,15 @@ __global__ void __launch_bounds__(kAttrThreads, 2) attribute_kernel(const AttrPa
         if (how == 1) n_aff_u += kTilesPerWarp; else n_aff_w += kTilesPerWarp;
         continue;
       }
+      if (try_in_object(r4, c, p.orw)) {
+        fast_rec += kTilesPerWarp;
+        n_fast += kTilesPerWarp;
+        continue;
+      }
     }
 #pragma unroll 1
     for (int t = 0; t < ntiles; ++t) {
-      const bool present = wfirst + t * 32 + lane < cnt;
+      const bool present = t * 32 + lane < cnt;
       uint4 r = r4[0];                       // register select, no local-memory indexing
 #pragma unroll
       for (int j = 1; j < kTilesPerWarp; ++j) if (t == j) r = r4[j];
@@ -593,39 +601,28 @@ __global__ void __launch_bounds__(kAttrThreads, 2) attribute_kernel(const AttrPa
           continue;
         }
       }
-      if (try_uniform_slow(p, s_l1, r, present, lane, c, k)) {
-        ++n_slow;
-        uni = true;
-        continue;
-      }
-      {  // rare: out of line, through copies so c and k stay in registers elsewhere
-        LaneCache c2 = c;
-        LaneCounts k2 = k;
-        process_slow(p, s_l1, r, present, lane, c2, k2);
-        c = c2;
-        k = k2;
-      }
+      if (!try_uniform_slow(p, s_l1, r, present, lane, my, wc))
+        process_slow(p, s_l1, r, present, lane, my, wc);
       ++n_slow;
+      c = mirror(my);
       const uint32_t m0 = __shfl_sync(FULL_MASK, c.meta, 0);
-      const uint32_t o0 = __shfl_sync(FULL_MASK, c.obj, 0);
-      uni = __all_sync(FULL_MASK, c.meta == m0 && c.obj == o0 && m0 != kNever && c.size <= 0xFFFFFFFFull);
+      const uint32_t o0 = __shfl_sync(FULL_MASK, my->obj, 0);
+      uni = __all_sync(FULL_MASK, c.meta == m0 && my->obj == o0 && m0 != kNever && c.size <= 0xFFFFFFFFull);
     }
   }
-  k.rec += fast_rec;
-  k.attr += fast_rec;
+  // A5: counters -- fast-path records per lane plus the warp's slow-path sums
+  const uint32_t fr = __reduce_add_sync(FULL_MASK, fast_rec);
+  __syncwarp();
   if (lane == 0) {
+    const uint32_t v[6] = {wc->rec + fr, wc->attr + fr, wc->unattr, wc->clip, wc->inval, wc->ovf};
+    const int slot[6] = {C_RECORDS, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID, C_RQ_OVERFLOW};
+#pragma unroll
+    for (int i = 0; i < 6; ++i)
+      if (v[i]) atomicAdd(&p.ctr[slot[i]], (unsigned long long)v[i]);
     atomicAdd(&p.ctr[C_TILES_AFFINE_UNION], (unsigned long long)n_aff_u);
     atomicAdd(&p.ctr[C_TILES_AFFINE_WORDS], (unsigned long long)n_aff_w);
     atomicAdd(&p.ctr[C_TILES_FAST], (unsigned long long)n_fast);
     atomicAdd(&p.ctr[C_TILES_SLOW], (unsigned long long)n_slow);
-  }
-  // A5: warp-reduce the counters, one atomic per warp and counter
-  const uint32_t v[6] = {k.rec, k.attr, k.unattr, k.clip, k.inval, k.ovf};
-  const int slot[6] = {C_RECORDS, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID, C_RQ_OVERFLOW};
-#pragma unroll
-  for (int i = 0; i < 6; ++i) {
-    const uint32_t sum = __reduce_add_sync(FULL_MASK, v[i]);
-    if (lane == 0 && sum) atomicAdd(&p.ctr[slot[i]], (unsigned long long)sum);
   }
 }
 
