@@ -9,7 +9,7 @@ b = json.load(open(f"{D}/bench.json"))
 lines += ["## bench.py (C2, N=1)", "", "```", json.dumps({k: b[k] for k in (
     "value", "unit", "ms_per_step", "phases_ms", "roofline", "e2e", "gpu_launches", "clocks",
     "attribution_paths_tiles", "counters")}, indent=1), "```", ""]
-rows = list(csv.reader(open(f"{D}/launches.csv")))
+rows = list(csv.reader(open(f"{D}/launches.csv"))) if os.path.exists(f"{D}/launches.csv") else []
 hdr = None; agg = collections.defaultdict(list)
 for r in rows:
     if "Kernel Name" in r: hdr = r; continue
@@ -17,12 +17,13 @@ for r in rows:
         d = dict(zip(hdr, r))
         if d.get("Metric Name") == "gpu__time_duration.sum":
             agg[d["Kernel Name"].split("(")[0]].append(float(d["Metric Value"]))
-tot = sum(sum(v) for v in agg.values())
-lines += ["## Launch list (ncu --metrics gpu__time_duration.sum --clock-control none; "
+tot = sum(sum(v) for v in agg.values()) or 1.0
+if agg:
+  lines += ["## Launch list (ncu --metrics gpu__time_duration.sum --clock-control none; "
           "bench.py --steps 3 --warmup 3 --e2e-steps 1; cold-cache, serialised: compare shares)", "",
           "| kernel | launches | mean us | share |", "|---|---|---|---|"]
 for k, v in sorted(agg.items(), key=lambda kv: -sum(kv[1])):
-    lines.append(f"| {k} | {len(v)} | {sum(v)/len(v)/1e3:.1f} | {sum(v)/tot*100:.1f}% |")
+  lines.append(f"| {k} | {len(v)} | {sum(v)/len(v)/1e3:.1f} | {sum(v)/tot*100:.1f}% |")
 lines.append("")
 lines.append("Note: the e2e leg launches the attribution kernel once per 4 Mi-record staging chunk, "
              "so per-launch means mix device-resident (1e8-record) and staged launches.")
