@@ -259,6 +259,24 @@ DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx *ctx,
  * (cached object and API), out[3] full per-lane path.  Synchronous. */
 DRGPUM_API drgpum_status drgpum_path_stats(drgpum_ctx *ctx, uint64_t out[4], void *stream);
 
+/* NEXT-1 redundant allocation (§5.1 l.253-260, Fig. 3; Def 3.3 l.154,
+ * X = 10% l.156): the paper's one-pass pairing over the used objects' first
+ * and last accessing APIs.  (reuser[k], donor[k]): object reuser[k] can reuse
+ * donor[k]'s memory -- donor's last access precedes reuser's first (last after
+ * first at equal timestamps), their sizes differ by at most pct% of the larger
+ * [R19-R21], each donor is handed out once, pairs in the order the tail-to-head
+ * walk finds them.  Up to cap pairs are written; *n_pairs is the total.
+ *
+ * drgpum_redundant_pairs is the host algorithm on plain arrays (sizes in
+ * bytes, T_first, T_last, used flags; load order).  drgpum_redundant_alloc
+ * runs it on the context's finalized stats (synchronous; finalizes if needed).
+ * EINVAL on NULL outputs / pct > 100. */
+DRGPUM_API drgpum_status drgpum_redundant_pairs(const uint64_t *sizes, const uint32_t *first,
+    const uint32_t *last, const uint8_t *used, uint64_t n, uint32_t pct,
+    uint32_t *reuser, uint32_t *donor, uint64_t cap, uint64_t *n_pairs);
+DRGPUM_API drgpum_status drgpum_redundant_alloc(drgpum_ctx *ctx, uint32_t pct,
+    uint32_t *reuser, uint32_t *donor, uint64_t cap, uint64_t *n_pairs, void *stream);
+
 /* Message for the last failed call on ctx (never NULL). */
 DRGPUM_API const char *drgpum_last_error(const drgpum_ctx *ctx);
 

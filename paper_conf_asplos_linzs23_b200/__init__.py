@@ -13,9 +13,10 @@ It never imports the CPU oracle (oracle/ is test infrastructure only).
 """
 from ._lib import (OBJECT_DTYPE, RECORD_DTYPE, STATS_DTYPE, REPORT_DTYPE, COUNTERS_DTYPE,
                    LAYOUT_DTYPE, NEVER, EA, LD, UA, ML, TI, DW, OA, OA_ACTIONABLE,
-                   FLAG_NAMES, DrgpumError, EXPORTS, LIB_PATH, load)
+                   FLAG_NAMES, DrgpumError, EXPORTS, LIB_PATH, load, redundant_pairs)
 from .session import Session
 
 __all__ = ["Session", "OBJECT_DTYPE", "RECORD_DTYPE", "STATS_DTYPE", "REPORT_DTYPE",
            "COUNTERS_DTYPE", "LAYOUT_DTYPE", "NEVER", "EA", "LD", "UA", "ML", "TI", "DW",
-           "OA", "OA_ACTIONABLE", "FLAG_NAMES", "DrgpumError", "EXPORTS", "LIB_PATH", "load"]
+           "OA", "OA_ACTIONABLE", "FLAG_NAMES", "DrgpumError", "EXPORTS", "LIB_PATH", "load",
+           "redundant_pairs"]

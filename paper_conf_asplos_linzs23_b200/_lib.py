@@ -61,7 +61,8 @@ EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_workspace_size",
            "drgpum_workspace_bind", "drgpum_reset", "drgpum_trace_attribute",
            "drgpum_trace_attribute_host", "drgpum_shadow_view", "drgpum_object_layout",
            "drgpum_merge_or", "drgpum_finalize", "drgpum_object_stats", "drgpum_patterns",
-           "drgpum_consistency_errors", "drgpum_path_stats", "drgpum_last_error", "drgpum_destroy",
+           "drgpum_consistency_errors", "drgpum_path_stats", "drgpum_redundant_pairs",
+           "drgpum_redundant_alloc", "drgpum_last_error", "drgpum_destroy",
            "drgpum_launch_count"]
 
 _lib = None
@@ -94,6 +95,8 @@ def load():
         "drgpum_patterns": ([P, ctypes.POINTER(Thresholds), P, P], I),
         "drgpum_consistency_errors": ([P, ctypes.POINTER(U64), P], I),
         "drgpum_path_stats": ([P, P, P], I),
+        "drgpum_redundant_pairs": ([P, P, P, P, U64, U32, P, P, U64, ctypes.POINTER(U64)], I),
+        "drgpum_redundant_alloc": ([P, U32, P, P, U64, ctypes.POINTER(U64), P], I),
         "drgpum_last_error": ([P], ctypes.c_char_p),
         "drgpum_destroy": ([P], None),
         "drgpum_launch_count": ([P], U64),
@@ -109,3 +112,25 @@ def load():
 def check(ctx, status):
     if status != 0:
         raise DrgpumError(status, load().drgpum_last_error(ctx).decode(errors="replace"))
+
+
+def redundant_pairs(sizes, first, last, used, pct=10):
+    """Host algorithm of NEXT-1 on plain arrays (no GPU needed): list of
+    (reuser, donor) object indices."""
+    L = load()
+    sizes = np.ascontiguousarray(sizes, dtype=np.uint64)
+    first = np.ascontiguousarray(first, dtype=np.uint32)
+    last = np.ascontiguousarray(last, dtype=np.uint32)
+    used = np.ascontiguousarray(used, dtype=np.uint8)
+    n = sizes.shape[0]
+    cnt = ctypes.c_uint64()
+    p = lambda a: ctypes.c_void_p(a.ctypes.data)
+    st = L.drgpum_redundant_pairs(p(sizes), p(first), p(last), p(used), n, pct, None, None, 0,
+                                  ctypes.byref(cnt))
+    if st:
+        raise DrgpumError(st, "drgpum_redundant_pairs")
+    a = np.zeros(cnt.value, np.uint32)
+    b = np.zeros(cnt.value, np.uint32)
+    L.drgpum_redundant_pairs(p(sizes), p(first), p(last), p(used), n, pct, p(a), p(b), cnt.value,
+                             ctypes.byref(cnt))
+    return list(zip(a.tolist(), b.tolist()))

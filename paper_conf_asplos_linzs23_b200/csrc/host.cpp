@@ -633,6 +633,29 @@ DRGPUM_API drgpum_status drgpum_path_stats(drgpum_ctx* ctx, uint64_t out[4], voi
   return DRGPUM_OK;
 }
 
+DRGPUM_API drgpum_status drgpum_redundant_alloc(drgpum_ctx* ctx, uint32_t pct, uint32_t* reuser,
+                                                uint32_t* donor, uint64_t cap, uint64_t* n_pairs,
+                                                void* stream) {
+  if (!ctx || !n_pairs || (cap && (!reuser || !donor))) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "redundant_alloc before workspace_bind");
+  std::vector<drgpum_object_stats_t> st(ctx->n_obj);
+  drgpum_status s = drgpum_object_stats(ctx, st.data(), nullptr, stream);
+  if (s != DRGPUM_OK) return s;
+  std::vector<uint64_t> sizes(ctx->n_obj);
+  std::vector<uint32_t> first(ctx->n_obj), last(ctx->n_obj);
+  std::vector<uint8_t> used(ctx->n_obj);
+  for (uint64_t o = 0; o < ctx->n_obj; ++o) {
+    sizes[o] = ctx->objs[o].size;
+    first[o] = st[o].t_first;
+    last[o] = st[o].t_last;
+    used[o] = st[o].n_access_apis > 0;
+  }
+  s = drgpum_redundant_pairs(sizes.data(), first.data(), last.data(), used.data(), ctx->n_obj, pct,
+                             reuser, donor, cap, n_pairs);
+  if (s != DRGPUM_OK) return fail(ctx, s, "redundant_pairs: invalid arguments");
+  return DRGPUM_OK;
+}
+
 DRGPUM_API const char* drgpum_last_error(const drgpum_ctx* ctx) {
   if (!ctx) return "null context";
   return ctx->err.c_str();

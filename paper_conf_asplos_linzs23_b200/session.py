@@ -140,6 +140,17 @@ class Session:
         check(self._h, self.L.drgpum_path_stats(self._h, _np_ptr(out), _stream_handle(stream)))
         return dict(zip(("affine_union", "affine_words", "tile_fast", "slow"), (int(x) for x in out)))
 
+    def redundant_allocations(self, pct=10, stream=None):
+        """NEXT-1: [(reuser, donor), ...] from this session's first/last uses."""
+        cnt = ctypes.c_uint64()
+        check(self._h, self.L.drgpum_redundant_alloc(self._h, pct, None, None, 0, ctypes.byref(cnt),
+                                                     _stream_handle(stream)))
+        a = np.zeros(cnt.value, np.uint32)
+        b = np.zeros(cnt.value, np.uint32)
+        check(self._h, self.L.drgpum_redundant_alloc(self._h, pct, _np_ptr(a), _np_ptr(b), cnt.value,
+                                                     ctypes.byref(cnt), _stream_handle(stream)))
+        return list(zip(a.tolist(), b.tolist()))
+
     def layout(self):
         out = np.zeros(self.n_obj, dtype=LAYOUT_DTYPE)
         check(self._h, self.L.drgpum_object_layout(self._h, _np_ptr(out)))

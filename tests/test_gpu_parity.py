@@ -211,3 +211,21 @@ def test_c2_full_size():
     p = build_config("C2")
     r = gen_records(p, 0, p.n_records)
     check_parity(p.objects, p.kinds, r)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_redundant_allocation_end_to_end(name):
+    """NEXT-1 on the GPU's first/last (drgpum_redundant_alloc) == the literal
+    walk (oracle/ra.py) on the oracle's first/last."""
+    from oracle.ra import redundant_allocations
+    p = build_config(name, **({"n_records": 1 << 22} if name == "C2" else {}))
+    r = gen_records(p, 0, p.n_records)
+    s = _session(p.objects, p.kinds)
+    s.attribute(torch.from_numpy(r.view(np.uint8)).cuda())
+    got = s.redundant_allocations(10)
+    orc = Oracle(p.objects, p.kinds)
+    orc.attribute(r)
+    ost, _ = orc.stats()
+    want = redundant_allocations(p.objects["size"], ost["t_first"], ost["t_last"],
+                                 ost["n_access_apis"] > 0, 10)
+    assert got == want and len(want) > 0
