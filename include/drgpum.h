@@ -186,6 +186,15 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx *ctx,
     const drgpum_object_t *h_objs, uint64_t n_obj,
     const uint8_t *h_api_kinds, uint32_t n_api);
 
+/* Optional analyses.  Set after objects_load and
+ * before workspace_size / workspace_bind (ESTATE otherwise); EINVAL on unknown
+ * bits.  DRGPUM_FEATURE_STRUCTURED (NEXT-3, structured access, Def 3.10
+ * l.200, §5.2 l.270) adds a u32 owner word per element of every object to the
+ * workspace, and every trace_attribute call then also runs the structured-
+ * access pass over its records. */
+enum { DRGPUM_FEATURE_STRUCTURED = 1 };
+DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx *ctx, uint32_t features);
+
 /* Bytes of device workspace the loaded program needs (ESTATE before load). */
 DRGPUM_API drgpum_status drgpum_workspace_size(const drgpum_ctx *ctx, uint64_t *bytes);
 
@@ -252,6 +261,14 @@ DRGPUM_API drgpum_status drgpum_patterns(drgpum_ctx *ctx,
  * (first/last folded by atomics vs the hit rows; must be 0). */
 DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx *ctx,
     uint64_t *h_errors, void *stream);
+
+/* NEXT-3 result (synchronous): h_sa[o] = 1 iff object o is accessed by at
+ * least two GPU APIs and no element of o is touched by two different APIs
+ * (each API touches its own slice, the slices do not overlap -- Def 3.10);
+ * h_overlap[o] = 1 iff some element is touched by two APIs.  Either output
+ * may be NULL.  ESTATE unless DRGPUM_FEATURE_STRUCTURED was enabled. */
+DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx *ctx, uint8_t *h_sa, uint8_t *h_overlap,
+                                           void *stream);
 
 /* Diagnostics (not part of the method): how many 32-record tiles took each
  * attribution path since the last reset -- out[0] affine run with one union

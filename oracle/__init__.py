@@ -55,6 +55,8 @@ def _load():
         L.oracle_get_bitmap.argtypes = [P, U64, P]
         L.oracle_get_accesses.argtypes = [P, U64, P, P, U64]
         L.oracle_get_accesses.restype = U64
+        L.oracle_track_structured.argtypes = [P]
+        L.oracle_structured.argtypes = [P, P, P]
         _lib = L
     return _lib
 
@@ -76,7 +78,7 @@ def validate(objects, kinds):
 class Oracle:
     """One oracle run over (objects, kinds); feed records with attribute()."""
 
-    def __init__(self, objects, kinds):
+    def __init__(self, objects, kinds, structured=False):
         L = _load()
         self.objects = np.ascontiguousarray(objects)
         self.kinds = np.ascontiguousarray(kinds, dtype=np.uint8)
@@ -86,6 +88,8 @@ class Oracle:
         self.status = st.value
         if not self._h:
             raise ValueError(f"oracle: objects rejected with status {st.value}")
+        if structured:
+            L.oracle_track_structured(self._h)
 
     def __del__(self):
         if getattr(self, "_h", None):
@@ -109,6 +113,14 @@ class Oracle:
         th = np.array(thresholds, dtype=np.uint32)
         _load().oracle_patterns(self._h, _ptr(th), _ptr(out))
         return out
+
+    def structured(self):
+        """NEXT-3: (sa u8[n_obj], overlap u8[n_obj]); needs structured=True."""
+        n = self.objects.shape[0]
+        sa = np.zeros(n, np.uint8)
+        ov = np.zeros(n, np.uint8)
+        _load().oracle_structured(self._h, _ptr(sa), _ptr(ov))
+        return sa, ov
 
     def bitmap(self, o):
         """Object o's bitmap as a bool array of n_elem entries."""

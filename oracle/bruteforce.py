@@ -138,3 +138,34 @@ def validate(objects, kinds):
             if pb < qe and qb < pe and max(int(p["t_alloc"]), int(q["t_alloc"])) < min(ptf, qtf):
                 return 2
     return 0
+
+
+def bruteforce_structured(objects, kinds, records):
+    """NEXT-3 structured access by definition (Def 3.10, l.200): per object,
+    the set of elements each accessing GPU API touches; SA iff at least two
+    APIs access O and their slices are pairwise disjoint.  Returns (sa, overlap)
+    lists of 0/1."""
+    n_api = len(kinds)
+    objs = [dict(base=int(o["base"]), size=int(o["size"]), E=int(o["elem_size"]),
+                 ta=int(o["t_alloc"]), tf=int(o["t_free"])) for o in objects]
+    slices = [dict() for _ in objs]          # ts -> set of elements
+    for r in records:
+        addr, size, meta = int(r["addr"]), int(r["size"]), int(r["meta"])
+        ts = meta & 0x7FFFFFFF
+        if size == 0 or ts >= n_api or kinds[ts] in (ALLOC, FREE) or addr + size > U64_MAX:
+            continue
+        for i, o in enumerate(objs):
+            if o["base"] <= addr < o["base"] + o["size"] and o["ta"] < ts and \
+                    (o["tf"] == NEVER or ts < o["tf"]):
+                end = min(addr + size, o["base"] + o["size"])
+                s = slices[i].setdefault(ts, set())
+                for b in range(addr, end):
+                    s.add((b - o["base"]) // o["E"])
+                break
+    sa, ov = [], []
+    for sl in slices:
+        sets = list(sl.values())
+        overlap = any(sets[a] & sets[b] for a in range(len(sets)) for b in range(a + 1, len(sets)))
+        ov.append(int(overlap))
+        sa.append(int(len(sets) >= 2 and not overlap))
+    return sa, ov

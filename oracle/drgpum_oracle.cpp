@@ -68,6 +68,11 @@ struct State {
   std::vector<std::map<uint32_t, Flags>> accesses;  // APIs that access O, by T
   Counters ctr;
   std::vector<std::vector<uint32_t>> alloc_at, free_at;   // per timestamp
+  // NEXT-3 structured access (Def 3.10): per object, element -> the GPU API
+  // that touched it, and whether any element was touched by two APIs
+  std::vector<std::map<uint64_t, uint32_t>> elem_api;
+  std::vector<uint8_t> overlap;
+  bool track_sa = false;
 };
 
 }  // namespace
@@ -144,6 +149,27 @@ void* oracle_new(const Obj* objs, uint64_t n_obj, const uint8_t* kinds,
 
 void oracle_free(void* p) { delete static_cast<State*>(p); }
 
+// NEXT-3: record, for every element, which GPU APIs touch it (call before
+// oracle_attribute).
+void oracle_track_structured(void* p) {
+  State& s = *static_cast<State*>(p);
+  s.track_sa = true;
+  s.elem_api.assign(s.objs.size(), {});
+  s.overlap.assign(s.objs.size(), 0);
+}
+
+// NEXT-3 structured access (Def 3.10, l.200; §5.2 l.270): object O matches if
+// each GPU API that accesses it touches a slice of O and the slices do not
+// overlap -- at least two accessing APIs and no element touched by two of
+// them.  out[o] = 1 if O matches; overlap[o] = 1 if two APIs share an element.
+void oracle_structured(void* p, uint8_t* out, uint8_t* overlap) {
+  State& s = *static_cast<State*>(p);
+  for (size_t o = 0; o < s.objs.size(); ++o) {
+    overlap[o] = s.overlap[o];
+    out[o] = (s.accesses[o].size() >= 2 && !s.overlap[o]) ? 1 : 0;
+  }
+}
+
 // Attribute n records.  May be called repeatedly (chunks); each call replays
 // the timeline over its own records.  Records are grouped by timestamp first
 // (stable counting sort) so that every record is looked up in M as M stands
@@ -197,6 +223,12 @@ void oracle_attribute(void* p, const Rec* recs, uint64_t n) {
       const uint64_t e0 = (r.addr - ob.base) / ob.elem_size;
       const uint64_t e1 = (end - 1 - ob.base) / ob.elem_size;
       for (uint64_t e = e0; e <= e1; ++e) s.bitmap[o][e] = true;
+      if (s.track_sa) {                                               // Def 3.10
+        for (uint64_t e = e0; e <= e1; ++e) {
+          auto ins = s.elem_api[o].emplace(e, t);
+          if (!ins.second && ins.first->second != t) s.overlap[o] = 1;
+        }
+      }
       if (t < s.first[o]) s.first[o] = t;
       if (t > s.last[o]) s.last[o] = t;
       Flags& f = s.accesses[o][t];   // value-initialised {false, false} on first touch

@@ -681,3 +681,90 @@ int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s) {
 }
 
 }  // namespace drgpum
+
+namespace drgpum {
+
+// ------------------------------------------------------------------ NEXT-3
+// Structured access (Def 3.10 l.200; §5.2 l.270): O matches if every GPU API
+// that accesses O touches its own slice and no two slices overlap.  Exactly
+// that, order-free: owner[e] holds (access rank + 1) of the first API that
+// claimed element e (a CAS from 0); an API that finds another API's tag on an
+// element marks O as overlapped.  Values only go 0 -> tag, so a stale plain
+// read is either 0 (then the CAS decides) or already final.
+__device__ __forceinline__ void sa_claim(uint32_t* owner, uint32_t* overlap, uint64_t g, uint32_t tag,
+                                         uint32_t obj) {
+  uint32_t cur = owner[g];
+  if (cur == 0) cur = atomicCAS(owner + g, 0u, tag);
+  if (cur != 0 && cur != tag) red_or(overlap + obj, 1u);
+}
+
+constexpr uint32_t kSaInline = 64;          // elements claimed by the lane itself
+constexpr uint64_t kSaChunk = 4096;         // queued work item (elements)
+
+__global__ void __launch_bounds__(256) structured_kernel(const __grid_constant__ SaParams q) {
+  const AttrParams& p = q.a;
+  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
+  // per-thread object cache: records of a thread are strided, but bursts are
+  // long, so consecutive records of one thread still share objects
+  uint64_t c_base = 0, c_size = 0, c_eb = 0;
+  uint32_t c_ta = 0, c_tf = 0, c_obj = kNone, c_shift = 0;
+  for (uint64_t i = tid; i < p.n; i += nth) {
+    const uint4 r = p.recs[i];
+    const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
+    const uint32_t size = r.z, ts = r.w & 0x7FFFFFFFu;
+    if (size == 0 || ts >= p.n_api || addr > ~0ull - size) continue;
+    const uint32_t rank = __ldg(p.acc_rank + ts);
+    if (rank == kNone) continue;
+    if (!(addr - c_base < c_size && ts > c_ta && ts < c_tf)) {
+      const uint32_t o = find_object(p, p.l1, addr, ts);   // level-1 keys from global here
+      if (o == kNone) continue;
+      const DevObj d = p.objs[o];
+      if (ts >= d.t_free) continue;
+      c_base = d.base; c_size = d.end - d.base; c_ta = d.t_alloc; c_tf = d.t_free;
+      c_obj = o; c_shift = d.shift; c_eb = __ldg(q.elem_base + o);
+    }
+    const uint64_t off = addr - c_base;
+    const uint64_t end = min(off + size, c_size);
+    const uint64_t e0 = off >> c_shift, e1 = (end - 1) >> c_shift;
+    const uint32_t tag = rank + 1;
+    if (e1 - e0 < kSaInline) {
+      for (uint64_t e = e0; e <= e1; ++e) sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
+      continue;
+    }
+    const uint64_t nch = (e1 - e0) / kSaChunk + 1;
+    const unsigned long long slot = atomicAdd(q.q_count, (unsigned long long)nch);
+    for (uint64_t k = 0; k < nch; ++k) {
+      const uint64_t lo = e0 + k * kSaChunk, hi = min(e1, lo + kSaChunk - 1);
+      if (slot + k < q.q_cap) {
+        q.q[slot + k] = SaRange{c_eb + lo, c_eb + hi, c_obj, tag, {0, 0}};
+      } else {
+        for (uint64_t e = lo; e <= hi; ++e) sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) structured_range_kernel(const __grid_constant__ SaParams q) {
+  const unsigned long long raw = *q.q_count;
+  const uint64_t cnt = raw < q.q_cap ? raw : q.q_cap;
+  const int lane = threadIdx.x & 31;
+  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  for (uint64_t e = gwarp; e < cnt; e += nwarps) {
+    const SaRange r = q.q[e];
+    for (uint64_t g = r.g_lo + lane; g <= r.g_hi; g += 32) sa_claim(q.owner, q.overlap, g, r.tag, r.obj);
+  }
+}
+
+int launch_structured(const SaParams& q, int num_sms, cudaStream_t s) {
+  if (q.a.n == 0) return 0;
+  cudaMemsetAsync(q.q_count, 0, sizeof(unsigned long long), s);
+  uint64_t blocks = (q.a.n + 255) / 256;
+  if (blocks > uint64_t(num_sms) * 8) blocks = uint64_t(num_sms) * 8;
+  structured_kernel<<<(unsigned)blocks, 256, 0, s>>>(q);
+  structured_range_kernel<<<num_sms * 4, 256, 0, s>>>(q);
+  return 2;
+}
+
+}  // namespace drgpum

@@ -35,6 +35,8 @@ struct Layout {
   uint64_t dyn_end;
   uint64_t objs, seg_start, seg_cand_off, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
   uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage;
+  // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
+  uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
   uint64_t total;
 };
 
@@ -69,6 +71,10 @@ struct drgpum_ctx {
   std::vector<drgpum_object_layout_t> layout;
   uint64_t bitmap_words = 0, hit_words = 0;
   uint32_t rq_cap = 1u << 20;
+  uint32_t features = 0;
+  std::vector<uint64_t> elem_base;
+  uint64_t n_elem_total = 0;
+  uint32_t sa_q_cap = 1u << 20;
   Layout L{};
   uint8_t* ws = nullptr;
   uint64_t ws_bytes = 0;
@@ -110,6 +116,8 @@ cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
 drgpum_status set_device(drgpum_ctx* ctx) { CK(cudaSetDevice(ctx->device)); return DRGPUM_OK; }
 
 uint32_t ilog2(uint32_t e) { uint32_t s = 0; while ((1u << s) < e) ++s; return s; }
+
+drgpum_status compute_layout(drgpum_ctx* c);
 
 // Build everything derived from (objects, kinds) on the host.
 drgpum_status build_tables(drgpum_ctx* c) {
@@ -243,8 +251,20 @@ drgpum_status build_tables(drgpum_ctx* c) {
     hw += (2ull * (r_hi - r_lo) + 31) / 32;
   }
   c->hit_words = hw;
+  c->elem_base.assign(n, 0);
+  uint64_t eb = 0;
+  for (uint64_t i = 0; i < n; ++i) { c->elem_base[i] = eb; eb += c->objs[i].size / c->objs[i].elem_size; }
+  c->n_elem_total = eb;
 
-  // workspace layout
+  return compute_layout(c);
+}
+
+// Workspace layout for the loaded program (and the enabled features).
+drgpum_status compute_layout(drgpum_ctx* c) {
+  const uint64_t n = c->n_obj;
+  const uint32_t n_api = c->n_api;
+  const uint64_t S = c->seg_start.size();
+  const uint64_t total = c->cand.size();
   Layout& L = c->L;
   uint64_t off = 0;
   auto put = [&](uint64_t bytes) { uint64_t o = off; off = align_up(off + bytes); return o; };
@@ -271,6 +291,15 @@ drgpum_status build_tables(drgpum_ctx* c) {
   L.reports = put(sizeof(drgpum_pattern_report_t) * n);
   L.rq = put(sizeof(RangeEntry) * c->rq_cap);
   L.stage = put(2 * kStageRecords * sizeof(drgpum_record_t));
+  L.sa_owner = L.sa_overlap = L.sa_elem_base = L.sa_q = L.sa_qcount = L.sa_end = off;
+  if (c->features & DRGPUM_FEATURE_STRUCTURED) {
+    L.sa_owner = put(4 * c->n_elem_total);
+    L.sa_overlap = put(4 * n);
+    L.sa_qcount = put(8);
+    L.sa_end = off;                           // [sa_owner, sa_end) is zeroed per trace
+    L.sa_elem_base = put(8 * n);
+    L.sa_q = put(sizeof(SaRange) * c->sa_q_cap);
+  }
   L.total = off;
   return DRGPUM_OK;
 }
@@ -303,6 +332,8 @@ drgpum_status validate(drgpum_ctx* c, const drgpum_object_t* objs, uint64_t n_ob
 drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s) {
   CK(cudaMemsetAsync(ctx->ws, 0, ctx->L.dyn_end, s));
   ctx->launches += launch_fill_u32(at<uint32_t>(ctx, ctx->L.first), kNever, ctx->n_obj, s);
+  if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
+    CK(cudaMemsetAsync(ctx->ws + ctx->L.sa_owner, 0, ctx->L.sa_end - ctx->L.sa_owner, s));
   ctx->final_valid = false;
   return DRGPUM_OK;
 }
@@ -328,6 +359,18 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   p.rq = at<RangeEntry>(c, c->L.rq);
   p.rq_cap = c->rq_cap;
   return p;
+}
+
+SaParams sa_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
+  SaParams q;
+  q.a = attr_params(c, recs, n);
+  q.owner = at<uint32_t>(c, c->L.sa_owner);
+  q.elem_base = at<uint64_t>(c, c->L.sa_elem_base);
+  q.overlap = at<uint32_t>(c, c->L.sa_overlap);
+  q.q = at<SaRange>(c, c->L.sa_q);
+  q.q_cap = c->sa_q_cap;
+  q.q_count = at<unsigned long long>(c, c->L.sa_qcount);
+  return q;
 }
 
 }  // namespace
@@ -367,6 +410,8 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   ctx->acc_rank.swap(tmp.acc_rank); ctx->acc_ts.swap(tmp.acc_ts); ctx->acc_cs.swap(tmp.acc_cs);
   ctx->n_hit.swap(tmp.n_hit); ctx->tiles.swap(tmp.tiles); ctx->tile_off.swap(tmp.tile_off);
   ctx->groups.swap(tmp.groups); ctx->group_off.swap(tmp.group_off);
+  ctx->elem_base.swap(tmp.elem_base); ctx->n_elem_total = tmp.n_elem_total;
+  ctx->features = 0;
   ctx->layout.swap(tmp.layout);
   ctx->bitmap_words = tmp.bitmap_words; ctx->hit_words = tmp.hit_words;
   ctx->L = tmp.L;
@@ -374,6 +419,35 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   ctx->ws_bytes = 0;
   ctx->state = S_LOADED;
   ctx->final_valid = false;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx* ctx, uint32_t features) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state != S_LOADED) return fail(ctx, DRGPUM_ESTATE, "set_features must follow objects_load and precede workspace_bind");
+  if (features & ~uint32_t(DRGPUM_FEATURE_STRUCTURED)) return fail(ctx, DRGPUM_EINVAL, "unknown feature bits");
+  ctx->features = features;
+  return compute_layout(ctx);
+}
+
+DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx* ctx, uint8_t* h_sa, uint8_t* h_overlap, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "structured before workspace_bind");
+  if (!(ctx->features & DRGPUM_FEATURE_STRUCTURED))
+    return fail(ctx, DRGPUM_ESTATE, "DRGPUM_FEATURE_STRUCTURED was not enabled");
+  std::vector<drgpum_object_stats_t> st(ctx->n_obj);
+  drgpum_status s = drgpum_object_stats(ctx, st.data(), nullptr, stream);
+  if (s != DRGPUM_OK) return s;
+  std::vector<uint32_t> ov(ctx->n_obj);
+  cudaStream_t strm = as_stream(stream);
+  if (ctx->n_obj) {
+    CK(cudaMemcpyAsync(ov.data(), ctx->ws + ctx->L.sa_overlap, 4 * ctx->n_obj, cudaMemcpyDeviceToHost, strm));
+    CK(cudaStreamSynchronize(strm));
+  }
+  for (uint64_t o = 0; o < ctx->n_obj; ++o) {
+    if (h_overlap) h_overlap[o] = ov[o] ? 1 : 0;
+    if (h_sa) h_sa[o] = (st[o].n_access_apis >= 2 && !ov[o]) ? 1 : 0;
+  }
   return DRGPUM_OK;
 }
 
@@ -417,6 +491,8 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
   if ((r = up(L.tiles, ctx->tiles.data(), sizeof(Tile) * ctx->tiles.size()))) return r;
   if ((r = up(L.groups, ctx->groups.data(), sizeof(Group) * ctx->groups.size()))) return r;
   if ((r = up(L.group_off, ctx->group_off.data(), 4 * ctx->group_off.size()))) return r;
+  if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
+    if ((r = up(L.sa_elem_base, ctx->elem_base.data(), 8 * n))) return r;
   if ((r = enqueue_reset(ctx, st))) return r;
   // host vectors stay alive in ctx, so the async uploads are safe; make the
   // bind synchronous anyway so callers may immediately reuse their stream
@@ -440,6 +516,8 @@ DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_re
     return fail(ctx, DRGPUM_EINVAL, "records must be non-NULL and 16-B aligned");
   AttrParams p = attr_params(ctx, d_recs, n);
   ctx->launches += launch_attribute(p, ctx->num_sms, as_stream(stream));
+  if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
+    ctx->launches += launch_structured(sa_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
   ctx->final_valid = false;
   CK(cudaGetLastError());
   return DRGPUM_OK;
@@ -475,6 +553,8 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
     CK(cudaStreamWaitEvent(st, ctx->ev_copied[b], 0));
     AttrParams p = attr_params(ctx, stage[b], m);
     ctx->launches += launch_attribute(p, ctx->num_sms, st);
+    if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
+      ctx->launches += launch_structured(sa_params(ctx, stage[b], m), ctx->num_sms, st);
     CK(cudaEventRecord(ctx->ev_used[b], st));
   }
   CK(cudaStreamSynchronize(ctx->copy_stream));

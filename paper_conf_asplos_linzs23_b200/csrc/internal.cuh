@@ -70,6 +70,18 @@ struct AttrParams {
   uint32_t rq_cap;
 };
 
+// NEXT-3 structured access pass (optional feature).
+struct SaRange { uint64_t g_lo, g_hi; uint32_t obj, tag; uint32_t pad[2]; };   // 32 B
+struct SaParams {
+  AttrParams a;              // records, object table, index, rank table
+  uint32_t* owner;           // [sum n_elem] access-rank+1 of the first API touching the element
+  const uint64_t* elem_base; // [n_obj] first global element index of each object
+  uint32_t* overlap;         // [n_obj] 1 if two APIs touched one element
+  SaRange* q;                // large-range queue
+  uint32_t q_cap;
+  unsigned long long* q_count;
+};
+
 struct FinalParams {
   const uint32_t* orw;
   const Tile* tiles;
@@ -95,6 +107,7 @@ struct FinalParams {
 
 // Launchers (return the number of kernels enqueued).
 int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);
+int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
 int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src,

@@ -38,7 +38,7 @@ class Session:
     kinds:   uint8 array, the GPU-API kind of every timestamp.
     """
 
-    def __init__(self, objects, kinds, device=None):
+    def __init__(self, objects, kinds, device=None, structured=False):
         if not torch.cuda.is_available():
             raise RuntimeError("drgpum Session needs a CUDA device (there is no CPU fallback)")
         self.L = _lib.load()
@@ -55,6 +55,8 @@ class Session:
         check(self._h, st)
         check(self._h, self.L.drgpum_objects_load(self._h, _np_ptr(self.objects), self.n_obj,
                                                   _np_ptr(self.kinds), self.kinds.shape[0]))
+        if structured:
+            check(self._h, self.L.drgpum_set_features(self._h, _lib.FEATURE_STRUCTURED))
         nbytes = ctypes.c_uint64()
         check(self._h, self.L.drgpum_workspace_size(self._h, ctypes.byref(nbytes)))
         self.workspace = torch.empty(max(int(nbytes.value), 256), dtype=torch.uint8,
@@ -139,6 +141,13 @@ class Session:
         out = np.zeros(4, dtype=np.uint64)
         check(self._h, self.L.drgpum_path_stats(self._h, _np_ptr(out), _stream_handle(stream)))
         return dict(zip(("affine_union", "affine_words", "tile_fast", "slow"), (int(x) for x in out)))
+
+    def structured(self, stream=None):
+        """NEXT-3: (sa u8[n_obj], overlap u8[n_obj]); needs structured=True."""
+        sa = np.zeros(self.n_obj, np.uint8)
+        ov = np.zeros(self.n_obj, np.uint8)
+        check(self._h, self.L.drgpum_structured(self._h, _np_ptr(sa), _np_ptr(ov), _stream_handle(stream)))
+        return sa, ov
 
     def redundant_allocations(self, pct=10, stream=None):
         """NEXT-1: [(reuser, donor), ...] from this session's first/last uses."""

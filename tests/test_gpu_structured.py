@@ -1,0 +1,67 @@
+"""GPU parity of NEXT-3 structured access (drgpum_set_features +
+drgpum_structured) with the oracle."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from oracle import Oracle  # noqa: E402
+from tracegen import build_config, build_tiny, gen_all_records  # noqa: E402
+from tests.golden_util import load, to_arrays  # noqa: E402
+
+
+def _gpu(objs, kinds, recs, chunks=1):
+    from paper_conf_asplos_linzs23_b200 import Session
+    s = Session(objs, kinds, structured=True)
+    d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
+    b = np.linspace(0, len(recs), chunks + 1).astype(np.int64)
+    for x, y in zip(b, b[1:]):
+        s.attribute(d[x * 16: y * 16])
+    return s, s.structured()
+
+
+def _oracle(objs, kinds, recs):
+    o = Oracle(objs, kinds, structured=True)
+    o.attribute(recs)
+    return o.structured()
+
+
+def _check(objs, kinds, recs, chunks=1):
+    s, (sa, ov) = _gpu(objs, kinds, recs, chunks)
+    osa, oov = _oracle(objs, kinds, recs)
+    assert np.array_equal(sa, osa) and np.array_equal(ov, oov)
+    return s, sa, ov
+
+
+def test_gramschmidt():
+    fx = load("gramschmidt_structured")
+    objs, kinds, recs, names = to_arrays(fx)
+    _, sa, _ = _check(objs, kinds, recs)
+    assert sa[names["R_gpu"]] == 1 and sa[names["Q_gpu"]] == 0
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_tiny(seed):
+    p = build_tiny(7100 + seed)
+    _check(p.objects, p.kinds, gen_all_records(p), chunks=1 + seed % 3)
+
+
+def test_c1():
+    p = build_config("C1")
+    _, sa, ov = _check(p.objects, p.kinds, gen_all_records(p))
+    assert ov.sum() > 0
+
+
+def test_reset_and_main_results_unchanged():
+    """The structured pass must not change the attribution results."""
+    from paper_conf_asplos_linzs23_b200 import Session
+    p = build_config("C1")
+    r = gen_all_records(p)
+    d = torch.from_numpy(r.view(np.uint8)).cuda()
+    a = Session(p.objects, p.kinds, structured=True)
+    b = Session(p.objects, p.kinds)
+    a.attribute(d); b.attribute(d)
+    assert np.array_equal(a.object_stats()[0], b.object_stats()[0])
+    a.reset(); a.attribute(d)
+    assert np.array_equal(a.structured()[0], _oracle(p.objects, p.kinds, r)[0])
