@@ -192,7 +192,7 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx *ctx,
  * l.200, §5.2 l.270) adds a u32 owner word per element of every object to the
  * workspace, and every trace_attribute call then also runs the structured-
  * access pass over its records. */
-enum { DRGPUM_FEATURE_STRUCTURED = 1 };
+enum { DRGPUM_FEATURE_STRUCTURED = 1, DRGPUM_FEATURE_FREQUENCY = 2 };
 DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx *ctx, uint32_t features);
 
 /* Bytes of device workspace the loaded program needs (ESTATE before load). */
@@ -269,6 +269,21 @@ DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx *ctx,
  * may be NULL.  ESTATE unless DRGPUM_FEATURE_STRUCTURED was enabled. */
 DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx *ctx, uint8_t *h_sa, uint8_t *h_overlap,
                                            void *stream);
+
+/* NEXT-2 results (synchronous; ESTATE unless DRGPUM_FEATURE_FREQUENCY, EINVAL
+ * if the records were not in timestamp order).  For every (object O, access
+ * API A in O's lifetime): n = elements A touched, S1 = sum of their access
+ * frequencies, S2 = sum of squares [R22].  NUAF at A iff the population
+ * coefficient of variation exceeds pct% (fn 3, l.222; X = 20% l.198), i.e.
+ * (n*S2 - S1^2) * 100^2 > pct^2 * S1^2.  drgpum_frequency: per object the
+ * number of APIs at which O matches (h_count) and the first one (h_first,
+ * DRGPUM_NEVER if none).  drgpum_frequency_slots: the raw {n, S1, S2} triples,
+ * u64[3 * n_slots], slots ordered by object (load order) then access API
+ * (object o's slots start at sum of n_hit_apis of the objects before it). */
+DRGPUM_API drgpum_status drgpum_frequency(drgpum_ctx *ctx, uint32_t pct, uint32_t *h_count,
+                                          uint32_t *h_first, void *stream);
+DRGPUM_API drgpum_status drgpum_frequency_slots(drgpum_ctx *ctx, uint64_t *h_acc,
+                                                uint64_t *n_slots, void *stream);
 
 /* Diagnostics (not part of the method): how many 32-record tiles took each
  * attribution path since the last reset -- out[0] affine run with one union

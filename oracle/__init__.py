@@ -57,6 +57,9 @@ def _load():
         L.oracle_get_accesses.restype = U64
         L.oracle_track_structured.argtypes = [P]
         L.oracle_structured.argtypes = [P, P, P]
+        L.oracle_track_frequency.argtypes = [P]
+        L.oracle_frequency.argtypes = [P, P, P, P, P, P, U64]
+        L.oracle_frequency.restype = U64
         _lib = L
     return _lib
 
@@ -78,7 +81,7 @@ def validate(objects, kinds):
 class Oracle:
     """One oracle run over (objects, kinds); feed records with attribute()."""
 
-    def __init__(self, objects, kinds, structured=False):
+    def __init__(self, objects, kinds, structured=False, frequency=False):
         L = _load()
         self.objects = np.ascontiguousarray(objects)
         self.kinds = np.ascontiguousarray(kinds, dtype=np.uint8)
@@ -90,6 +93,8 @@ class Oracle:
             raise ValueError(f"oracle: objects rejected with status {st.value}")
         if structured:
             L.oracle_track_structured(self._h)
+        if frequency:
+            L.oracle_track_frequency(self._h)
 
     def __del__(self):
         if getattr(self, "_h", None):
@@ -122,6 +127,14 @@ class Oracle:
         _load().oracle_structured(self._h, _ptr(sa), _ptr(ov))
         return sa, ov
 
+    def frequency(self):
+        """NEXT-2 rows (obj, ts, n, s1, s2) in (object, ts) order; needs frequency=True."""
+        L = _load()
+        k = L.oracle_frequency(self._h, None, None, None, None, None, 0)
+        cols = [np.zeros(k, np.uint32), np.zeros(k, np.uint32)] + [np.zeros(k, np.uint64) for _ in range(3)]
+        L.oracle_frequency(self._h, *[_ptr(c) for c in cols], k)
+        return tuple(cols)
+
     def bitmap(self, o):
         """Object o's bitmap as a bool array of n_elem entries."""
         ne = int(self.objects["size"][o] // self.objects["elem_size"][o])
@@ -151,3 +164,11 @@ def run_oracle(objects, kinds, records, thresholds=DEFAULT_THRESHOLDS):
     o.attribute(records)
     st, ctr = o.stats()
     return o, st, ctr, o.patterns(thresholds)
+
+
+def nuaf_cv_exceeds(n, s1, s2, pct=20):
+    """Def 3.9 / fn 3: coefficient of variation (population) of the n touched
+    elements' frequencies > pct%, exactly: pct^2 is compared in integers,
+    CV^2 = (n*S2 - S1^2) / S1^2 > (pct/100)^2."""
+    n, s1, s2 = int(n), int(s1), int(s2)
+    return s1 > 0 and (n * s2 - s1 * s1) * 100 * 100 > pct * pct * s1 * s1

@@ -169,3 +169,32 @@ def bruteforce_structured(objects, kinds, records):
         ov.append(int(overlap))
         sa.append(int(len(sets) >= 2 and not overlap))
     return sa, ov
+
+
+def bruteforce_frequency(objects, kinds, records):
+    """NEXT-2 by definition (Def 3.9 l.196, §5.2 l.271): for every (object,
+    accessing API), the access frequency of each element that API touches
+    (byte-wise expansion); rows (obj, ts, n, S1, S2) sorted by (obj, ts)."""
+    n_api = len(kinds)
+    objs = [dict(base=int(o["base"]), size=int(o["size"]), E=int(o["elem_size"]),
+                 ta=int(o["t_alloc"]), tf=int(o["t_free"])) for o in objects]
+    hm = {}
+    for r in records:
+        addr, size, meta = int(r["addr"]), int(r["size"]), int(r["meta"])
+        ts = meta & 0x7FFFFFFF
+        if size == 0 or ts >= n_api or kinds[ts] in (ALLOC, FREE) or addr + size > U64_MAX:
+            continue
+        for i, o in enumerate(objs):
+            if o["base"] <= addr < o["base"] + o["size"] and o["ta"] < ts and \
+                    (o["tf"] == NEVER or ts < o["tf"]):
+                end = min(addr + size, o["base"] + o["size"])
+                elems = {(b - o["base"]) // o["E"] for b in range(addr, end)}
+                d = hm.setdefault((i, ts), {})
+                for e in elems:
+                    d[e] = d.get(e, 0) + 1
+                break
+    rows = []
+    for (i, ts) in sorted(hm):
+        f = list(hm[(i, ts)].values())
+        rows.append((i, ts, len(f), sum(f), sum(c * c for c in f)))
+    return rows

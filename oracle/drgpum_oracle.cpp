@@ -73,6 +73,10 @@ struct State {
   std::vector<std::map<uint64_t, uint32_t>> elem_api;
   std::vector<uint8_t> overlap;
   bool track_sa = false;
+  // NEXT-2 non-uniform access frequency (Def 3.9, l.271): per (object, API)
+  // the "hashmap" of element -> access frequency of that API
+  std::map<std::pair<uint32_t, uint32_t>, std::map<uint64_t, uint64_t>> freq;
+  bool track_freq = false;
 };
 
 }  // namespace
@@ -158,6 +162,36 @@ void oracle_track_structured(void* p) {
   s.overlap.assign(s.objs.size(), 0);
 }
 
+// NEXT-2: keep, per (object, GPU API), the access frequency of every element
+// that API touches (call before oracle_attribute).
+void oracle_track_frequency(void* p) {
+  static_cast<State*>(p)->track_freq = true;
+}
+
+// NEXT-2 non-uniform access frequency (Def 3.9 l.196; §5.2 l.271; fn 3 l.222:
+// coefficient of variation).  For every (object O, accessing API A): n =
+// number of elements A touched (cells of A's hashmap for O), S1 = sum of
+// their frequencies, S2 = sum of squares.  Rows are written in (object, ts)
+// order: obj[k], ts[k], n[k], s1[k], s2[k]; returns the number of rows.
+uint64_t oracle_frequency(void* p, uint32_t* obj, uint32_t* ts, uint64_t* n, uint64_t* s1,
+                          uint64_t* s2, uint64_t cap) {
+  State& s = *static_cast<State*>(p);
+  uint64_t k = 0;
+  for (const auto& kv : s.freq) {
+    if (k < cap) {
+      uint64_t a = 0, b = 0;
+      for (const auto& ec : kv.second) { a += ec.second; b += ec.second * ec.second; }
+      obj[k] = kv.first.first;
+      ts[k] = kv.first.second;
+      n[k] = kv.second.size();
+      s1[k] = a;
+      s2[k] = b;
+    }
+    ++k;
+  }
+  return k;
+}
+
 // NEXT-3 structured access (Def 3.10, l.200; §5.2 l.270): object O matches if
 // each GPU API that accesses it touches a slice of O and the slices do not
 // overlap -- at least two accessing APIs and no element touched by two of
@@ -223,6 +257,10 @@ void oracle_attribute(void* p, const Rec* recs, uint64_t n) {
       const uint64_t e0 = (r.addr - ob.base) / ob.elem_size;
       const uint64_t e1 = (end - 1 - ob.base) / ob.elem_size;
       for (uint64_t e = e0; e <= e1; ++e) s.bitmap[o][e] = true;
+      if (s.track_freq) {                                             // l.271
+        auto& hm = s.freq[{o, t}];
+        for (uint64_t e = e0; e <= e1; ++e) hm[e] += 1;
+      }
       if (s.track_sa) {                                               // Def 3.10
         for (uint64_t e = e0; e <= e1; ++e) {
           auto ins = s.elem_api[o].emplace(e, t);

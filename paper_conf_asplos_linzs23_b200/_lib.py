@@ -30,6 +30,7 @@ assert STATS_DTYPE.itemsize == 56 and REPORT_DTYPE.itemsize == 32 and LAYOUT_DTY
 
 NEVER = 0xFFFFFFFF
 FEATURE_STRUCTURED = 1
+FEATURE_FREQUENCY = 2
 API_ALLOC, API_FREE, API_MEMCPY, API_MEMSET, API_KERNEL = 0, 1, 2, 3, 4
 EA, LD, UA, ML, TI, DW, OA, OA_ACTIONABLE = 1, 2, 4, 8, 16, 32, 64, 128
 FLAG_NAMES = {EA: "EA", LD: "LD", UA: "UA", ML: "ML", TI: "TI", DW: "DW", OA: "OA",
@@ -59,6 +60,7 @@ class DrgpumError(RuntimeError):
 
 
 EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_set_features", "drgpum_structured",
+           "drgpum_frequency", "drgpum_frequency_slots",
            "drgpum_workspace_size",
            "drgpum_workspace_bind", "drgpum_reset", "drgpum_trace_attribute",
            "drgpum_trace_attribute_host", "drgpum_shadow_view", "drgpum_object_layout",
@@ -99,6 +101,8 @@ def load():
         "drgpum_path_stats": ([P, P, P], I),
         "drgpum_set_features": ([P, U32], I),
         "drgpum_structured": ([P, P, P, P], I),
+        "drgpum_frequency": ([P, U32, P, P, P], I),
+        "drgpum_frequency_slots": ([P, P, ctypes.POINTER(U64), P], I),
         "drgpum_redundant_pairs": ([P, P, P, P, U64, U32, P, P, U64, ctypes.POINTER(U64)], I),
         "drgpum_redundant_alloc": ([P, U32, P, P, U64, ctypes.POINTER(U64), P], I),
         "drgpum_last_error": ([P], ctypes.c_char_p),

@@ -37,6 +37,8 @@ struct Layout {
   uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage;
   // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
+  // NEXT-2 frequency (feature): cells[sum n_elem], acc[n_slots][3], state, queue, outputs
+  uint64_t fq_cells, fq_acc, fq_state, fq_qcount, fq_end, fq_slot_base, fq_q, fq_out_count, fq_out_first;
   uint64_t total;
 };
 
@@ -72,8 +74,8 @@ struct drgpum_ctx {
   uint64_t bitmap_words = 0, hit_words = 0;
   uint32_t rq_cap = 1u << 20;
   uint32_t features = 0;
-  std::vector<uint64_t> elem_base;
-  uint64_t n_elem_total = 0;
+  std::vector<uint64_t> elem_base, slot_base;
+  uint64_t n_elem_total = 0, n_slots = 0;
   uint32_t sa_q_cap = 1u << 20;
   Layout L{};
   uint8_t* ws = nullptr;
@@ -255,6 +257,10 @@ drgpum_status build_tables(drgpum_ctx* c) {
   uint64_t eb = 0;
   for (uint64_t i = 0; i < n; ++i) { c->elem_base[i] = eb; eb += c->objs[i].size / c->objs[i].elem_size; }
   c->n_elem_total = eb;
+  c->slot_base.assign(n, 0);
+  uint64_t sb = 0;
+  for (uint64_t i = 0; i < n; ++i) { c->slot_base[i] = sb; sb += c->n_hit[i]; }
+  c->n_slots = sb;
 
   return compute_layout(c);
 }
@@ -292,13 +298,27 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   L.rq = put(sizeof(RangeEntry) * c->rq_cap);
   L.stage = put(2 * kStageRecords * sizeof(drgpum_record_t));
   L.sa_owner = L.sa_overlap = L.sa_elem_base = L.sa_q = L.sa_qcount = L.sa_end = off;
+  if (c->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY))
+    L.sa_elem_base = put(8 * n);              // shared by both features
   if (c->features & DRGPUM_FEATURE_STRUCTURED) {
     L.sa_owner = put(4 * c->n_elem_total);
     L.sa_overlap = put(4 * n);
     L.sa_qcount = put(8);
     L.sa_end = off;                           // [sa_owner, sa_end) is zeroed per trace
-    L.sa_elem_base = put(8 * n);
     L.sa_q = put(sizeof(SaRange) * c->sa_q_cap);
+  }
+  L.fq_cells = L.fq_acc = L.fq_state = L.fq_qcount = L.fq_end = off;
+  L.fq_slot_base = L.fq_q = L.fq_out_count = L.fq_out_first = off;
+  if (c->features & DRGPUM_FEATURE_FREQUENCY) {
+    L.fq_cells = put(8 * c->n_elem_total);
+    L.fq_acc = put(24 * c->n_slots);
+    L.fq_state = put(8);
+    L.fq_qcount = put(8);
+    L.fq_end = off;                           // [fq_cells, fq_end) is zeroed per trace
+    L.fq_slot_base = put(8 * n);
+    L.fq_q = put(sizeof(FreqRange) * c->sa_q_cap);
+    L.fq_out_count = put(4 * n);
+    L.fq_out_first = put(4 * n);
   }
   L.total = off;
   return DRGPUM_OK;
@@ -334,6 +354,8 @@ drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s) {
   ctx->launches += launch_fill_u32(at<uint32_t>(ctx, ctx->L.first), kNever, ctx->n_obj, s);
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     CK(cudaMemsetAsync(ctx->ws + ctx->L.sa_owner, 0, ctx->L.sa_end - ctx->L.sa_owner, s));
+  if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
+    CK(cudaMemsetAsync(ctx->ws + ctx->L.fq_cells, 0, ctx->L.fq_end - ctx->L.fq_cells, s));
   ctx->final_valid = false;
   return DRGPUM_OK;
 }
@@ -359,6 +381,20 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   p.rq = at<RangeEntry>(c, c->L.rq);
   p.rq_cap = c->rq_cap;
   return p;
+}
+
+FreqParams fq_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
+  FreqParams q;
+  q.a = attr_params(c, recs, n);
+  q.cells = at<unsigned long long>(c, c->L.fq_cells);
+  q.elem_base = at<uint64_t>(c, c->L.sa_elem_base);
+  q.slot_base = at<uint64_t>(c, c->L.fq_slot_base);
+  q.acc = at<unsigned long long>(c, c->L.fq_acc);
+  q.q = at<FreqRange>(c, c->L.fq_q);
+  q.q_cap = c->sa_q_cap;
+  q.q_count = at<unsigned long long>(c, c->L.fq_qcount);
+  q.state = at<uint32_t>(c, c->L.fq_state);
+  return q;
 }
 
 SaParams sa_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
@@ -411,6 +447,7 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   ctx->n_hit.swap(tmp.n_hit); ctx->tiles.swap(tmp.tiles); ctx->tile_off.swap(tmp.tile_off);
   ctx->groups.swap(tmp.groups); ctx->group_off.swap(tmp.group_off);
   ctx->elem_base.swap(tmp.elem_base); ctx->n_elem_total = tmp.n_elem_total;
+  ctx->slot_base.swap(tmp.slot_base); ctx->n_slots = tmp.n_slots;
   ctx->features = 0;
   ctx->layout.swap(tmp.layout);
   ctx->bitmap_words = tmp.bitmap_words; ctx->hit_words = tmp.hit_words;
@@ -425,7 +462,8 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
 DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx* ctx, uint32_t features) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state != S_LOADED) return fail(ctx, DRGPUM_ESTATE, "set_features must follow objects_load and precede workspace_bind");
-  if (features & ~uint32_t(DRGPUM_FEATURE_STRUCTURED)) return fail(ctx, DRGPUM_EINVAL, "unknown feature bits");
+  if (features & ~uint32_t(DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY))
+    return fail(ctx, DRGPUM_EINVAL, "unknown feature bits");
   ctx->features = features;
   return compute_layout(ctx);
 }
@@ -447,6 +485,57 @@ DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx* ctx, uint8_t* h_sa, uint8
   for (uint64_t o = 0; o < ctx->n_obj; ++o) {
     if (h_overlap) h_overlap[o] = ov[o] ? 1 : 0;
     if (h_sa) h_sa[o] = (st[o].n_access_apis >= 2 && !ov[o]) ? 1 : 0;
+  }
+  return DRGPUM_OK;
+}
+
+static drgpum_status frequency_ready(drgpum_ctx* ctx, cudaStream_t st) {
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "frequency before workspace_bind");
+  if (!(ctx->features & DRGPUM_FEATURE_FREQUENCY))
+    return fail(ctx, DRGPUM_ESTATE, "DRGPUM_FEATURE_FREQUENCY was not enabled");
+  uint32_t state[2];
+  CK(cudaMemcpyAsync(state, ctx->ws + ctx->L.fq_state, 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (state[0]) return fail(ctx, DRGPUM_EINVAL, "frequency analysis needs records in API (timestamp) order");
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_frequency(drgpum_ctx* ctx, uint32_t pct, uint32_t* h_count,
+                                          uint32_t* h_first, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  cudaStream_t st = as_stream(stream);
+  drgpum_status r = frequency_ready(ctx, st);
+  if (r != DRGPUM_OK) return r;
+  FreqReduceParams q;
+  q.acc = at<unsigned long long>(ctx, ctx->L.fq_acc);
+  q.slot_base = at<uint64_t>(ctx, ctx->L.fq_slot_base);
+  q.n_hit = at<uint32_t>(ctx, ctx->L.n_hit);
+  q.objs = at<DevObj>(ctx, ctx->L.objs);
+  q.acc_ts = at<uint32_t>(ctx, ctx->L.acc_ts);
+  q.n_obj = ctx->n_obj;
+  q.pct = pct;
+  q.out_count = at<uint32_t>(ctx, ctx->L.fq_out_count);
+  q.out_first = at<uint32_t>(ctx, ctx->L.fq_out_first);
+  ctx->launches += launch_frequency_reduce(q, ctx->num_sms, st);
+  CK(cudaGetLastError());
+  if (h_count && ctx->n_obj)
+    CK(cudaMemcpyAsync(h_count, q.out_count, 4 * ctx->n_obj, cudaMemcpyDeviceToHost, st));
+  if (h_first && ctx->n_obj)
+    CK(cudaMemcpyAsync(h_first, q.out_first, 4 * ctx->n_obj, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_frequency_slots(drgpum_ctx* ctx, uint64_t* h_acc, uint64_t* n_slots,
+                                                void* stream) {
+  if (!ctx || !n_slots) return DRGPUM_EINVAL;
+  cudaStream_t st = as_stream(stream);
+  drgpum_status r = frequency_ready(ctx, st);
+  if (r != DRGPUM_OK) return r;
+  *n_slots = ctx->n_slots;
+  if (h_acc && ctx->n_slots) {
+    CK(cudaMemcpyAsync(h_acc, ctx->ws + ctx->L.fq_acc, 24 * ctx->n_slots, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
   }
   return DRGPUM_OK;
 }
@@ -491,8 +580,10 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
   if ((r = up(L.tiles, ctx->tiles.data(), sizeof(Tile) * ctx->tiles.size()))) return r;
   if ((r = up(L.groups, ctx->groups.data(), sizeof(Group) * ctx->groups.size()))) return r;
   if ((r = up(L.group_off, ctx->group_off.data(), 4 * ctx->group_off.size()))) return r;
-  if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
+  if (ctx->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY))
     if ((r = up(L.sa_elem_base, ctx->elem_base.data(), 8 * n))) return r;
+  if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
+    if ((r = up(L.fq_slot_base, ctx->slot_base.data(), 8 * n))) return r;
   if ((r = enqueue_reset(ctx, st))) return r;
   // host vectors stay alive in ctx, so the async uploads are safe; make the
   // bind synchronous anyway so callers may immediately reuse their stream
@@ -518,6 +609,8 @@ DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_re
   ctx->launches += launch_attribute(p, ctx->num_sms, as_stream(stream));
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     ctx->launches += launch_structured(sa_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
+  if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
+    ctx->launches += launch_frequency(fq_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
   ctx->final_valid = false;
   CK(cudaGetLastError());
   return DRGPUM_OK;
@@ -555,6 +648,8 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
     ctx->launches += launch_attribute(p, ctx->num_sms, st);
     if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
       ctx->launches += launch_structured(sa_params(ctx, stage[b], m), ctx->num_sms, st);
+    if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
+      ctx->launches += launch_frequency(fq_params(ctx, stage[b], m), ctx->num_sms, st);
     CK(cudaEventRecord(ctx->ev_used[b], st));
   }
   CK(cudaStreamSynchronize(ctx->copy_stream));

@@ -82,6 +82,31 @@ struct SaParams {
   unsigned long long* q_count;
 };
 
+// NEXT-2 non-uniform access frequency pass (optional feature).
+struct FreqRange { uint64_t g_lo, g_hi, slot; uint32_t tag, pad; };   // 32 B
+struct FreqParams {
+  AttrParams a;                  // records, object table, index, rank table
+  unsigned long long* cells;     // [sum n_elem] (API tag << 32) | count within that API
+  const uint64_t* elem_base;     // [n_obj] first global element of each object
+  const uint64_t* slot_base;     // [n_obj] first (object, access API) slot of each object
+  unsigned long long* acc;       // [n_slots][3]: n touched elements, S1 = sum f, S2 = sum f^2
+  FreqRange* q;
+  uint32_t q_cap;
+  unsigned long long* q_count;
+  uint32_t* state;               // [0] records not sorted by ts, [1] last ts of the previous call
+};
+struct FreqReduceParams {
+  const unsigned long long* acc;
+  const uint64_t* slot_base;
+  const uint32_t* n_hit;         // [n_obj] slots per object
+  const DevObj* objs;
+  const uint32_t* acc_ts;
+  uint64_t n_obj;
+  uint32_t pct;
+  uint32_t* out_count;           // [n_obj] APIs at which the object matches NUAF
+  uint32_t* out_first;           // [n_obj] first such timestamp (kNever if none)
+};
+
 struct FinalParams {
   const uint32_t* orw;
   const Tile* tiles;
@@ -108,6 +133,8 @@ struct FinalParams {
 // Launchers (return the number of kernels enqueued).
 int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);
 int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
+int launch_frequency(const FreqParams& p, int num_sms, cudaStream_t s);
+int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t s);
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
 int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src,

@@ -38,7 +38,7 @@ class Session:
     kinds:   uint8 array, the GPU-API kind of every timestamp.
     """
 
-    def __init__(self, objects, kinds, device=None, structured=False):
+    def __init__(self, objects, kinds, device=None, structured=False, frequency=False):
         if not torch.cuda.is_available():
             raise RuntimeError("drgpum Session needs a CUDA device (there is no CPU fallback)")
         self.L = _lib.load()
@@ -55,8 +55,9 @@ class Session:
         check(self._h, st)
         check(self._h, self.L.drgpum_objects_load(self._h, _np_ptr(self.objects), self.n_obj,
                                                   _np_ptr(self.kinds), self.kinds.shape[0]))
-        if structured:
-            check(self._h, self.L.drgpum_set_features(self._h, _lib.FEATURE_STRUCTURED))
+        feats = (_lib.FEATURE_STRUCTURED if structured else 0) | (_lib.FEATURE_FREQUENCY if frequency else 0)
+        if feats:
+            check(self._h, self.L.drgpum_set_features(self._h, feats))
         nbytes = ctypes.c_uint64()
         check(self._h, self.L.drgpum_workspace_size(self._h, ctypes.byref(nbytes)))
         self.workspace = torch.empty(max(int(nbytes.value), 256), dtype=torch.uint8,
@@ -148,6 +149,24 @@ class Session:
         ov = np.zeros(self.n_obj, np.uint8)
         check(self._h, self.L.drgpum_structured(self._h, _np_ptr(sa), _np_ptr(ov), _stream_handle(stream)))
         return sa, ov
+
+    def frequency(self, pct=20, stream=None):
+        """NEXT-2: (count u32[n_obj], first_ts u32[n_obj]) of the APIs at which
+        each object matches non-uniform access frequency; needs frequency=True."""
+        cnt = np.zeros(self.n_obj, np.uint32)
+        first = np.zeros(self.n_obj, np.uint32)
+        check(self._h, self.L.drgpum_frequency(self._h, pct, _np_ptr(cnt), _np_ptr(first),
+                                               _stream_handle(stream)))
+        return cnt, first
+
+    def frequency_slots(self, stream=None):
+        """NEXT-2 raw sums: u64[n_slots, 3] = (n, S1, S2) per (object, access API)."""
+        n = ctypes.c_uint64()
+        check(self._h, self.L.drgpum_frequency_slots(self._h, None, ctypes.byref(n), _stream_handle(stream)))
+        out = np.zeros((n.value, 3), np.uint64)
+        check(self._h, self.L.drgpum_frequency_slots(self._h, _np_ptr(out), ctypes.byref(n),
+                                                     _stream_handle(stream)))
+        return out
 
     def redundant_allocations(self, pct=10, stream=None):
         """NEXT-1: [(reuser, donor), ...] from this session's first/last uses."""
