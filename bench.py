@@ -47,6 +47,7 @@ def args_():
     ap.add_argument("--records", type=int, default=None, help="override the record count")
     ap.add_argument("--e2e-steps", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-next", action="store_true", help="skip the SURVEY §8(f) NEXT-row timings")
     ap.add_argument("--cpu-sample", type=int, default=None,
                     help="records in the oracle's timed sample (default: whole workload up to 1e8)")
     ap.add_argument("--ref-sample", type=int, default=8_000_000,
@@ -152,6 +153,64 @@ def reference_arm(a):
     }), flush=True)
 
 
+def next_rows(prog, d_recs, plain_attr_ms, reps=5):
+    """SURVEY §8(f) rows on the same resident trace, each timed on its own
+    (not part of the step): NEXT-3 SA and NEXT-2 NUAF as the extra device time
+    their passes add to drgpum_trace_attribute (CUDA events), NEXT-1 RA and
+    NEXT-4 (graph + Kahn + patterns on T, 8 streams) as host wall time of the
+    synchronous C-ABI calls."""
+    import torch
+    from paper_conf_asplos_linzs23_b200 import Session
+    from tracegen.streams import assign_streams
+    stream = torch.cuda.current_stream()
+    N = prog.n_records
+    out = {}
+    for name, kw, query in (("NEXT-3 structured access", {"structured": True}, lambda s: s.structured()),
+                            ("NEXT-2 non-uniform access frequency", {"frequency": True},
+                             lambda s: s.frequency(20))):
+        s = Session(prog.objects, prog.kinds, **kw)
+        for _ in range(2):
+            s.reset(); s.attribute(d_recs); query(s)
+        torch.cuda.synchronize()
+        ms = []
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.reset()
+            e0.record(stream)
+            s.attribute(d_recs)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms.append(e0.elapsed_time(e1))
+        w0 = time.perf_counter()
+        query(s)
+        q_ms = (time.perf_counter() - w0) * 1e3
+        m = float(np.median(ms))
+        out[name] = {"attribute_with_pass_ms": m, "pass_ms": m - plain_attr_ms,
+                     "records_per_s_pass": N / ((m - plain_attr_ms) / 1e3) if m > plain_attr_ms else None,
+                     "pass_gbs_records_only": 16.0 * N / ((m - plain_attr_ms) / 1e3) / 1e9
+                     if m > plain_attr_ms else None,
+                     "query_ms": q_ms}
+        del s
+        torch.cuda.empty_cache()
+    s = Session(prog.objects, prog.kinds)
+    s.attribute(d_recs)
+    s.object_stats()
+    w0 = time.perf_counter()
+    pairs = s.redundant_allocations(10)
+    out["NEXT-1 redundant allocation"] = {"ms": (time.perf_counter() - w0) * 1e3, "pairs": len(pairs)}
+    streams = assign_streams(prog.n_api, 8, 0)
+    s.dependency_graph(streams)
+    w0 = time.perf_counter()
+    T, src, dst, lab = s.dependency_graph(streams)
+    g_ms = (time.perf_counter() - w0) * 1e3
+    w0 = time.perf_counter()
+    s.patterns_topo(T)
+    out["NEXT-4 multi-stream graph + Kahn"] = {
+        "graph_and_levels_ms": g_ms, "patterns_topo_ms": (time.perf_counter() - w0) * 1e3,
+        "streams": 8, "edges": int(src.shape[0]), "levels": int(T.max()) + 1 if T.size else 0}
+    return out
+
+
 def main():
     a = args_()
     if a.impl == "reference":
@@ -254,6 +313,9 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_s = float(t[0])
     clocks = clk.stop()
+    nxt = None
+    if world == 1 and not a.no_next:
+        nxt = next_rows(prog, d_recs, float(ph_mean[1]))
 
     if rank != 0:
         dist.destroy_process_group()
@@ -308,6 +370,7 @@ def main():
         "counters": {k: int(ctr[k]) for k in ctr.dtype.names},
         "attribution_paths_tiles": paths,
         "wall_s_device_region": wall_dev,
+        "next": nxt,
     }
     print(json.dumps(line), flush=True)
     if world > 1:

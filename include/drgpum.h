@@ -309,6 +309,52 @@ DRGPUM_API drgpum_status drgpum_redundant_pairs(const uint64_t *sizes, const uin
 DRGPUM_API drgpum_status drgpum_redundant_alloc(drgpum_ctx *ctx, uint32_t pct,
     uint32_t *reuser, uint32_t *donor, uint64_t cap, uint64_t *n_pairs, void *stream);
 
+/* NEXT-4 multi-stream GPU applications (§5.3 l.273-297).
+ *
+ * Dependency graph G = (V, E) of Definition 5.1 (l.277-286): the vertices are
+ * the timeline's APIs (timestamps 0..n_api-1 in invocation order, the value
+ * access records carry [R22]); an edge i -> j exists when j is i's immediate
+ * successor on the same stream (INTRA, l.281) or when, on some object, i
+ * allocates/writes and j reads with no write in between (RAW, l.283), i
+ * allocates/writes and j frees/writes with no access in between (WAW,
+ * l.284), or i reads and j frees/writes with no write in between (WAR,
+ * l.285).  Reads and writes are the per-(object, API) read/write sets the
+ * attribution found [R24].  Kahn's algorithm with a global T (l.295) assigns
+ * every vertex its topological level: T = 0 for in-degree-zero vertices, and
+ * each round of deletions increments T. */
+enum {
+  DRGPUM_DEP_INTRA = 1,     /* same stream, immediate successor (l.281) */
+  DRGPUM_DEP_RAW = 2,       /* read-after-write (l.283) */
+  DRGPUM_DEP_WAW = 4,       /* write/free-after-write (l.284) */
+  DRGPUM_DEP_WAR = 8        /* write/free-after-read (l.285) */
+};
+
+/* Kahn levels of an arbitrary edge list (src[k] -> dst[k], vertices < n_api;
+ * duplicates allowed).  h_T: u32[n_api] out.  Host only, synchronous.
+ * EINVAL on NULL pointers, an out-of-range vertex, or a cycle. */
+DRGPUM_API drgpum_status drgpum_kahn_levels(uint32_t n_api, const uint32_t *src,
+    const uint32_t *dst, uint64_t n_edges, uint32_t *h_T);
+
+/* Build G for the trace attributed so far and level it.  h_stream: u32[n_api]
+ * stream id of every API (any values; equal ids = same stream).  Outputs
+ * (each may be NULL): h_T u32[n_api] the Kahn timestamps; up to cap edges in
+ * (src, dst) order, duplicates merged with their labels OR-ed (h_src, h_dst
+ * u32, h_label u8 DRGPUM_DEP_* bits); *n_edges (required) the edge count.
+ * Synchronous (copies the hit rows to the host). */
+DRGPUM_API drgpum_status drgpum_dependency_graph(drgpum_ctx *ctx, const uint32_t *h_stream,
+    uint32_t *h_T, uint32_t *h_src, uint32_t *h_dst, uint8_t *h_label, uint64_t cap,
+    uint64_t *n_edges, void *stream);
+
+/* Pattern reports on topological timestamps h_T (u32[n_api], each < n_api,
+ * e.g. drgpum_dependency_graph's).  EA / LD / TI / DW and their distances are
+ * evaluated with an object's accesses ordered by (T, timestamp), "between"
+ * counting every API whose T lies strictly between [R23], distances = T
+ * differences (l.297); UA / ML / OA / OA_ACTIONABLE are time-free and equal
+ * drgpum_patterns'.  With T = the invocation index this is drgpum_patterns.
+ * Synchronous; EINVAL on NULL / out-of-range T. */
+DRGPUM_API drgpum_status drgpum_patterns_topo(drgpum_ctx *ctx, const uint32_t *h_T,
+    const drgpum_thresholds_t *th, drgpum_pattern_report_t *h_out, void *stream);
+
 /* Message for the last failed call on ctx (never NULL). */
 DRGPUM_API const char *drgpum_last_error(const drgpum_ctx *ctx);
 

@@ -13,10 +13,11 @@ It never imports the CPU oracle (oracle/ is test infrastructure only).
 """
 from ._lib import (OBJECT_DTYPE, RECORD_DTYPE, STATS_DTYPE, REPORT_DTYPE, COUNTERS_DTYPE,
                    LAYOUT_DTYPE, NEVER, EA, LD, UA, ML, TI, DW, OA, OA_ACTIONABLE,
-                   FLAG_NAMES, DrgpumError, EXPORTS, LIB_PATH, load, redundant_pairs)
+                   FLAG_NAMES, DrgpumError, EXPORTS, LIB_PATH, load, redundant_pairs, kahn_levels,
+                   DEP_INTRA, DEP_RAW, DEP_WAW, DEP_WAR)
 from .session import Session
 
 __all__ = ["Session", "OBJECT_DTYPE", "RECORD_DTYPE", "STATS_DTYPE", "REPORT_DTYPE",
            "COUNTERS_DTYPE", "LAYOUT_DTYPE", "NEVER", "EA", "LD", "UA", "ML", "TI", "DW",
            "OA", "OA_ACTIONABLE", "FLAG_NAMES", "DrgpumError", "EXPORTS", "LIB_PATH", "load",
-           "redundant_pairs"]
+           "redundant_pairs", "kahn_levels", "DEP_INTRA", "DEP_RAW", "DEP_WAW", "DEP_WAR"]

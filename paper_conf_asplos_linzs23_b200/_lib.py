@@ -31,6 +31,7 @@ assert STATS_DTYPE.itemsize == 56 and REPORT_DTYPE.itemsize == 32 and LAYOUT_DTY
 NEVER = 0xFFFFFFFF
 FEATURE_STRUCTURED = 1
 FEATURE_FREQUENCY = 2
+DEP_INTRA, DEP_RAW, DEP_WAW, DEP_WAR = 1, 2, 4, 8
 API_ALLOC, API_FREE, API_MEMCPY, API_MEMSET, API_KERNEL = 0, 1, 2, 3, 4
 EA, LD, UA, ML, TI, DW, OA, OA_ACTIONABLE = 1, 2, 4, 8, 16, 32, 64, 128
 FLAG_NAMES = {EA: "EA", LD: "LD", UA: "UA", ML: "ML", TI: "TI", DW: "DW", OA: "OA",
@@ -66,7 +67,8 @@ EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_set_features", "drgpu
            "drgpum_trace_attribute_host", "drgpum_shadow_view", "drgpum_object_layout",
            "drgpum_merge_or", "drgpum_finalize", "drgpum_object_stats", "drgpum_patterns",
            "drgpum_consistency_errors", "drgpum_path_stats", "drgpum_redundant_pairs",
-           "drgpum_redundant_alloc", "drgpum_last_error", "drgpum_destroy",
+           "drgpum_redundant_alloc", "drgpum_kahn_levels", "drgpum_dependency_graph",
+           "drgpum_patterns_topo", "drgpum_last_error", "drgpum_destroy",
            "drgpum_launch_count"]
 
 _lib = None
@@ -105,6 +107,9 @@ def load():
         "drgpum_frequency_slots": ([P, P, ctypes.POINTER(U64), P], I),
         "drgpum_redundant_pairs": ([P, P, P, P, U64, U32, P, P, U64, ctypes.POINTER(U64)], I),
         "drgpum_redundant_alloc": ([P, U32, P, P, U64, ctypes.POINTER(U64), P], I),
+        "drgpum_kahn_levels": ([U32, P, P, U64, P], I),
+        "drgpum_dependency_graph": ([P, P, P, P, P, P, U64, ctypes.POINTER(U64), P], I),
+        "drgpum_patterns_topo": ([P, P, P, P, P], I),
         "drgpum_last_error": ([P], ctypes.c_char_p),
         "drgpum_destroy": ([P], None),
         "drgpum_launch_count": ([P], U64),
@@ -142,3 +147,16 @@ def redundant_pairs(sizes, first, last, used, pct=10):
     L.drgpum_redundant_pairs(p(sizes), p(first), p(last), p(used), n, pct, p(a), p(b), cnt.value,
                              ctypes.byref(cnt))
     return list(zip(a.tolist(), b.tolist()))
+
+
+def kahn_levels(n_api, src, dst):
+    """NEXT-4 host algorithm on a plain edge list: u32[n_api] Kahn levels."""
+    L = load()
+    src = np.ascontiguousarray(src, dtype=np.uint32)
+    dst = np.ascontiguousarray(dst, dtype=np.uint32)
+    T = np.zeros(n_api, np.uint32)
+    p = lambda a: ctypes.c_void_p(a.ctypes.data)
+    st = L.drgpum_kahn_levels(n_api, p(src), p(dst), src.shape[0], p(T))
+    if st:
+        raise DrgpumError(st, "drgpum_kahn_levels")
+    return T

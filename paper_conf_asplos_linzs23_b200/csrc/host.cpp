@@ -24,6 +24,7 @@
 
 #include "../../include/drgpum.h"
 #include "internal.cuh"
+#include "multistream.h"
 
 using namespace drgpum;
 
@@ -828,6 +829,141 @@ DRGPUM_API drgpum_status drgpum_redundant_alloc(drgpum_ctx* ctx, uint32_t pct, u
   s = drgpum_redundant_pairs(sizes.data(), first.data(), last.data(), used.data(), ctx->n_obj, pct,
                              reuser, donor, cap, n_pairs);
   if (s != DRGPUM_OK) return fail(ctx, s, "redundant_pairs: invalid arguments");
+  return DRGPUM_OK;
+}
+
+}  // extern "C"
+
+namespace {
+// Every object's accessing APIs in invocation order with their read/write
+// bits, from the hit rows on the device (CSR: off[n_obj + 1]).
+drgpum_status gather_accesses(drgpum_ctx* ctx, cudaStream_t st, std::vector<uint64_t>& off,
+                              std::vector<uint32_t>& api, std::vector<uint8_t>& rw) {
+  std::vector<uint32_t> hit(ctx->hit_words);
+  if (ctx->hit_words)
+    CK(cudaMemcpyAsync(hit.data(), ctx->ws + ctx->L.orw + 4 * ctx->bitmap_words, 4 * ctx->hit_words,
+                       cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  off.assign(ctx->n_obj + 1, 0);
+  api.clear();
+  rw.clear();
+  for (uint64_t o = 0; o < ctx->n_obj; ++o) {
+    const auto& l = ctx->layout[o];
+    const uint32_t* row = hit.data() + l.hit_word;
+    const uint64_t nw = (2ull * l.n_hit_apis + 31) / 32;
+    for (uint64_t w = 0; w < nw; ++w)
+      for (uint32_t b = row[w]; b;) {
+        const uint32_t slot = uint32_t(w * 16 + (__builtin_ctz(b) >> 1));
+        const uint32_t pair = (row[w] >> (2 * (slot & 15))) & 3u;
+        b &= ~(3u << (2 * (slot & 15)));
+        api.push_back(ctx->acc_ts[l.r_lo + slot]);
+        rw.push_back(uint8_t(pair));
+      }
+    off[o + 1] = api.size();
+  }
+  return DRGPUM_OK;
+}
+}  // namespace
+
+extern "C" {
+
+DRGPUM_API drgpum_status drgpum_dependency_graph(drgpum_ctx* ctx, const uint32_t* h_stream,
+                                                 uint32_t* h_T, uint32_t* h_src, uint32_t* h_dst,
+                                                 uint8_t* h_label, uint64_t cap, uint64_t* n_edges,
+                                                 void* stream) {
+  if (!ctx || !n_edges || (ctx->n_api && !h_stream) || (cap && !h_src && !h_dst && !h_label))
+    return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "dependency_graph before workspace_bind");
+  std::vector<uint64_t> off;
+  std::vector<uint32_t> api;
+  std::vector<uint8_t> rw;
+  drgpum_status s = gather_accesses(ctx, as_stream(stream), off, api, rw);
+  if (s != DRGPUM_OK) return s;
+  std::vector<drgpum_ms::Edge> e;
+  e.reserve(ctx->n_api + 3 * api.size());
+  drgpum_ms::stream_edges(h_stream, ctx->n_api, e);
+  for (uint64_t o = 0; o < ctx->n_obj; ++o)
+    drgpum_ms::object_edges(ctx->objs[o].t_alloc, ctx->objs[o].t_free, api.data() + off[o],
+                            rw.data() + off[o], off[o + 1] - off[o], e);
+  drgpum_ms::canonicalize(e);
+  *n_edges = e.size();
+  for (uint64_t k = 0; k < std::min<uint64_t>(cap, e.size()); ++k) {
+    if (h_src) h_src[k] = e[k].src;
+    if (h_dst) h_dst[k] = e[k].dst;
+    if (h_label) h_label[k] = uint8_t(e[k].label);
+  }
+  if (h_T) {
+    if (!drgpum_ms::kahn(ctx->n_api, e, h_T))   // edges only go forward in time
+      return fail(ctx, DRGPUM_EINVAL, "dependency graph has a cycle");
+  }
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_patterns_topo(drgpum_ctx* ctx, const uint32_t* h_T,
+                                              const drgpum_thresholds_t* th,
+                                              drgpum_pattern_report_t* h_out, void* stream) {
+  if (!ctx || !h_out || (ctx->n_api && !h_T)) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "patterns_topo before workspace_bind");
+  const uint32_t n_api = ctx->n_api;
+  for (uint32_t v = 0; v < n_api; ++v)
+    if (h_T[v] >= n_api) return fail(ctx, DRGPUM_EINVAL, "T[%u] = %u >= n_api", v, h_T[v]);
+  drgpum_thresholds_t t = th ? *th : drgpum_thresholds_t{2, 80, 80};
+  drgpum_status s = drgpum_patterns(ctx, &t, h_out, stream);    // time-free flags
+  if (s != DRGPUM_OK) return s;
+  std::vector<uint64_t> off;
+  std::vector<uint32_t> api;
+  std::vector<uint8_t> rw;
+  s = gather_accesses(ctx, as_stream(stream), off, api, rw);
+  if (s != DRGPUM_OK) return s;
+  // P[L] = number of APIs with T < L; between(a, b) = P[T_b] - P[T_a + 1]
+  std::vector<uint64_t> P(uint64_t(n_api) + 2, 0);
+  for (uint32_t v = 0; v < n_api; ++v) ++P[h_T[v] + 1];
+  for (uint64_t L = 1; L < P.size(); ++L) P[L] += P[L - 1];
+  auto between = [&](uint32_t a, uint32_t b) -> uint64_t {
+    const uint32_t ta = h_T[a], tb = h_T[b];
+    return tb > ta ? P[tb] - P[ta + 1] : 0;
+  };
+  constexpr uint32_t kTime = DRGPUM_EA | DRGPUM_LD | DRGPUM_TI | DRGPUM_DW;
+  std::vector<uint32_t> idx;
+  for (uint64_t o = 0; o < ctx->n_obj; ++o) {
+    drgpum_pattern_report_t& r = h_out[o];
+    r.flags &= ~kTime;
+    r.ea_distance = r.ld_distance = r.ti_ranges = r.ti_max_idle = r.dw_pairs = 0;
+    r.ti_total_idle = 0;
+    const uint64_t n = off[o + 1] - off[o];
+    if (!n) continue;
+    idx.resize(n);
+    std::iota(idx.begin(), idx.end(), uint32_t(off[o]));
+    std::sort(idx.begin(), idx.end(), [&](uint32_t a, uint32_t b) {
+      const uint32_t ta = h_T[api[a]], tb = h_T[api[b]];
+      return ta != tb ? ta < tb : api[a] < api[b];
+    });
+    const auto& ob = ctx->objs[o];
+    const uint32_t f = api[idx.front()], l = api[idx.back()];
+    if (between(ob.t_alloc, f) >= 1) {                                   // Def 3.1
+      r.flags |= DRGPUM_EA;
+      r.ea_distance = h_T[f] - h_T[ob.t_alloc];
+    }
+    if (ob.t_free != DRGPUM_NEVER && between(l, ob.t_free) >= 1) {       // Def 3.2
+      r.flags |= DRGPUM_LD;
+      r.ld_distance = h_T[ob.t_free] - h_T[l];
+    }
+    for (uint64_t k = 1; k < n; ++k) {
+      const uint32_t a = idx[k - 1], b = idx[k];
+      const uint64_t g = between(api[a], api[b]);                       // Def 3.6
+      if (g >= t.ti_min_idle) {
+        ++r.ti_ranges;
+        r.ti_max_idle = std::max<uint32_t>(r.ti_max_idle, uint32_t(g));
+        r.ti_total_idle += g;
+      }
+      const uint8_t ka = ctx->kinds[api[a]], kb = ctx->kinds[api[b]];    // Def 3.7
+      const bool cs_a = ka == DRGPUM_API_MEMCPY || ka == DRGPUM_API_MEMSET;
+      const bool cs_b = kb == DRGPUM_API_MEMCPY || kb == DRGPUM_API_MEMSET;
+      if (cs_a && cs_b && (rw[a] & 2) && (rw[b] & 2)) ++r.dw_pairs;
+    }
+    if (r.ti_ranges) r.flags |= DRGPUM_TI;
+    if (r.dw_pairs) r.flags |= DRGPUM_DW;
+  }
   return DRGPUM_OK;
 }
 

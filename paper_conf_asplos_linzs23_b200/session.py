@@ -49,6 +49,7 @@ class Session:
                                             else objs.view(OBJECT_DTYPE))
         self.kinds = np.ascontiguousarray(kinds, dtype=np.uint8)
         self.n_obj = int(self.objects.shape[0])
+        self.n_api = int(self.kinds.shape[0])
         h = ctypes.c_void_p()
         st = self.L.drgpum_create(self.device.index, ctypes.byref(h))
         self._h = h
@@ -129,6 +130,35 @@ class Session:
         th = _thresholds(thresholds)
         check(self._h, self.L.drgpum_patterns(self._h, ctypes.byref(th), _np_ptr(out),
                                               _stream_handle(stream)))
+        return out
+
+    def dependency_graph(self, streams, stream=None):
+        """NEXT-4: (T u32[n_api], src u32[E], dst u32[E], label u8[E]) of the
+        Def 5.1 graph for API stream ids ``streams``."""
+        streams = np.ascontiguousarray(streams, dtype=np.uint32)
+        if streams.shape[0] != self.n_api:
+            raise ValueError("streams must have one entry per API")
+        n = ctypes.c_uint64()
+        T = np.zeros(self.n_api, np.uint32)
+        check(self._h, self.L.drgpum_dependency_graph(self._h, _np_ptr(streams), None, None, None, None,
+                                                      0, ctypes.byref(n), _stream_handle(stream)))
+        src = np.zeros(n.value, np.uint32)
+        dst = np.zeros(n.value, np.uint32)
+        lab = np.zeros(n.value, np.uint8)
+        check(self._h, self.L.drgpum_dependency_graph(self._h, _np_ptr(streams), _np_ptr(T), _np_ptr(src),
+                                                      _np_ptr(dst), _np_ptr(lab), n.value,
+                                                      ctypes.byref(n), _stream_handle(stream)))
+        return T, src, dst, lab
+
+    def patterns_topo(self, T, thresholds=None, stream=None):
+        """NEXT-4: pattern reports on topological timestamps T (u32[n_api])."""
+        T = np.ascontiguousarray(T, dtype=np.uint32)
+        if T.shape[0] != self.n_api:
+            raise ValueError("T must have one entry per API")
+        out = np.zeros(self.n_obj, dtype=REPORT_DTYPE)
+        th = _thresholds(thresholds)
+        check(self._h, self.L.drgpum_patterns_topo(self._h, _np_ptr(T), ctypes.byref(th), _np_ptr(out),
+                                                   _stream_handle(stream)))
         return out
 
     def consistency_errors(self, stream=None):

@@ -153,3 +153,30 @@ def test_edges_forward_and_levels_consistent(seed):
             writes = v == ev[-1] and obj["t_free"] != NEVER or acc[o].get(v, (0, 0))[1]
             if writes:
                 assert all(T[u] < T[v] for u in ev[:i])
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_library_kahn_levels_host(seed):
+    """drgpum_kahn_levels (product, host code) == the literal oracle."""
+    from paper_conf_asplos_linzs23_b200 import kahn_levels as lib_kahn
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(1, 300))
+    m = int(rng.integers(0, 4 * n))
+    a = rng.integers(0, n, m)
+    b = rng.integers(0, n, m)
+    keep = a != b
+    src, dst = np.minimum(a, b)[keep], np.maximum(a, b)[keep]
+    perm = rng.permutation(len(src))          # any order, duplicates included
+    T = lib_kahn(n, src[perm], dst[perm])
+    assert T.tolist() == kahn_levels(n, {(int(x), int(y)): 1 for x, y in zip(src, dst)})
+
+
+def test_library_kahn_rejects_cycles_and_bad_vertices():
+    from paper_conf_asplos_linzs23_b200 import kahn_levels as lib_kahn, DrgpumError
+    with pytest.raises(DrgpumError):
+        lib_kahn(3, [0, 1, 2], [1, 2, 0])
+    with pytest.raises(DrgpumError):
+        lib_kahn(3, [0], [3])
+    with pytest.raises(DrgpumError):
+        lib_kahn(2, [1], [1])
+    assert lib_kahn(0, [], []).size == 0

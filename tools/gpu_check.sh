@@ -14,9 +14,9 @@ tail -3 $OUT/smoke.log
 timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err; echo "bench rc=$?"
 cat $OUT/bench.json; tail -5 $OUT/bench.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
-    python bench.py --steps 3 --warmup 3 --e2e-steps 1 --no-cpu-baseline > $OUT/ncu_bench.log 2>&1; echo "ncu list rc=$?"
+    python bench.py --steps 3 --warmup 3 --e2e-steps 1 --no-cpu-baseline --no-next > $OUT/ncu_bench.log 2>&1; echo "ncu list rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:attribute_kernel -s 3 -c 1 \
-    -o $OUT/attr python bench.py --steps 1 --warmup 3 --e2e-steps 1 --no-cpu-baseline > $OUT/ncu_full.log 2>&1; echo "ncu full rc=$?"
+    -o $OUT/attr python bench.py --steps 1 --warmup 3 --e2e-steps 1 --no-cpu-baseline --no-next > $OUT/ncu_full.log 2>&1; echo "ncu full rc=$?"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:"tile_reduce|object_finalize|range_expand" -s 6 -c 3 \
-    -o $OUT/fin python bench.py --steps 1 --warmup 3 --e2e-steps 1 --no-cpu-baseline > $OUT/ncu_fin.log 2>&1; echo "ncu fin rc=$?"
+    -o $OUT/fin python bench.py --steps 1 --warmup 3 --e2e-steps 1 --no-cpu-baseline --no-next > $OUT/ncu_fin.log 2>&1; echo "ncu fin rc=$?"
 ls -la $OUT
