@@ -691,11 +691,15 @@ namespace drgpum {
 // claimed element e (a CAS from 0); an API that finds another API's tag on an
 // element marks O as overlapped.  Values only go 0 -> tag, so a stale plain
 // read is either 0 (then the CAS decides) or already final.
-__device__ __forceinline__ void sa_claim(uint32_t* owner, uint32_t* overlap, uint64_t g, uint32_t tag,
+__device__ __forceinline__ bool sa_claim(uint32_t* owner, uint32_t* overlap, uint64_t g, uint32_t tag,
                                          uint32_t obj) {
   uint32_t cur = owner[g];
   if (cur == 0) cur = atomicCAS(owner + g, 0u, tag);
-  if (cur != 0 && cur != tag) red_or(overlap + obj, 1u);
+  if (cur == 0 || cur == tag) return false;
+  // one writer per object in the common case: the flag is read (L2) first so
+  // that threads arriving after it is set do not serialise on its address
+  if (!__ldcg(overlap + obj)) red_or(overlap + obj, 1u);
+  return true;
 }
 
 constexpr uint32_t kSaInline = 64;          // elements claimed by the lane itself
@@ -709,6 +713,7 @@ __global__ void __launch_bounds__(256) structured_kernel(const __grid_constant__
   // long, so consecutive records of one thread still share objects
   uint64_t c_base = 0, c_size = 0, c_eb = 0;
   uint32_t c_ta = 0, c_tf = 0, c_obj = kNone, c_shift = 0;
+  bool c_dead = false;                        // cached object already overlapped: SA decided
   for (uint64_t i = tid; i < p.n; i += nth) {
     const uint4 r = p.recs[i];
     const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
@@ -723,13 +728,15 @@ __global__ void __launch_bounds__(256) structured_kernel(const __grid_constant__
       if (ts >= d.t_free) continue;
       c_base = d.base; c_size = d.end - d.base; c_ta = d.t_alloc; c_tf = d.t_free;
       c_obj = o; c_shift = d.shift; c_eb = __ldg(q.elem_base + o);
+      c_dead = __ldcg(q.overlap + o) != 0;
     }
+    if (c_dead) continue;
     const uint64_t off = addr - c_base;
     const uint64_t end = min(off + size, c_size);
     const uint64_t e0 = off >> c_shift, e1 = (end - 1) >> c_shift;
     const uint32_t tag = rank + 1;
     if (e1 - e0 < kSaInline) {
-      for (uint64_t e = e0; e <= e1; ++e) sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
+      for (uint64_t e = e0; e <= e1 && !c_dead; ++e) c_dead = sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
       continue;
     }
     const uint64_t nch = (e1 - e0) / kSaChunk + 1;
@@ -739,7 +746,7 @@ __global__ void __launch_bounds__(256) structured_kernel(const __grid_constant__
       if (slot + k < q.q_cap) {
         q.q[slot + k] = SaRange{c_eb + lo, c_eb + hi, c_obj, tag, {0, 0}};
       } else {
-        for (uint64_t e = lo; e <= hi; ++e) sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
+        for (uint64_t e = lo; e <= hi && !c_dead; ++e) c_dead = sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
       }
     }
   }
@@ -753,7 +760,12 @@ __global__ void __launch_bounds__(256) structured_range_kernel(const __grid_cons
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
   for (uint64_t e = gwarp; e < cnt; e += nwarps) {
     const SaRange r = q.q[e];
-    for (uint64_t g = r.g_lo + lane; g <= r.g_hi; g += 32) sa_claim(q.owner, q.overlap, g, r.tag, r.obj);
+    if (__ldcg(q.overlap + r.obj)) continue;
+    for (uint64_t b = r.g_lo; b <= r.g_hi; b += 32) {     // warp-uniform trip count
+      const uint64_t g = b + lane;
+      const bool hit = g <= r.g_hi && sa_claim(q.owner, q.overlap, g, r.tag, r.obj);
+      if (__any_sync(0xffffffffu, hit)) break;
+    }
   }
 }
 

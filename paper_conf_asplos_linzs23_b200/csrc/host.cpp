@@ -40,6 +40,7 @@ struct Layout {
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
   // NEXT-2 frequency (feature): cells[sum n_elem], acc[n_slots][3], state, queue, outputs
   uint64_t fq_cells, fq_acc, fq_state, fq_qcount, fq_end, fq_slot_base, fq_q, fq_out_count, fq_out_first;
+  uint64_t fq_seg, fq_seg_count;
   uint64_t total;
 };
 
@@ -309,7 +310,7 @@ drgpum_status compute_layout(drgpum_ctx* c) {
     L.sa_q = put(sizeof(SaRange) * c->sa_q_cap);
   }
   L.fq_cells = L.fq_acc = L.fq_state = L.fq_qcount = L.fq_end = off;
-  L.fq_slot_base = L.fq_q = L.fq_out_count = L.fq_out_first = off;
+  L.fq_slot_base = L.fq_q = L.fq_out_count = L.fq_out_first = L.fq_seg = L.fq_seg_count = off;
   if (c->features & DRGPUM_FEATURE_FREQUENCY) {
     L.fq_cells = put(8 * c->n_elem_total);
     L.fq_acc = put(24 * c->n_slots);
@@ -318,6 +319,8 @@ drgpum_status compute_layout(drgpum_ctx* c) {
     L.fq_end = off;                           // [fq_cells, fq_end) is zeroed per trace
     L.fq_slot_base = put(8 * n);
     L.fq_q = put(sizeof(FreqRange) * c->sa_q_cap);
+    L.fq_seg = put(16 * (uint64_t(c->n_api) + 2));
+    L.fq_seg_count = put(4 * (uint64_t(c->num_sms) * 8 + 2));
     L.fq_out_count = put(4 * n);
     L.fq_out_first = put(4 * n);
   }
@@ -395,6 +398,8 @@ FreqParams fq_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   q.q_cap = c->sa_q_cap;
   q.q_count = at<unsigned long long>(c, c->L.fq_qcount);
   q.state = at<uint32_t>(c, c->L.fq_state);
+  q.seg = at<uint64_t>(c, c->L.fq_seg);
+  q.seg_count = at<uint32_t>(c, c->L.fq_seg_count);
   return q;
 }
 

@@ -94,6 +94,8 @@ struct FreqParams {
   uint32_t q_cap;
   unsigned long long* q_count;
   uint32_t* state;               // [0] records not sorted by ts, [1] last ts of the previous call
+  uint64_t* seg;                 // [2 (n_api + 2)] scratch: run start per ts | compacted run starts
+  uint32_t* seg_count;           // [max grid blocks + 2] scratch for the compaction
 };
 struct FreqReduceParams {
   const unsigned long long* acc;
