@@ -6,7 +6,7 @@
  * analysis (Lin, Zhou, Su, ASPLOS '23).  "P:NNN" cites line NNN of the paper
  * text (/root/reference/PAPER.md at build time; the text is not needed at run
  * time).  Readings of the paper where it is silent or ambiguous are the
- * numbered items R1..R18 of DESIGN.md §"Readings".
+ * numbered items R1..R27 of DESIGN.md §"Readings".
  *
  *   objects + GPU-API timeline  --drgpum_objects_load-->  memory map M as a
  *       static segment index (§5.1)
@@ -313,13 +313,13 @@ DRGPUM_API drgpum_status drgpum_redundant_alloc(drgpum_ctx *ctx, uint32_t pct,
  *
  * Dependency graph G = (V, E) of Definition 5.1 (l.277-286): the vertices are
  * the timeline's APIs (timestamps 0..n_api-1 in invocation order, the value
- * access records carry [R22]); an edge i -> j exists when j is i's immediate
+ * access records carry [R24]); an edge i -> j exists when j is i's immediate
  * successor on the same stream (INTRA, l.281) or when, on some object, i
  * allocates/writes and j reads with no write in between (RAW, l.283), i
  * allocates/writes and j frees/writes with no access in between (WAW,
  * l.284), or i reads and j frees/writes with no write in between (WAR,
  * l.285).  Reads and writes are the per-(object, API) read/write sets the
- * attribution found [R24].  Kahn's algorithm with a global T (l.295) assigns
+ * attribution found [R25].  Kahn's algorithm with a global T (l.295) assigns
  * every vertex its topological level: T = 0 for in-degree-zero vertices, and
  * each round of deletions increments T. */
 enum {
@@ -348,7 +348,7 @@ DRGPUM_API drgpum_status drgpum_dependency_graph(drgpum_ctx *ctx, const uint32_t
 /* Pattern reports on topological timestamps h_T (u32[n_api], each < n_api,
  * e.g. drgpum_dependency_graph's).  EA / LD / TI / DW and their distances are
  * evaluated with an object's accesses ordered by (T, timestamp), "between"
- * counting every API whose T lies strictly between [R23], distances = T
+ * counting every API whose T lies strictly between [R26], distances = T
  * differences (l.297); UA / ML / OA / OA_ACTIONABLE are time-free and equal
  * drgpum_patterns'.  With T = the invocation index this is drgpum_patterns.
  * Synchronous; EINVAL on NULL / out-of-range T. */

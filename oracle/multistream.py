@@ -10,10 +10,10 @@ Follows PAPER.md §5.3 literally:
     in-degree-zero vertices of a round get the same T;
   * ``patterns_topo``      -- the time-dependent patterns (EA Def 3.1, LD Def
     3.2, TI Def 3.6, DW Def 3.7) with "between" counted over all APIs whose T
-    lies strictly between (R23) and distances as T differences
+    lies strictly between (R26) and distances as T differences
     (l.297 "computing the difference between their timestamps").
 
-Readings (R22-R25): vertices are the APIs in invocation order (the
+Readings (R24-R27): vertices are the APIs in invocation order (the
 index the records carry); an object's events are its ALLOC (a write that
 "allocates"), its accessing APIs with the read/write flags the attribution
 found, and its FREE (a "free"); "following v_i and before v_j" is invocation

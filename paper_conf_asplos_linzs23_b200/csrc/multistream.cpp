@@ -2,13 +2,13 @@
 // Def 5.1 l.277-286, algorithm l.295, Fig. 4 l.291-297).
 //
 // Vertices are the GPU APIs in invocation order (the timestamp every access
-// record carries, reading R22).  Data edges come from the attribution's
+// record carries, reading R24).  Data edges come from the attribution's
 // per-(object, API) read/write sets -- the hit rows the kernels build -- so
 // the graph costs O(accesses) per object instead of the paper's per-API
 // shadow-memory lookups.  One left-to-right pass per object keeps the last
 // writer (the ALLOC counts as one), whether any accessor followed it, and the
 // readers since it; that is exactly Def 5.1's "no v_k (reads/)writes O_x
-// following v_i and before v_j" conditions (R24):
+// following v_i and before v_j" conditions (R25):
 //   RAW  last writer            -> every reader
 //   WAR  each reader since the last write (the writer itself if it reads)
 //                               -> the next writer / the FREE
