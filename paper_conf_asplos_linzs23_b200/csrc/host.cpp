@@ -39,8 +39,8 @@ struct Layout {
   // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
   // NEXT-2 frequency (feature): cells[sum n_elem], acc[n_slots][3], state, queue, outputs
-  uint64_t fq_cells, fq_acc, fq_state, fq_qcount, fq_end, fq_slot_base, fq_q, fq_out_count, fq_out_first;
-  uint64_t fq_seg, fq_seg_count;
+  uint64_t fq_cells, fq_acc, fq_state, fq_q, fq_end, fq_slot_base, fq_out_count, fq_out_first;
+  uint64_t fq_ctl, fq_run_start, fq_segs, fq_seg_of_ts, fq_seg_left;
   uint64_t total;
 };
 
@@ -309,18 +309,21 @@ drgpum_status compute_layout(drgpum_ctx* c) {
     L.sa_end = off;                           // [sa_owner, sa_end) is zeroed per trace
     L.sa_q = put(sizeof(SaRange) * c->sa_q_cap);
   }
-  L.fq_cells = L.fq_acc = L.fq_state = L.fq_qcount = L.fq_end = off;
-  L.fq_slot_base = L.fq_q = L.fq_out_count = L.fq_out_first = L.fq_seg = L.fq_seg_count = off;
+  L.fq_cells = L.fq_acc = L.fq_state = L.fq_q = L.fq_end = off;
+  L.fq_slot_base = L.fq_out_count = L.fq_out_first = off;
+  L.fq_ctl = L.fq_run_start = L.fq_segs = L.fq_seg_of_ts = L.fq_seg_left = off;
   if (c->features & DRGPUM_FEATURE_FREQUENCY) {
     L.fq_cells = put(8 * c->n_elem_total);
     L.fq_acc = put(24 * c->n_slots);
-    L.fq_state = put(8);
-    L.fq_qcount = put(8);
+    L.fq_state = put(16);
+    L.fq_q = put(sizeof(FreqChunk) * c->sa_q_cap);
     L.fq_end = off;                           // [fq_cells, fq_end) is zeroed per trace
     L.fq_slot_base = put(8 * n);
-    L.fq_q = put(sizeof(FreqRange) * c->sa_q_cap);
-    L.fq_seg = put(16 * (uint64_t(c->n_api) + 2));
-    L.fq_seg_count = put(4 * (uint64_t(c->num_sms) * 8 + 2));
+    L.fq_ctl = put(sizeof(FreqCtl));
+    L.fq_run_start = put(8 * (uint64_t(c->n_api) + 1));
+    L.fq_segs = put(8 * (uint64_t(c->n_api) + 2));
+    L.fq_seg_of_ts = put(4 * (uint64_t(c->n_api) + 1));
+    L.fq_seg_left = put(4 * (uint64_t(c->n_api) + 1));
     L.fq_out_count = put(4 * n);
     L.fq_out_first = put(4 * n);
   }
@@ -394,12 +397,15 @@ FreqParams fq_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   q.elem_base = at<uint64_t>(c, c->L.sa_elem_base);
   q.slot_base = at<uint64_t>(c, c->L.fq_slot_base);
   q.acc = at<unsigned long long>(c, c->L.fq_acc);
-  q.q = at<FreqRange>(c, c->L.fq_q);
+  q.acc_ts = at<uint32_t>(c, c->L.acc_ts);
+  q.q = at<FreqChunk>(c, c->L.fq_q);
   q.q_cap = c->sa_q_cap;
-  q.q_count = at<unsigned long long>(c, c->L.fq_qcount);
   q.state = at<uint32_t>(c, c->L.fq_state);
-  q.seg = at<uint64_t>(c, c->L.fq_seg);
-  q.seg_count = at<uint32_t>(c, c->L.fq_seg_count);
+  q.ctl = at<FreqCtl>(c, c->L.fq_ctl);
+  q.run_start = at<uint64_t>(c, c->L.fq_run_start);
+  q.segs = at<uint64_t>(c, c->L.fq_segs);
+  q.seg_of_ts = at<uint32_t>(c, c->L.fq_seg_of_ts);
+  q.seg_left = at<uint32_t>(c, c->L.fq_seg_left);
   return q;
 }
 

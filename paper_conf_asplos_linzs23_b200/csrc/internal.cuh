@@ -83,19 +83,25 @@ struct SaParams {
 };
 
 // NEXT-2 non-uniform access frequency pass (optional feature).
-struct FreqRange { uint64_t g_lo, g_hi, slot; uint32_t tag, pad; };   // 32 B
+struct FreqChunk { uint64_t g_lo, g_hi, slot; uint32_t tag, seg, ready, pad; };  // 40 B
+struct FreqCtl {                 // per call, zeroed before the scan
+  unsigned long long n_segs, n_tiles, tile_next, tiles_done, q_head, q_tail, end_valid, rank_first, gen;
+};
 struct FreqParams {
-  AttrParams a;                  // records, object table, index, rank table
+  AttrParams a;                  // records, object table, index, rank table, hit rows
   unsigned long long* cells;     // [sum n_elem] (API tag << 32) | count within that API
   const uint64_t* elem_base;     // [n_obj] first global element of each object
   const uint64_t* slot_base;     // [n_obj] first (object, access API) slot of each object
   unsigned long long* acc;       // [n_slots][3]: n touched elements, S1 = sum f, S2 = sum f^2
-  FreqRange* q;
+  const uint32_t* acc_ts;        // [n_acc] timestamp of each access rank
+  FreqChunk* q;                  // wide-record chunk queue (ready = call generation)
   uint32_t q_cap;
-  unsigned long long* q_count;
-  uint32_t* state;               // [0] records not sorted by ts, [1] last ts of the previous call
-  uint64_t* seg;                 // [2 (n_api + 2)] scratch: run start per ts | compacted run starts
-  uint32_t* seg_count;           // [max grid blocks + 2] scratch for the compaction
+  uint32_t* state;               // [0] records not sorted by ts, [1] last ts of the previous call, [2] generation
+  FreqCtl* ctl;
+  uint64_t* run_start;           // [n_api + 1] run start per ts; [n_api] = start of the invalid tail
+  uint64_t* segs;                // [n_api + 2] segment starts, then the end of the valid records
+  uint32_t* seg_of_ts;           // [n_api] segment index of each ts with records in this call
+  uint32_t* seg_left;            // [n_api + 1] unfinished tile parts / chunks per segment
 };
 struct FreqReduceParams {
   const unsigned long long* acc;
