@@ -40,7 +40,8 @@ struct Layout {
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
   // NEXT-2 frequency (feature): cells[sum n_elem], acc[n_slots][3], state, queue, outputs
   uint64_t fq_cells, fq_acc, fq_state, fq_q, fq_end, fq_slot_base, fq_out_count, fq_out_first;
-  uint64_t fq_ctl, fq_run_start, fq_segs, fq_seg_of_ts, fq_seg_left;
+  uint64_t fq_ctl, fq_run_start, fq_segs, fq_seg_of_ts, fq_seg_touch, fq_seg_off, fq_seg_logcap, fq_solo;
+  uint64_t fq_batch_first, fq_batch_extent, fq_slot_recs, fq_slot_touch, fq_slot_list, fq_table;
   uint64_t total;
 };
 
@@ -122,6 +123,16 @@ drgpum_status set_device(drgpum_ctx* ctx) { CK(cudaSetDevice(ctx->device)); retu
 uint32_t ilog2(uint32_t e) { uint32_t s = 0; while ((1u << s) < e) ++s; return s; }
 
 drgpum_status compute_layout(drgpum_ctx* c);
+
+// NEXT-2 per-API hash tables: entries per batch (power of two).  Small
+// enough that a batch's tables stay resident in L2 (random atomics on
+// DRAM-resident lines run at a few G/s), 2^12 .. 2^21 entries (32 MiB; the
+// table region is twice that)
+uint64_t freq_budget(const drgpum_ctx* c) {
+  uint64_t want = std::max<uint64_t>(2 * c->n_elem_total, 1ull << 12), b = 1;
+  while (b < want && b < (1ull << 21)) b <<= 1;
+  return b;
+}
 
 // Build everything derived from (objects, kinds) on the host.
 drgpum_status build_tables(drgpum_ctx* c) {
@@ -311,7 +322,9 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   }
   L.fq_cells = L.fq_acc = L.fq_state = L.fq_q = L.fq_end = off;
   L.fq_slot_base = L.fq_out_count = L.fq_out_first = off;
-  L.fq_ctl = L.fq_run_start = L.fq_segs = L.fq_seg_of_ts = L.fq_seg_left = off;
+  L.fq_ctl = L.fq_run_start = L.fq_segs = L.fq_seg_of_ts = L.fq_seg_touch = L.fq_seg_off = off;
+  L.fq_seg_logcap = L.fq_solo = L.fq_batch_first = L.fq_batch_extent = off;
+  L.fq_slot_recs = L.fq_slot_touch = L.fq_slot_list = L.fq_table = off;
   if (c->features & DRGPUM_FEATURE_FREQUENCY) {
     L.fq_cells = put(8 * c->n_elem_total);
     L.fq_acc = put(24 * c->n_slots);
@@ -323,7 +336,16 @@ drgpum_status compute_layout(drgpum_ctx* c) {
     L.fq_run_start = put(8 * (uint64_t(c->n_api) + 1));
     L.fq_segs = put(8 * (uint64_t(c->n_api) + 2));
     L.fq_seg_of_ts = put(4 * (uint64_t(c->n_api) + 1));
-    L.fq_seg_left = put(4 * (uint64_t(c->n_api) + 1));
+    L.fq_seg_touch = put(8 * (uint64_t(c->n_api) + 1));
+    L.fq_seg_off = put(8 * (uint64_t(c->n_api) + 1));
+    L.fq_seg_logcap = put(uint64_t(c->n_api) + 1);
+    L.fq_solo = put(4 * (uint64_t(c->n_api) + 1));
+    L.fq_batch_first = put(4 * (uint64_t(kFreqMaxBatches) + 1));
+    L.fq_batch_extent = put(8 * uint64_t(kFreqMaxBatches));
+    L.fq_slot_recs = put(4 * c->n_slots);
+    L.fq_slot_touch = put(8 * c->n_slots);
+    L.fq_slot_list = put(sizeof(FreqSlotSeg) * c->n_slots);
+    L.fq_table = put(2 * sizeof(FreqEntry) * freq_budget(c));
     L.fq_out_count = put(4 * n);
     L.fq_out_first = put(4 * n);
   }
@@ -397,7 +419,6 @@ FreqParams fq_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   q.elem_base = at<uint64_t>(c, c->L.sa_elem_base);
   q.slot_base = at<uint64_t>(c, c->L.fq_slot_base);
   q.acc = at<unsigned long long>(c, c->L.fq_acc);
-  q.acc_ts = at<uint32_t>(c, c->L.acc_ts);
   q.q = at<FreqChunk>(c, c->L.fq_q);
   q.q_cap = c->sa_q_cap;
   q.state = at<uint32_t>(c, c->L.fq_state);
@@ -405,7 +426,18 @@ FreqParams fq_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   q.run_start = at<uint64_t>(c, c->L.fq_run_start);
   q.segs = at<uint64_t>(c, c->L.fq_segs);
   q.seg_of_ts = at<uint32_t>(c, c->L.fq_seg_of_ts);
-  q.seg_left = at<uint32_t>(c, c->L.fq_seg_left);
+  q.seg_touch = at<unsigned long long>(c, c->L.fq_seg_touch);
+  q.seg_off = at<uint64_t>(c, c->L.fq_seg_off);
+  q.seg_logcap = at<uint8_t>(c, c->L.fq_seg_logcap);
+  q.solo = at<uint32_t>(c, c->L.fq_solo);
+  q.batch_first = at<uint32_t>(c, c->L.fq_batch_first);
+  q.batch_extent = at<unsigned long long>(c, c->L.fq_batch_extent);
+  q.max_batches = kFreqMaxBatches;
+  q.slot_recs = at<uint32_t>(c, c->L.fq_slot_recs);
+  q.slot_touch = at<unsigned long long>(c, c->L.fq_slot_touch);
+  q.slot_list = at<FreqSlotSeg>(c, c->L.fq_slot_list);
+  q.table = at<FreqEntry>(c, c->L.fq_table);
+  q.budget = freq_budget(c);
   return q;
 }
 
@@ -508,7 +540,8 @@ static drgpum_status frequency_ready(drgpum_ctx* ctx, cudaStream_t st) {
   uint32_t state[2];
   CK(cudaMemcpyAsync(state, ctx->ws + ctx->L.fq_state, 8, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
-  if (state[0]) return fail(ctx, DRGPUM_EINVAL, "frequency analysis needs records in API (timestamp) order");
+  if (state[0] & 1) return fail(ctx, DRGPUM_EINVAL, "frequency analysis needs records in API (timestamp) order");
+  if (state[0]) return fail(ctx, DRGPUM_ENOMEM, "frequency analysis: per-call table plan overflow (split the call)");
   return DRGPUM_OK;
 }
 
@@ -622,7 +655,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_re
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     ctx->launches += launch_structured(sa_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
-    ctx->launches += launch_frequency(fq_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
+    ctx->launches += launch_frequency(fq_params(ctx, d_recs, n), ctx->n_slots, ctx->num_sms, as_stream(stream));
   ctx->final_valid = false;
   CK(cudaGetLastError());
   return DRGPUM_OK;
@@ -661,7 +694,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
     if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
       ctx->launches += launch_structured(sa_params(ctx, stage[b], m), ctx->num_sms, st);
     if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
-      ctx->launches += launch_frequency(fq_params(ctx, stage[b], m), ctx->num_sms, st);
+      ctx->launches += launch_frequency(fq_params(ctx, stage[b], m), ctx->n_slots, ctx->num_sms, st);
     CK(cudaEventRecord(ctx->ev_used[b], st));
   }
   CK(cudaStreamSynchronize(ctx->copy_stream));

@@ -83,25 +83,39 @@ struct SaParams {
 };
 
 // NEXT-2 non-uniform access frequency pass (optional feature).
-struct FreqChunk { uint64_t g_lo, g_hi, slot; uint32_t tag, seg, ready, pad; };  // 40 B
+struct FreqChunk { uint64_t g_lo, g_hi, slot; uint32_t tag, seg; };   // 32 B wide-record chunk
+struct FreqEntry { unsigned long long key, cnt; };                     // 16 B per-API hash entry
+struct FreqSlotSeg { uint64_t slot; uint32_t seg, pad; };
 struct FreqCtl {                 // per call, zeroed before the scan
-  unsigned long long n_segs, n_tiles, tile_next, tiles_done, q_head, q_tail, end_valid, rank_first, gen;
+  unsigned long long n_segs, end_valid, n_list, q_count, n_batches, n_solo, pad0, pad1;
 };
+constexpr uint8_t kFreqSolo = 0xFF;
+constexpr uint32_t kFreqMaxBatches = 65536;    // seg_logcap: segment counted in the element cells, alone
 struct FreqParams {
-  AttrParams a;                  // records, object table, index, rank table, hit rows
-  unsigned long long* cells;     // [sum n_elem] (API tag << 32) | count within that API
+  AttrParams a;                  // records, object table, index, rank table
+  unsigned long long* cells;     // [sum n_elem] (API tag << 32) | count within that API (solo segments)
   const uint64_t* elem_base;     // [n_obj] first global element of each object
   const uint64_t* slot_base;     // [n_obj] first (object, access API) slot of each object
   unsigned long long* acc;       // [n_slots][3]: n touched elements, S1 = sum f, S2 = sum f^2
-  const uint32_t* acc_ts;        // [n_acc] timestamp of each access rank
-  FreqChunk* q;                  // wide-record chunk queue (ready = call generation)
+  FreqChunk* q;                  // wide-record chunk queue
   uint32_t q_cap;
-  uint32_t* state;               // [0] records not sorted by ts, [1] last ts of the previous call, [2] generation
+  uint32_t max_batches;
+  uint32_t* state;               // [0] records not sorted by ts, [1] last ts of the previous call
   FreqCtl* ctl;
   uint64_t* run_start;           // [n_api + 1] run start per ts; [n_api] = start of the invalid tail
   uint64_t* segs;                // [n_api + 2] segment starts, then the end of the valid records
   uint32_t* seg_of_ts;           // [n_api] segment index of each ts with records in this call
-  uint32_t* seg_left;            // [n_api + 1] unfinished tile parts / chunks per segment
+  unsigned long long* seg_touch; // [n_api + 1] element touches that need the segment's hash table
+  uint64_t* seg_off;             // [n_api + 1] table offset (entries) inside its batch's region
+  uint8_t* seg_logcap;           // [n_api + 1] log2 table capacity, 0 = no table, kFreqSolo
+  uint32_t* solo;                // [n_api + 1] solo segments in trace order
+  uint32_t* batch_first;         // [max_batches + 1] first segment of each batch (kNone if empty)
+  unsigned long long* batch_extent;  // [max_batches] table entries the batch uses
+  uint32_t* slot_recs;           // [n_slots] records per (object, API) slot in this call
+  unsigned long long* slot_touch;    // [n_slots] element touches per slot in this call
+  FreqSlotSeg* slot_list;        // [n_slots] slots touched in this call, with their segment
+  FreqEntry* table;              // [2 * budget] per-API hash tables of one batch
+  uint64_t budget;               // table entries per batch (power of two)
 };
 struct FreqReduceParams {
   const unsigned long long* acc;
@@ -141,7 +155,7 @@ struct FinalParams {
 // Launchers (return the number of kernels enqueued).
 int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);
 int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
-int launch_frequency(const FreqParams& p, int num_sms, cudaStream_t s);
+int launch_frequency(const FreqParams& p, uint64_t n_slots, int num_sms, cudaStream_t s);
 int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t s);
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
