@@ -404,6 +404,27 @@ int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s) {
   return 1;
 }
 
+// Reset of a trace's dynamic state in one pass of 16-B stores: zeros, except
+// the first[] section (16-B units [one_lo, one_hi)), which starts at NEVER.
+__global__ void __launch_bounds__(256) reset_kernel(uint4* __restrict__ ws, uint64_t n16, uint64_t one_lo,
+                                                   uint64_t one_hi) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n16; i += stride) {
+    const uint32_t v = (i >= one_lo && i < one_hi) ? 0xFFFFFFFFu : 0u;
+    ws[i] = make_uint4(v, v, v, v);
+  }
+}
+
+int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_bytes, int num_sms, cudaStream_t s) {
+  const uint64_t n16 = (bytes + 15) / 16;
+  if (!n16) return 0;
+  uint64_t b = (n16 + 255) / 256;
+  if (b > uint64_t(num_sms) * 16) b = uint64_t(num_sms) * 16;
+  reset_kernel<<<(unsigned)b, 256, 0, s>>>(reinterpret_cast<uint4*>(ws), n16, first_off / 16,
+                                            (first_off + first_bytes + 15) / 16);
+  return 1;
+}
+
 // B7: OR n_src received slices into the owned words (after an all-to-all).
 __global__ void __launch_bounds__(256) merge_or_kernel(uint32_t* __restrict__ dst,
     const uint32_t* __restrict__ src, uint32_t n_src, uint64_t stride, uint64_t n_words) {

@@ -379,8 +379,8 @@ drgpum_status validate(drgpum_ctx* c, const drgpum_object_t* objs, uint64_t n_ob
 }
 
 drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s) {
-  CK(cudaMemsetAsync(ctx->ws, 0, ctx->L.dyn_end, s));
-  ctx->launches += launch_fill_u32(at<uint32_t>(ctx, ctx->L.first), kNever, ctx->n_obj, s);
+  // dynamic state: shadow words, last, counters = 0; first = NEVER (one kernel)
+  ctx->launches += launch_reset(ctx->ws, ctx->L.dyn_end, ctx->L.first, 4 * ctx->n_obj, ctx->num_sms, s);
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     CK(cudaMemsetAsync(ctx->ws + ctx->L.sa_owner, 0, ctx->L.sa_end - ctx->L.sa_owner, s));
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)

@@ -159,6 +159,7 @@ int launch_frequency(const FreqParams& p, uint64_t n_slots, int num_sms, cudaStr
 int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t s);
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
+int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_bytes, int num_sms, cudaStream_t s);
 int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src,
                     uint64_t src_stride, uint64_t n_words, int num_sms, cudaStream_t s);
 
