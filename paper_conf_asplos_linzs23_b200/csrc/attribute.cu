@@ -35,47 +35,70 @@ constexpr int kAttrThreads = kConsumerWarps * 32;
 constexpr int kStages = 3;                                   // per-warp ring depth
 constexpr int kTilesPerWarp = 4;                             // 32-record tiles per stage
 constexpr int kWarpRecords = kTilesPerWarp * 32;             // 128 records = 2 KB per stage
-// per block: 8 warps x 3 x 2 KB rings + 4 KB level-1 keys + barriers + 256 x 56 B
-// lane caches + counters = ~66 KB: three blocks (24 warps) per SM with ~26 KB of L1
-constexpr size_t kAttrSmem = size_t(kConsumerWarps) * kStages * kWarpRecords * 16 + kL1MaxKeys * 8 +
-                             size_t(kConsumerWarps) * kStages * 16 + size_t(kAttrThreads) * 56 +
-                             size_t(kConsumerWarps) * 24;
-// Dynamic work units: chunk k of a launch covers records [chunk_start(k),
-// chunk_start(k+1)): big chunks (fewer cache warm-ups at chunk starts) for
-// the first ~80% of the records, small ones at the end (balance).
-constexpr uint64_t kChunkBig = 8192, kChunkSmall = 1024;
-__device__ __forceinline__ uint64_t chunk_start(uint64_t k, uint64_t n) {
-  const uint64_t k_big = (n / 5 * 4) / kChunkBig;
+// Work units: chunk k of a launch covers records [chunk_start(k),
+// chunk_start(k+1)).  Big chunks (fewer cache warm-ups at chunk starts) cover
+// the first kBigPct% of the records, small ones the rest (balance).  With
+// kStatic, the big part is instead one contiguous range per warp, handed out
+// without an atomic (ticket k < W is warp k's range).  Measured on C2 (A/B on
+// one box, tools/ab.sh): 8192/4096 at 80% beats 8192/1024 by 6%, uniform 4096
+// by 5%, uniform 2048 by 16% (each chunk start costs a cache warm-up through
+// the slow path) and the static split by 14% (warps spread over the whole
+// trace touch the whole shadow at once: the REDs' L2 working set grows).
+#ifndef DRGPUM_CHUNK_BIG
+#define DRGPUM_CHUNK_BIG 8192
+#endif
+#ifndef DRGPUM_CHUNK_SMALL
+#define DRGPUM_CHUNK_SMALL 4096
+#endif
+#ifndef DRGPUM_BIG_PCT
+#define DRGPUM_BIG_PCT 80
+#endif
+#ifndef DRGPUM_STATIC
+#define DRGPUM_STATIC 0
+#endif
+constexpr uint64_t kChunkBig = DRGPUM_CHUNK_BIG, kChunkSmall = DRGPUM_CHUNK_SMALL;
+constexpr uint64_t kBigPct = DRGPUM_BIG_PCT;
+constexpr bool kStatic = DRGPUM_STATIC != 0;
+__device__ __forceinline__ uint64_t chunk_start(uint64_t k, uint64_t n, uint32_t n_warps) {
+  if (kStatic) {
+    const uint64_t per = n / 100 * kBigPct / n_warps;
+    return k <= n_warps ? k * per : n_warps * per + (k - n_warps) * kChunkSmall;
+  }
+  const uint64_t k_big = (n / 100 * kBigPct) / kChunkBig;
   return k <= k_big ? k * kChunkBig : k_big * kChunkBig + (k - k_big) * kChunkSmall;
 }
 
 // ------------------------------------------------------------------ PTX helpers
+// Shared memory is addressed through 32-bit shared-window addresses (no
+// generic -> shared conversion in the loop).
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
 }
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-               : "memory");
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
 }
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+// bar + OFF: the constant offset stays an immediate of the instruction (no
+// hoisted, register-resident base per field)
+template <uint32_t OFF>
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   uint32_t done;
   do {
     asm volatile(
-        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-        : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1+%3], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done) : "r"(bar), "r"(parity), "n"(OFF) : "memory");
   } while (!done);
 }
-__device__ __forceinline__ void tma_load_1d(void* smem_dst, const void* gsrc, uint32_t bytes,
-                                            uint64_t* bar, uint64_t policy) {
+__device__ __forceinline__ void tma_load_1d(uint32_t dst, const void* gsrc, uint32_t bytes, uint32_t bar,
+                                            uint64_t policy) {
   asm volatile(
       "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
-      ::"r"(smem_u32(smem_dst)), "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)), "l"(policy) : "memory");
+      ::"r"(dst), "l"(gsrc), "r"(bytes), "r"(bar), "l"(policy) : "memory");
 }
 __device__ __forceinline__ uint64_t evict_first_policy() {
   uint64_t p;
@@ -87,6 +110,41 @@ __device__ __forceinline__ uint4 lds128(uint32_t saddr) {
   asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];"
                : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(saddr));
   return r;
+}
+template <uint32_t OFF>
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(a), "n"(OFF) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t lds64(uint32_t a) {
+  uint64_t v;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts64(uint32_t a, uint64_t v) {
+  asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+template <uint32_t OFF>
+__device__ __forceinline__ void red_shared_add(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0+%2], %1;" ::"r"(a), "r"(v), "n"(OFF) : "memory");
+}
+// Work cursor: u32 chunk tickets (the low half of the u64 counter slot).  The
+// returned ticket is consumed one chunk later, so the atomic's latency hides
+// behind a chunk of work.  Called by lane 0 only; the address is offset by
+// %laneid * 8 (= 0 there) so that ptxas cannot prove it warp-uniform and does
+// not turn the atomic into a warp-aggregated one whose broadcast would wait
+// for the result right away.
+__device__ __forceinline__ uint32_t take_ticket(unsigned long long* slot) {
+  uint32_t k;
+  asm volatile(
+      "{ .reg .u32 l; .reg .u64 o, a; mov.u32 l, %%laneid; mul.wide.u32 o, l, 8; add.u64 a, %1, o;"
+      " atom.relaxed.gpu.global.add.u32 %0, [a], 1; }"
+      : "=r"(k) : "l"(slot) : "memory");
+  return k;
 }
 
 __device__ __forceinline__ uint32_t bits_mask(uint32_t b0, uint32_t b1) {  // bits b0..b1 inclusive
@@ -161,12 +219,76 @@ struct SlowCache {                       // 56 B
 };
 struct FastCache { uint64_t base, size, bm_word; uint32_t shift, meta; };
 
-struct WarpCounts { uint32_t rec, attr, unattr, clip, inval, ovf; };   // per warp, shared memory
+// per warp, shared memory: record counters of the slow paths and the tile
+// counts by path (diagnostics; shared-memory REDs keep them out of registers)
+struct WarpCounts { uint32_t rec, attr, unattr, clip, inval, ovf, aff_u, aff_w, fast, slow; };
+
+// Per-warp shared region, addressed through ONE 32-bit shared address: the
+// ring stages, their barriers and record counts, lane 0's fetch position and
+// the counters.
+struct alignas(16) WarpSmem {
+  uint4 ring[kStages][kWarpRecords];   // 3 x 2 KB stages
+  uint64_t full[kStages];              // one mbarrier per stage
+  uint64_t f_pos, f_hi;                // lane 0: rest of the current chunk [f_pos, f_hi)
+  uint32_t cnt[kStages];               // records in each stage (0 = end of work)
+  uint32_t pad;
+  WarpCounts wc;
+};
+constexpr uint32_t kOffFull = offsetof(WarpSmem, full), kOffPos = offsetof(WarpSmem, f_pos),
+                   kOffHi = offsetof(WarpSmem, f_hi), kOffCnt = offsetof(WarpSmem, cnt),
+                   kOffWc = offsetof(WarpSmem, wc);
+static_assert(offsetof(WarpCounts, aff_w) == offsetof(WarpCounts, aff_u) + 4, "aff_u / aff_w adjacent");
+// block layout: 8 x WarpSmem | level-1 keys (4 KB) | 256 x 56-B lane caches
+// = ~66 KB: three blocks (24 warps) per SM with ~26 KB of L1
+constexpr size_t kL1Off = size_t(kConsumerWarps) * sizeof(WarpSmem);
+constexpr size_t kCacheOff = kL1Off + size_t(kL1MaxKeys) * 8;
+constexpr size_t kAttrSmem = kCacheOff + size_t(kAttrThreads) * 56;
+
+__device__ __forceinline__ uint8_t* attr_smem() {
+  extern __shared__ __align__(128) uint8_t smem[];
+  return smem;
+}
+// Slow-path views, rebuilt from threadIdx inside the out-of-line functions so
+// that the hot loop keeps no pointers to them live.
+__device__ __forceinline__ const uint64_t* slow_l1() {
+  return reinterpret_cast<const uint64_t*>(attr_smem() + kL1Off);
+}
+__device__ __forceinline__ SlowCache* slow_cache() {
+  return reinterpret_cast<SlowCache*>(attr_smem() + kCacheOff) + threadIdx.x;
+}
+static_assert(sizeof(SlowCache) == 56, "kAttrSmem assumes 56-B lane caches");
+__device__ __forceinline__ WarpCounts* slow_counts() {
+  return &reinterpret_cast<WarpSmem*>(attr_smem())[threadIdx.x >> 5].wc;
+}
+
 
 __device__ __forceinline__ FastCache mirror(const SlowCache* c) {
   return FastCache{c->base, c->size, c->bm_word, c->shift, c->meta};
 }
 
+__device__ __forceinline__ SegEntry ldg_seg(const SegEntry* e) {
+  const uint4 v = __ldg(reinterpret_cast<const uint4*>(e));
+  return SegEntry{(uint64_t(v.y) << 32) | v.x, v.z, v.w};
+}
+
+// The object of segment entry e live at ts, or kNone.  Candidates are sorted
+// by t_alloc with disjoint lifetimes (R5): only the last one allocated before
+// ts can be live at ts (its t_free is checked by the caller).
+__device__ __forceinline__ uint32_t resolve_seg(const AttrParams& p, uint32_t ref, uint32_t aux, uint32_t ts) {
+  if (ref == kNone) return kNone;
+  if (!(ref & kMultiBit)) return aux < ts ? ref : kNone;
+  const uint32_t c0 = ref & ~kMultiBit;
+  uint32_t l = c0, h = c0 + aux;
+  const uint2* cand = reinterpret_cast<const uint2*>(p.cand);
+  while (l < h) {
+    const uint32_t mid = (l + h) >> 1;
+    if (__ldg(&cand[mid].y) < ts) l = mid + 1; else h = mid;
+  }
+  return l == c0 ? kNone : __ldg(&cand[l - 1].x);
+}
+
+// Per-lane lookup (A2): level-1 keys (every l1_stride-th segment start) in
+// shared memory, then a binary search of the segment entries in L2.
 __device__ __forceinline__ uint32_t find_object(const AttrParams& p, const uint64_t* s_l1,
                                                 uint64_t addr, uint32_t ts) {
   if (p.n_seg == 0 || addr < s_l1[0]) return kNone;
@@ -177,22 +299,61 @@ __device__ __forceinline__ uint32_t find_object(const AttrParams& p, const uint6
   }
   uint32_t a = lo * p.l1_stride;      // level 2 (L2): last segment start <= addr
   uint32_t b = min(a + p.l1_stride, p.n_seg);
+  SegEntry ea = ldg_seg(p.seg + a);   // independent of the search: overlaps it
   while (b - a > 1) {
     const uint32_t mid = (a + b) >> 1;
-    if (__ldg(p.seg_start + mid) <= addr) a = mid; else b = mid;
+    const SegEntry em = ldg_seg(p.seg + mid);
+    if (em.start <= addr) { a = mid; ea = em; } else b = mid;
   }
-  const uint32_t c0 = __ldg(p.seg_cand_off + a), c1 = __ldg(p.seg_cand_off + a + 1);
-  if (c0 == c1) return kNone;
-  // candidates sorted by t_alloc with disjoint lifetimes: only the last one
-  // allocated before ts can be live at ts
-  uint32_t l = c0, h = c1;
+  return resolve_seg(p, ea.ref, ea.aux, ts);
+}
+
+// Warp-cooperative lookup of ONE (addr, ts), uniform across the warp: every
+// search level is one 32-ary round (one shared-memory or L2 load per lane and
+// a ballot) instead of log2 dependent loads -- the chunk-start and burst-start
+// tiles wait on this chain.
+__device__ __forceinline__ uint32_t find_object_warp(const AttrParams& p, const uint64_t* s_l1, uint64_t addr,
+                                                     uint32_t ts, int lane) {
+  if (p.n_seg == 0 || addr < s_l1[0]) return kNone;
+  // level 1: n_l1 <= 1024 keys, two rounds (s_l1[0] <= addr, so bit 0 is set)
+  const uint32_t n1 = p.n_l1, step = (n1 + 31) >> 5;
+  uint32_t k = uint32_t(lane) * step;
+  uint32_t bal = __ballot_sync(FULL_MASK, k < n1 && s_l1[k] <= addr);
+  uint32_t lo = uint32_t(31 - __clz(bal)) * step;
+  k = lo + uint32_t(lane);
+  bal = __ballot_sync(FULL_MASK, uint32_t(lane) < step && k < n1 && s_l1[k] <= addr);
+  lo += uint32_t(31 - __clz(bal));
+  // level 2: 32-ary rounds over the <= l1_stride entries after key lo
+  uint32_t a = lo * p.l1_stride, w = min(p.l1_stride, p.n_seg - a);
+  uint32_t ref = kNone, aux = 0;
+  for (;;) {
+    const uint32_t sp = (w + 31) >> 5;
+    const bool in = uint32_t(lane) * sp < w;
+    SegEntry e{~0ull, kNone, 0};
+    if (in) e = ldg_seg(p.seg + a + uint32_t(lane) * sp);
+    bal = __ballot_sync(FULL_MASK, in && e.start <= addr);   // bit 0: seg[a].start <= addr
+    const int j = 31 - __clz(bal);
+    a += uint32_t(j) * sp;
+    if (sp == 1) {
+      ref = __shfl_sync(FULL_MASK, e.ref, j);
+      aux = __shfl_sync(FULL_MASK, e.aux, j);
+      break;
+    }
+    w = min(sp, w - uint32_t(j) * sp);
+  }
+  if (ref == kNone) return kNone;
+  if (!(ref & kMultiBit)) return aux < ts ? ref : kNone;
+  // several candidates (address reuse): the last one with t_alloc < ts
   const uint2* cand = reinterpret_cast<const uint2*>(p.cand);
-  while (l < h) {
-    const uint32_t mid = (l + h) >> 1;
-    if (__ldg(&cand[mid].y) < ts) l = mid + 1; else h = mid;
+  const uint32_t c0 = ref & ~kMultiBit;
+  uint32_t hit = kNone;
+  for (uint32_t b0 = 0; b0 < aux; b0 += 32) {
+    const uint32_t i = b0 + uint32_t(lane);
+    const uint32_t ok = __ballot_sync(FULL_MASK, i < aux && __ldg(&cand[c0 + i].y) < ts);
+    if (ok) hit = c0 + b0 + uint32_t(31 - __clz(ok));
+    if (ok != FULL_MASK) break;   // sorted by t_alloc: the rest are later
   }
-  if (l == c0) return kNone;
-  return __ldg(&cand[l - 1].x);
+  return hit == kNone ? kNone : __ldg(&cand[hit].x);
 }
 
 __device__ __noinline__ void enqueue_range(RangeEntry* rq, uint32_t rq_cap, unsigned long long* ctr,
@@ -236,8 +397,10 @@ __device__ __forceinline__ void add_counts(WarpCounts* wc, int lane, uint32_t re
 // The complete per-lane algorithm (every lane, any record).  Leaves each lane
 // with c->meta = the record's meta when the record was attributed, so that
 // following records of the same (object, API, rw) take the fast paths.
-__device__ __noinline__ void process_slow(const AttrParams& p, const uint64_t* s_l1, uint4 r,
-                                          bool present, int lane, SlowCache* c, WarpCounts* wc) {
+__device__ __noinline__ void process_slow(const AttrParams& p, uint4 r, bool present, int lane) {
+  const uint64_t* s_l1 = slow_l1();
+  SlowCache* c = slow_cache();
+  WarpCounts* wc = slow_counts();
   const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
   const uint32_t size = r.z;
   const uint32_t ts = r.w & 0x7FFFFFFFu;
@@ -441,20 +604,19 @@ __device__ __forceinline__ bool try_in_object(const uint4 (&r)[kTilesPerWarp], c
 // object (the first tile of every burst).  One lane resolves the object and
 // folds first/last/hit once for the warp; the lanes adopt the object into
 // their caches.  Returns false (no side effect) when the precondition fails.
-__device__ __noinline__ bool try_uniform_slow(const AttrParams& p, const uint64_t* s_l1, uint4 r,
-                                              bool present, int lane, SlowCache* c, WarpCounts* wc) {
+__device__ __noinline__ bool try_uniform_slow(const AttrParams& p, uint4 r, bool present, int lane) {
+  const uint64_t* s_l1 = slow_l1();
+  SlowCache* c = slow_cache();
+  WarpCounts* wc = slow_counts();
   const uint32_t meta = r.w;
   const uint32_t meta0 = __shfl_sync(FULL_MASK, meta, 0);   // all lanes: never inside && / ||
   if (!__all_sync(FULL_MASK, present && meta == meta0)) return false;
   const uint32_t ts = meta & 0x7FFFFFFFu, is_w = meta >> 31;
   if (ts >= p.n_api) return false;
-  const uint32_t rank = __ldg(p.acc_rank + ts);
-  if (rank == kNone) return false;
+  const uint32_t rank = __ldg(p.acc_rank + ts);   // checked after the search: its latency overlaps it
   const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
-  uint32_t o = kNone;
-  if (lane == 0) o = find_object(p, s_l1, addr, ts);
-  o = __shfl_sync(FULL_MASK, o, 0);
-  if (o == kNone) return false;
+  const uint32_t o = find_object_warp(p, s_l1, __shfl_sync(FULL_MASK, addr, 0), ts, lane);
+  if (rank == kNone || o == kNone) return false;
   const uint4* q = reinterpret_cast<const uint4*>(p.objs + o);
   const uint4 a = __ldg(q), b = __ldg(q + 1), d = __ldg(q + 2);
   if (ts >= d.y) return false;
@@ -485,67 +647,76 @@ __device__ __noinline__ bool try_uniform_slow(const AttrParams& p, const uint64_
 
 __global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid_constant__ AttrParams p) {
   extern __shared__ __align__(128) uint8_t smem[];
-  const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  // shared memory: per-warp rings | level-1 keys | barriers, slot counts |
-  // per-lane slow caches | per-warp counters
-  uint4* ring = reinterpret_cast<uint4*>(smem) + size_t(warp) * kStages * kWarpRecords;
-  uint8_t* tail = smem + size_t(kConsumerWarps) * kStages * kWarpRecords * 16;
-  uint64_t* s_l1 = reinterpret_cast<uint64_t*>(tail);
-  uint64_t* full = s_l1 + kL1MaxKeys + warp * kStages;
-  uint32_t* slot_cnt = reinterpret_cast<uint32_t*>(s_l1 + kL1MaxKeys + kConsumerWarps * kStages) + warp * kStages;
-  SlowCache* caches = reinterpret_cast<SlowCache*>(
-      tail + kL1MaxKeys * 8 + kConsumerWarps * kStages * 16);
-  WarpCounts* wcounts = reinterpret_cast<WarpCounts*>(caches + kAttrThreads);
-  SlowCache* my = caches + threadIdx.x;
-  WarpCounts* wc = wcounts + warp;
+  // this warp's region (shared-window address): ring | barriers | fetch state | counters
+  const uint32_t wsm = smem_u32(smem) + (threadIdx.x >> 5) * uint32_t(sizeof(WarpSmem));
 
   // Work distribution: warps take contiguous chunks (chunk_start) of records
   // from a global cursor (dynamic, so slow warps do not set the kernel's end).
-  // Only lane 0 touches the fetch state.
-  const uint64_t policy = evict_first_policy();
-  uint64_t f_pos = 0, f_hi = 0;
+  // Only lane 0 touches the fetch state (shared memory, plus the prefetched
+  // ticket of the next chunk in a register).
+  const uint32_t n_warps = gridDim.x * (kAttrThreads / 32);
+  // lane 0: ticket of the next chunk, taken two stages ahead (static: its own range first)
+  uint32_t f_next = kStatic ? blockIdx.x * (kAttrThreads / 32) + (threadIdx.x >> 5) : kNone;
+  auto ticket = [&]() { return take_ticket(&p.ctr[C_WORK]) + (kStatic ? n_warps : 0u); };
   auto fetch = [&](int s) {   // lane 0: fill slot s with the next <= 128 records, or mark the end
+    uint64_t f_pos = lds64(wsm + kOffPos), f_hi = lds64(wsm + kOffHi);
     if (f_pos == f_hi) {
-      const uint64_t kc = atomicAdd(&p.ctr[C_WORK], 1ull);
-      f_pos = min(chunk_start(kc, p.n), p.n);
-      f_hi = min(chunk_start(kc + 1, p.n), p.n);
+      do {   // skip empty chunks (only possible at the end or in a tiny static part)
+        const uint32_t kc = f_next == kNone ? ticket() : f_next;
+        f_next = kNone;
+        f_pos = min(chunk_start(kc, p.n, n_warps), p.n);
+        f_hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps), p.n);
+      } while (f_pos == f_hi && f_pos < p.n);
       if (f_pos >= p.n) f_pos = f_hi = p.n;
+      sts64(wsm + kOffHi, f_hi);
     }
     const uint32_t cnt = uint32_t(min(uint64_t(kWarpRecords), f_hi - f_pos));
-    slot_cnt[s] = cnt;
+    sts32(wsm + kOffCnt + 4 * s, cnt);
+    const uint32_t bar = wsm + kOffFull + 8 * s;
     if (cnt) {
-      mbar_arrive_expect_tx(&full[s], cnt * 16);
-      tma_load_1d(ring + size_t(s) * kWarpRecords, p.recs + f_pos, cnt * 16, &full[s], policy);
+      mbar_arrive_expect_tx(bar, cnt * 16);
+      tma_load_1d(wsm + s * (kWarpRecords * 16), p.recs + f_pos, cnt * 16, bar, evict_first_policy());
       f_pos += cnt;
+      sts64(wsm + kOffPos, f_pos);
+      // the next chunk's ticket is taken when this one has at most two stages
+      // left: its latency hides behind them, and no warp holds a reservation
+      // long enough to unbalance the end of the launch
+      if (f_next == kNone && f_hi - f_pos <= 2 * kWarpRecords && f_hi < p.n)
+        f_next = ticket();
     } else {
-      mbar_arrive(&full[s]);   // end of work: complete the phase with cnt = 0
+      mbar_arrive(bar);   // end of work: complete the phase with cnt = 0
     }
   };
 
+  SlowCache* my = slow_cache();
   my->base = 0; my->size = 0; my->bm_word = 0; my->hit_word = 0;
   my->t_alloc = 0; my->t_free = 0; my->r_lo = 0; my->shift = 0; my->obj = kNone; my->meta = kNever;
   if (lane == 0) {
-    *wc = WarpCounts{0, 0, 0, 0, 0, 0};
-    for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+    *slow_counts() = WarpCounts{0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+    sts64(wsm + kOffPos, 0);
+    sts64(wsm + kOffHi, 0);
+    for (int s = 0; s < kStages; ++s) mbar_init(wsm + kOffFull + 8 * s, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     for (int s = 0; s < kStages; ++s) fetch(s);
   }
-  for (uint32_t i = threadIdx.x; i < p.n_l1; i += blockDim.x) s_l1[i] = p.l1[i];
+  {
+    uint64_t* s_l1 = reinterpret_cast<uint64_t*>(smem + kL1Off);
+    for (uint32_t i = threadIdx.x; i < p.n_l1; i += blockDim.x) s_l1[i] = p.l1[i];
+  }
   __syncthreads();
 
   FastCache c = mirror(my);
   uint32_t fast_rec = 0;
-  uint32_t n_aff_u = 0, n_aff_w = 0, n_fast = 0, n_slow = 0;   // diagnostics (warp-uniform)
   bool uni = false;  // warp-uniform: all lanes cache one object (< 4 GiB) and one (API, rw)
   for (uint32_t st = 0;; ++st) {
     const int s = int(st % kStages);
-    mbar_wait(&full[s], (st / kStages) & 1);
-    const uint32_t cnt = slot_cnt[s];
+    mbar_wait<kOffFull>(wsm + 8 * s, (st / kStages) & 1);
+    const uint32_t cnt = lds32<kOffCnt>(wsm + 4 * s);
     if (cnt == 0) break;                                   // warp-uniform
     const int ntiles = int((cnt + 31) / 32);
     // copy the stage to registers (lane l: records l, 32+l, 64+l, 96+l) and refill the slot
-    const uint32_t sbuf = smem_u32(ring + size_t(s) * kWarpRecords) + lane * 16;
+    const uint32_t sbuf = wsm + s * (kWarpRecords * 16) + lane * 16;
     uint4 r4[kTilesPerWarp];
     if (cnt == kWarpRecords) {                             // full stage (all but a chunk's tail)
 #pragma unroll
@@ -556,27 +727,26 @@ __global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid
         r4[t] = t * 32 + lane < cnt ? lds128(sbuf + t * 512) : make_uint4(0, 0, 0, 0);
     }
     // The vote consumes every lane's loaded registers, so all of this warp's
-    // reads of the slot have completed before lane 0 refills it (no memory
-    // fence: that would also wait for this lane's outstanding global REDs).
+    // reads of the slot have completed before lane 0 refills it.  This is a
+    // write-after-read across proxies with the reads already retired, so no
+    // proxy fence (as a consumer release before a TMA refill; a memory fence
+    // would also wait for this lane's outstanding global REDs).
     uint32_t dep = 0;
 #pragma unroll
     for (int t = 0; t < kTilesPerWarp; ++t) dep ^= r4[t].x ^ r4[t].w;
     const bool never = __any_sync(FULL_MASK, dep == 0x9E3779B9u && lane == 32);
-    if (lane == 0 && !never) {
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      fetch(s);
-    }
+    if (lane == 0 && !never) fetch(s);
     __syncwarp();
     if (uni && ntiles == kTilesPerWarp) {
       const int how = try_affine(r4, c, p.orw, lane);
       if (how) {
         fast_rec += kTilesPerWarp;
-        if (how == 1) n_aff_u += kTilesPerWarp; else n_aff_w += kTilesPerWarp;
+        if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, aff_u)>(wsm + (how == 1 ? 0 : 4), kTilesPerWarp);
         continue;
       }
       if (try_in_object(r4, c, p.orw)) {
         fast_rec += kTilesPerWarp;
-        n_fast += kTilesPerWarp;
+        if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, fast)>(wsm, kTilesPerWarp);
         continue;
       }
     }
@@ -597,13 +767,13 @@ __global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid
         if (__all_sync(FULL_MASK, ok)) {
           fast_or(p.orw, c.bm_word, e0, e1, lane);
           ++fast_rec;
-          ++n_fast;
+          if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, fast)>(wsm, 1);
           continue;
         }
       }
-      if (!try_uniform_slow(p, s_l1, r, present, lane, my, wc))
-        process_slow(p, s_l1, r, present, lane, my, wc);
-      ++n_slow;
+      if (!try_uniform_slow(p, r, present, lane)) process_slow(p, r, present, lane);
+      if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, slow)>(wsm, 1);
+      SlowCache* my = slow_cache();
       c = mirror(my);
       const uint32_t m0 = __shfl_sync(FULL_MASK, c.meta, 0);
       const uint32_t o0 = __shfl_sync(FULL_MASK, my->obj, 0);
@@ -614,15 +784,16 @@ __global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid
   const uint32_t fr = __reduce_add_sync(FULL_MASK, fast_rec);
   __syncwarp();
   if (lane == 0) {
+    const WarpCounts* wc = slow_counts();
     const uint32_t v[6] = {wc->rec + fr, wc->attr + fr, wc->unattr, wc->clip, wc->inval, wc->ovf};
     const int slot[6] = {C_RECORDS, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID, C_RQ_OVERFLOW};
 #pragma unroll
     for (int i = 0; i < 6; ++i)
       if (v[i]) atomicAdd(&p.ctr[slot[i]], (unsigned long long)v[i]);
-    atomicAdd(&p.ctr[C_TILES_AFFINE_UNION], (unsigned long long)n_aff_u);
-    atomicAdd(&p.ctr[C_TILES_AFFINE_WORDS], (unsigned long long)n_aff_w);
-    atomicAdd(&p.ctr[C_TILES_FAST], (unsigned long long)n_fast);
-    atomicAdd(&p.ctr[C_TILES_SLOW], (unsigned long long)n_slow);
+    atomicAdd(&p.ctr[C_TILES_AFFINE_UNION], (unsigned long long)wc->aff_u);
+    atomicAdd(&p.ctr[C_TILES_AFFINE_WORDS], (unsigned long long)wc->aff_w);
+    atomicAdd(&p.ctr[C_TILES_FAST], (unsigned long long)wc->fast);
+    atomicAdd(&p.ctr[C_TILES_SLOW], (unsigned long long)wc->slow);
   }
 }
 

@@ -34,7 +34,7 @@ enum State { S_CREATED = 0, S_LOADED = 1, S_BOUND = 2 };
 struct Layout {
   uint64_t orw, first, last, ctr;           // dynamic (reset per trace)
   uint64_t dyn_end;
-  uint64_t objs, seg_start, seg_cand_off, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
+  uint64_t objs, seg_start, seg_cand_off, seg, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
   uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage;
   // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
@@ -64,6 +64,7 @@ struct drgpum_ctx {
   std::vector<DevObj> dobj;
   std::vector<uint64_t> seg_start;
   std::vector<uint32_t> seg_cand_off;
+  std::vector<SegEntry> seg;
   std::vector<CandEntry> cand;
   std::vector<uint64_t> l1;
   uint32_t l1_stride = 1;
@@ -204,6 +205,16 @@ drgpum_status build_tables(drgpum_ctx* c) {
                     c->cand[k - 1].obj, c->cand[k].obj);
     }
   }
+  if (n >= kMultiBit || total >= kMultiBit)
+    return fail(c, DRGPUM_ENOMEM, "segment index needs < 2^31 objects and candidate entries");
+  c->seg.assign(S, SegEntry{0, kNone, 0});
+  for (uint64_t j = 0; j < S; ++j) {
+    SegEntry& e = c->seg[j];
+    e.start = pts[j];
+    const uint32_t c0 = c->seg_cand_off[j], k = c->seg_cand_off[j + 1] - c0;
+    if (k == 1) { e.ref = c->cand[c0].obj; e.aux = c->cand[c0].t_alloc; }
+    else if (k > 1) { e.ref = kMultiBit | c0; e.aux = k; }
+  }
   // level-1 keys for shared memory
   c->l1_stride = (uint32_t)std::max<uint64_t>(1, (S + kL1MaxKeys - 1) / kL1MaxKeys);
   c->l1.clear();
@@ -295,6 +306,7 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   L.objs = put(sizeof(DevObj) * n);
   L.seg_start = put(8 * S);
   L.seg_cand_off = put(4 * (S + 1));
+  L.seg = put(sizeof(SegEntry) * S);
   L.cand = put(sizeof(CandEntry) * total);
   L.l1 = put(8 * c->l1.size());
   L.acc_rank = put(4ull * n_api);
@@ -396,6 +408,7 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   p.objs = at<DevObj>(c, c->L.objs);
   p.seg_start = at<uint64_t>(c, c->L.seg_start);
   p.seg_cand_off = at<uint32_t>(c, c->L.seg_cand_off);
+  p.seg = at<SegEntry>(c, c->L.seg);
   p.cand = at<CandEntry>(c, c->L.cand);
   p.l1 = at<uint64_t>(c, c->L.l1);
   p.n_seg = (uint32_t)c->seg_start.size();
@@ -485,7 +498,7 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   if (s != DRGPUM_OK) { ctx->err = tmp.err; return s; }
   ctx->n_obj = tmp.n_obj; ctx->n_api = tmp.n_api; ctx->n_acc = tmp.n_acc;
   ctx->objs.swap(tmp.objs); ctx->kinds.swap(tmp.kinds); ctx->dobj.swap(tmp.dobj);
-  ctx->seg_start.swap(tmp.seg_start); ctx->seg_cand_off.swap(tmp.seg_cand_off);
+  ctx->seg_start.swap(tmp.seg_start); ctx->seg_cand_off.swap(tmp.seg_cand_off); ctx->seg.swap(tmp.seg);
   ctx->cand.swap(tmp.cand); ctx->l1.swap(tmp.l1); ctx->l1_stride = tmp.l1_stride;
   ctx->acc_rank.swap(tmp.acc_rank); ctx->acc_ts.swap(tmp.acc_ts); ctx->acc_cs.swap(tmp.acc_cs);
   ctx->n_hit.swap(tmp.n_hit); ctx->tiles.swap(tmp.tiles); ctx->tile_off.swap(tmp.tile_off);
@@ -616,6 +629,7 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
   if ((r = up(L.objs, ctx->dobj.data(), sizeof(DevObj) * n))) return r;
   if ((r = up(L.seg_start, ctx->seg_start.data(), 8 * ctx->seg_start.size()))) return r;
   if ((r = up(L.seg_cand_off, ctx->seg_cand_off.data(), 4 * ctx->seg_cand_off.size()))) return r;
+  if ((r = up(L.seg, ctx->seg.data(), sizeof(SegEntry) * ctx->seg.size()))) return r;
   if ((r = up(L.cand, ctx->cand.data(), sizeof(CandEntry) * ctx->cand.size()))) return r;
   if ((r = up(L.l1, ctx->l1.data(), 8 * ctx->l1.size()))) return r;
   if ((r = up(L.acc_rank, ctx->acc_rank.data(), 4 * ctx->acc_rank.size()))) return r;

@@ -29,6 +29,16 @@ static_assert(sizeof(DevObj) == 48, "DevObj layout");
 // are sorted by t_alloc and have disjoint lifetimes).
 struct CandEntry { uint32_t obj, t_alloc; };
 
+// Segment entry (16 B): the start address and, when the segment has exactly
+// one candidate (the common, reuse-free case), that object and its t_alloc,
+// so a lookup resolves in one load per search level.
+//   ref = object id (< 2^31), aux = its t_alloc       one candidate
+//   ref = kNone                                      no candidate
+//   ref = kMultiBit | cand_off, aux = count           several (cand[] by t_alloc)
+constexpr uint32_t kMultiBit = 0x80000000u;
+struct alignas(16) SegEntry { uint64_t start; uint32_t ref, aux; };
+static_assert(sizeof(SegEntry) == 16, "SegEntry layout");
+
 // Range-expansion queue entry: inclusive global bit range, <= kRangeChunkWords words.
 struct RangeEntry { uint64_t bit_lo, bit_hi; };
 
@@ -58,6 +68,7 @@ struct AttrParams {
   const DevObj* objs;
   const uint64_t* seg_start;
   const uint32_t* seg_cand_off;
+  const SegEntry* seg;       // [n_seg]
   const CandEntry* cand;
   const uint64_t* l1;        // every l1_stride-th segment start
   uint32_t n_seg, n_l1, l1_stride, n_api;
