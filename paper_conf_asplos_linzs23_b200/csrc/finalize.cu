@@ -96,107 +96,183 @@ __device__ __forceinline__ BitMonoid bm_shfl_down(const BitMonoid& m, int d) {
                    __shfl_down_sync(FULL_MASK, m.best, d)};
 }
 
-// B4: one warp per tile (<= kTileWords = 1024 words of one object), read with
-// eight coalesced 16-B loads per lane issued up front.  Each 128-word block
-// (lane l holds words 4l..4l+3) is reduced without shuffle trees: lane runs
-// by sequential folds, then popcount by REDUX.SUM, lowest/highest accessed
-// bit by ballot + one shuffle, and the longest zero run by joining every
-// lane's leading zeros to the trailing zeros of the previous non-empty lane
-// (ballot + one indexed shuffle + REDUX.MAX).  Bits past the object's last
-// element are treated as 1 ("sentinels") for the run view so no zero run
-// extends past n_elems; they never count as accessed.
-__global__ void __launch_bounds__(256) tile_reduce_kernel(const uint32_t* __restrict__ orw,
+// Longest run of zeros of u strictly between its lowest and highest set bit
+// (0 with fewer than two set bits).  Binary lifting: A_j marks starts of runs
+// >= 2^j (A_{j+1} = A_j & A_j >> 2^j); cur marks starts of runs >= run;
+// extend run by 2^j, j = 4..0, whenever a run continues for another 2^j bits.
+// Out of line: the second pass of tile_reduce_kernel is the only caller.
+__device__ __noinline__ uint32_t interior_zero_run(uint32_t u) {
+  if (u == 0) return 0;
+  const uint32_t lo = __ffs(u) - 1, hi = 31 - __clz(u);
+  if (hi <= lo + 1) return 0;
+  const uint32_t y = ~u & ((1u << hi) - 1u) & ~((2u << lo) - 1u);
+  const uint32_t a1 = y & (y >> 1), a2 = a1 & (a1 >> 2), a3 = a2 & (a2 >> 4), a4 = a3 & (a3 >> 8);
+  const uint32_t A[5] = {y, a1, a2, a3, a4};
+  uint32_t cur = 0xFFFFFFFFu, run = 0;
+#pragma unroll
+  for (int j = 4; j >= 0; --j) {
+    const uint32_t t = cur & (A[j] >> run);
+    run += t ? (1u << j) : 0u;
+    cur = t ? t : cur;
+  }
+  return run;
+}
+
+// B4: one warp per tile (<= kTileWords = 1024 words of one object); lane l
+// folds the 32 consecutive words [32l, 32l+32) sequentially (eight 16-B
+// loads, the tile's lines shared through L1), then ONE warp join per tile:
+// popcount by REDUX.SUM, lowest/highest accessed bit by ballot + one shuffle,
+// and the longest zero run by joining every lane's leading zeros to the
+// trailing zeros of the previous non-empty lane (ballot + one indexed shuffle
+// + REDUX.MAX).  Bits past the object's last element are treated as 1
+// ("sentinels") for the run view so no zero run extends past n_elems; they
+// never count as accessed.  Zero runs inside one word (<= 30 bits) are skipped
+// in the first pass and computed in a second pass only when the tile's other
+// runs are all shorter than 30 -- otherwise they cannot change its longest
+// run (dense strided sweeps need them; untouched or sparse regions do not).
+__global__ void __launch_bounds__(256, 4) tile_reduce_kernel(const uint32_t* __restrict__ orw,
     const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out) {
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  constexpr int kBlocks = kTileWords / 128;
+  constexpr uint32_t kLaneWords = kTileWords / 32;          // 32 words = 1024 bits per lane
+  constexpr uint32_t kLaneBits = kLaneWords * 32;
+  static_assert(kLaneWords == 32, "transpose below assumes 8 x 16-B chunks per lane");
+  // per-warp 4-KB transpose buffer: the tile is read coalesced (lane l: words
+  // 128b + 4l .. +3) and each 16-B chunk stored where its owning lane reads
+  // it back; slot = owner * 8 + (chunk ^ (owner & 7)) keeps both sides free
+  // of bank conflicts
+  __shared__ uint4 s_tile[8][kTileWords / 4];
+  uint4* buf = s_tile[threadIdx.x >> 5];
   for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
     const Tile tl = tiles[t];
     const uint32_t nbits = uint32_t(tl.n_bits);
-    uint4 v[kBlocks];
+    const uint32_t w0 = kLaneWords * uint32_t(lane);
+    uint4 v[kLaneWords / 4];
 #pragma unroll
-    for (int b = 0; b < kBlocks; ++b) {
-      const uint32_t w = b * 128 + 4 * lane;
+    for (int b = 0; b < int(kLaneWords / 4); ++b) {
+      const uint32_t w = 128 * b + 4 * lane;
       v[b] = w < tl.n_words ? __ldg(reinterpret_cast<const uint4*>(orw + tl.word_lo + w))
                             : make_uint4(0, 0, 0, 0);
     }
-    M32 acc = m32_identity();   // identical in every lane
+    __syncwarp();   // the previous tile's reads of buf are done
 #pragma unroll
-    for (int b = 0; b < kBlocks; ++b) {
-      const uint32_t wb = b * 128 + 4 * lane;   // tile-relative word of v[b].x
-      uint32_t real[4] = {v[b].x, v[b].y, v[b].z, v[b].w};
-      uint32_t run[4] = {v[b].x, v[b].y, v[b].z, v[b].w};
-      const bool partial = uint32_t(b + 1) * 128 * 32 > nbits;   // warp-uniform
-      const bool lz = (v[b].x | v[b].y | v[b].z | v[b].w) == 0u;
-      const bool lo1 = (v[b].x & v[b].y & v[b].z & v[b].w) == 0xFFFFFFFFu;
-      if (!partial) {                                 // whole block untouched / fully accessed
-        if (__all_sync(FULL_MASK, lz)) { acc = m32_cat(acc, M32{4096, 0, kNoPos32, kNoPos32, 4096, 4096, 4096}); continue; }
-        if (__all_sync(FULL_MASK, lo1)) { acc = m32_cat(acc, M32{4096, 4096, 0, 4095, 0, 0, 0}); continue; }
-      }
-      if (partial) {   // block reaches past the tile's last bit
+    for (int b = 0; b < int(kLaneWords / 4); ++b) {
+      const uint32_t owner = 4 * b + (lane >> 3), chunk = lane & 7;
+      buf[owner * 8 + (chunk ^ (owner & 7))] = v[b];
+    }
+    __syncwarp();
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const uint32_t bj = (wb + j) * 32;
-          const uint32_t nv = bj >= nbits ? 0u : min(32u, nbits - bj);
-          const uint32_t vm = nv == 32 ? 0xFFFFFFFFu : ((1u << nv) - 1u);
-          real[j] &= vm;
-          run[j] = real[j] | ~vm;
-        }
-      }
-      // lane: real popcount / first / last accessed bit; run-view fold
-      uint32_t pop = 0, lo = kNoPos32, hi = kNoPos32;
-      M32 r;
-      if (!partial && lz) {
-        r = M32{128, 0, kNoPos32, kNoPos32, 128, 128, 128};
-      } else if (!partial && lo1) {
-        r = M32{128, 128, 0, 127, 0, 0, 0};
-        pop = 128; lo = 0; hi = 127;
-      } else {
-        r = m32_identity();
+    for (int k = 0; k < int(kLaneWords / 4); ++k) v[k] = buf[lane * 8 + (k ^ (lane & 7))];
+    // lane fold, branch-free per word: real popcount and the nonzero real
+    // words (lowest / highest accessed bit at the end); run view: z = zeros
+    // since the last 1, so a word with a 1 closes a zero run of z + ctz(u)
+    // bits (the prefix run if it is the lane's first 1), then z = clz(u)
+    uint32_t pop = 0, nzr = 0, z = 0, pre = kLaneBits, gapmax = 0;
+    bool seen = false;
+    auto step = [&](int j, uint32_t real, uint32_t u) {
+      pop += __popc(real);
+      nzr |= real ? (1u << j) : 0u;
+      const bool has = u != 0u;
+      const uint32_t c = z + __clz(__brev(u));
+      gapmax = (has && seen) ? max(gapmax, c) : gapmax;
+      pre = (has && !seen) ? c : pre;
+      seen = seen || has;
+      z = has ? __clz(u) : z + 32u;
+    };
+    // lane-uniform: does any of this lane's bits lie past the last element?
+    const bool masked = (w0 + kLaneWords) * 32 > nbits;
+    auto views = [&](int j, uint32_t& real, uint32_t& run) {
+      const uint4& q = v[j >> 2];
+      const uint32_t x = (j & 3) == 0 ? q.x : (j & 3) == 1 ? q.y : (j & 3) == 2 ? q.z : q.w;
+      const uint32_t bj = (w0 + j) * 32;
+      const uint32_t nv = bj >= nbits ? 0u : min(32u, nbits - bj);
+      const uint32_t vm = nv == 32 ? 0xFFFFFFFFu : ((1u << nv) - 1u);
+      real = masked ? x & vm : x;
+      run = masked ? real | ~vm : x;
+    };
+    if (!masked) {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          pop += __popc(real[j]);
-          if (real[j]) {
-            if (lo == kNoPos32) lo = 32 * j + __ffs(real[j]) - 1;
-            hi = 32 * j + 31 - __clz(real[j]);
-          }
-          r = m32_cat(r, m32_word(run[j], 32));
-        }
+      for (int k = 0; k < int(kLaneWords / 4); ++k) {
+        step(4 * k, v[k].x, v[k].x);
+        step(4 * k + 1, v[k].y, v[k].y);
+        step(4 * k + 2, v[k].z, v[k].z);
+        step(4 * k + 3, v[k].w, v[k].w);
       }
-      // block (128 words): combine the 32 lanes in order
-      M32 blk;
-      blk.len = 4096;
-      blk.pop = __reduce_add_sync(FULL_MASK, pop);
-      const uint32_t nzp = __ballot_sync(FULL_MASK, pop != 0);
-      if (nzp) {
-        const int fl = __ffs(nzp) - 1, ll = 31 - __clz(nzp);
-        blk.lo = 128 * fl + __shfl_sync(FULL_MASK, lo, fl);
-        blk.hi = 128 * ll + __shfl_sync(FULL_MASK, hi, ll);
-      } else {
-        __shfl_sync(FULL_MASK, lo, 0);   // keep the shuffles convergent
-        __shfl_sync(FULL_MASK, hi, 0);
-        blk.lo = blk.hi = kNoPos32;
+    } else {
+#pragma unroll
+      for (int j = 0; j < int(kLaneWords); ++j) {
+        uint32_t real, u;
+        views(j, real, u);
+        step(j, real, u);
       }
-      const uint32_t nz = __ballot_sync(FULL_MASK, r.pop != 0);   // lanes with a 1 in the run view
-      const uint32_t below = nz & ((1u << lane) - 1u);
-      const int i = below ? 31 - __clz(below) : -1;
-      const uint32_t suf_i = __shfl_sync(FULL_MASK, r.suf, i < 0 ? 0 : i);
-      const uint32_t run_j = (i < 0 ? 0u : suf_i + 128u * uint32_t(lane - i - 1)) +
-                             (i < 0 ? 128u * lane : 0u) + r.pre;
-      const uint32_t cand = r.pop ? max(r.best, run_j) : 0u;
-      uint32_t best = __reduce_max_sync(FULL_MASK, cand);
-      if (nz == 0) {
-        blk.pre = blk.suf = blk.best = 4096;
-        __shfl_sync(FULL_MASK, r.pre, 0);
-        __shfl_sync(FULL_MASK, r.suf, 0);
-      } else {
-        const int f = __ffs(nz) - 1, l = 31 - __clz(nz);
-        blk.pre = 128 * f + __shfl_sync(FULL_MASK, r.pre, f);
-        blk.suf = 128 * (31 - l) + __shfl_sync(FULL_MASK, r.suf, l);
-        blk.best = max(best, blk.suf);
+    }
+    // lowest / highest accessed bit of the lane from its first / last nonzero
+    // real word (read back from the transpose buffer, masked like above)
+    uint32_t lo = kNoPos32, hi = kNoPos32;
+    if (nzr) {
+      const uint32_t* wl = reinterpret_cast<const uint32_t*>(buf + lane * 8);
+      const int jl = __ffs(nzr) - 1, jh = 31 - __clz(nzr);
+      const uint32_t xl = wl[4 * ((jl >> 2) ^ (lane & 7)) + (jl & 3)];
+      const uint32_t xh = wl[4 * ((jh >> 2) ^ (lane & 7)) + (jh & 3)];
+      const uint32_t bl = (w0 + jl) * 32, bh = (w0 + jh) * 32;
+      const uint32_t nl = min(32u, nbits - bl), nh = min(32u, nbits - bh);   // both words hold real bits
+      const uint32_t ml = nl == 32 ? xl : xl & ((1u << nl) - 1u);
+      const uint32_t mh = nh == 32 ? xh : xh & ((1u << nh) - 1u);
+      lo = 32 * jl + __ffs(ml) - 1;
+      hi = 32 * jh + 31 - __clz(mh);
+    }
+    const int first1 = seen ? int(pre) : -1;
+    const int last1 = seen ? int(kLaneBits - 1 - z) : -1;
+    M32 r;
+    r.len = kLaneBits;
+    r.pop = first1 >= 0 ? 1u : 0u;   // "has a 1 in the run view"
+    r.pre = first1 >= 0 ? uint32_t(first1) : kLaneBits;
+    r.suf = first1 >= 0 ? uint32_t(int(kLaneBits) - 1 - last1) : kLaneBits;
+    r.best = first1 >= 0 ? max(gapmax, max(r.pre, r.suf)) : kLaneBits;
+    // tile: combine the 32 lanes in order
+    M32 acc;
+    acc.len = 32 * kLaneBits;
+    acc.pop = __reduce_add_sync(FULL_MASK, pop);
+    const uint32_t nzp = __ballot_sync(FULL_MASK, pop != 0);
+    if (nzp) {
+      const int fl = __ffs(nzp) - 1, ll = 31 - __clz(nzp);
+      acc.lo = kLaneBits * fl + __shfl_sync(FULL_MASK, lo, fl);
+      acc.hi = kLaneBits * ll + __shfl_sync(FULL_MASK, hi, ll);
+    } else {
+      __shfl_sync(FULL_MASK, lo, 0);   // keep the shuffles convergent
+      __shfl_sync(FULL_MASK, hi, 0);
+      acc.lo = acc.hi = kNoPos32;
+    }
+    const uint32_t nz = __ballot_sync(FULL_MASK, r.pop != 0);   // lanes with a 1 in the run view
+    const uint32_t below = nz & ((1u << lane) - 1u);
+    const int i = below ? 31 - __clz(below) : -1;
+    const uint32_t suf_i = __shfl_sync(FULL_MASK, r.suf, i < 0 ? 0 : i);
+    const uint32_t run_j = (i < 0 ? 0u : suf_i + kLaneBits * uint32_t(lane - i - 1)) +
+                           (i < 0 ? kLaneBits * lane : 0u) + r.pre;
+    const uint32_t cand = r.pop ? max(r.best, run_j) : 0u;
+    const uint32_t best = __reduce_max_sync(FULL_MASK, cand);
+    if (nz == 0) {
+      acc.pre = acc.suf = acc.best = 32 * kLaneBits;
+      __shfl_sync(FULL_MASK, r.pre, 0);
+      __shfl_sync(FULL_MASK, r.suf, 0);
+    } else {
+      const int f = __ffs(nz) - 1, l = 31 - __clz(nz);
+      acc.pre = kLaneBits * f + __shfl_sync(FULL_MASK, r.pre, f);
+      acc.suf = kLaneBits * (31 - l) + __shfl_sync(FULL_MASK, r.suf, l);
+      acc.best = max(best, acc.suf);
+    }
+    // pass 2: zero runs inside single words (<= 30 bits) matter only if every
+    // other run of the tile is shorter
+    if (acc.best < 30) {
+      uint32_t im = 0;
+#pragma unroll
+      for (int j = 0; j < int(kLaneWords); ++j) {
+        uint32_t real, u;
+        views(j, real, u);
+        if (u != 0u && u != 0xFFFFFFFFu) im = max(im, interior_zero_run(u));
       }
-      acc = m32_cat(acc, blk);
+      acc.best = max(acc.best, __reduce_max_sync(FULL_MASK, im));
     }
     if (lane == 0) {
       BitMonoid r;

@@ -15,6 +15,6 @@ for r in $(seq 1 $ROUNDS); do
     (cd /tmp/ab_$name && timeout 300 python bench.py --no-next --no-cpu-baseline --e2e-steps 1 --steps 40 ${BENCH_ARGS:-}) > $OUT/${name}_$r.json 2> $OUT/${name}_$r.err
     python -c "
 import json; d=json.load(open('$OUT/${name}_$r.json'))
-print('$name', $r, 'attr_ms %.4f'%d['phases_ms']['attribute'], 'step_ms %.4f'%d['ms_per_step'], 'frac %.4f'%d['roofline']['frac'], 'clk', d['clocks']['sm_mhz'], 'rec', d['counters']['records'], d['counters']['attributed'])" | tee -a $OUT/summary.txt
+print('$name', $r, 'attr_ms %.4f'%d['phases_ms']['attribute'], 'fin_ms %.4f'%d['phases_ms']['finalize'], 'step_ms %.4f'%d['ms_per_step'], 'frac %.4f'%d['roofline']['frac'], 'clk', d['clocks']['sm_mhz'], 'rec', d['counters']['records'], d['counters']['attributed'])" | tee -a $OUT/summary.txt
   done
 done
