@@ -48,6 +48,8 @@ def args_():
     ap.add_argument("--e2e-steps", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-next", action="store_true", help="skip the SURVEY §8(f) NEXT-row timings")
+    ap.add_argument("--no-graph", action="store_true",
+                    help="time eager launches instead of CUDA-graph replays of the step")
     ap.add_argument("--cpu-sample", type=int, default=None,
                     help="records in the oracle's timed sample (default: whole workload up to 1e8)")
     ap.add_argument("--ref-sample", type=int, default=8_000_000,
@@ -255,11 +257,33 @@ def main():
     for _ in range(a.warmup):
         one_step(d_recs)
     torch.cuda.synchronize()
+    l0 = s.launch_count()
+    one_step(d_recs)
+    graph_launches = s.launch_count() - l0   # kernels of the library per step
 
     # ---------------- device-resident timed region
+    # Phase breakdown: eager launches with events between the phases.
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(a.steps)]
+    torch.cuda.synchronize()
+    for k in range(a.steps):
+        one_step(d_recs, evs[k])
+    torch.cuda.synchronize()
+    ph = np.array([[e[i].elapsed_time(e[i + 1]) for i in range(4)] for e in evs])  # ms
+    ph_mean = ph.mean(axis=0)
+    # The step itself: one CUDA graph of the library's launches (reset,
+    # attribute + range expansion, finalize), replayed K times -- the same
+    # kernels without per-launch host gaps.  Multi-rank steps (NCCL merge)
+    # run eagerly.
+    use_graph = world == 1 and not a.no_graph
+    if use_graph:
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            one_step(d_recs)
+        for _ in range(a.warmup):
+            graph.replay()
+        torch.cuda.synchronize()
     clk = ClockSampler(local)
     time.sleep(0.3)
-    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(a.steps)]
     t_start = torch.cuda.Event(enable_timing=True)
     t_end = torch.cuda.Event(enable_timing=True)
     launches0 = s.launch_count()
@@ -268,15 +292,18 @@ def main():
     wall0 = time.perf_counter()
     t_start.record(stream)
     for k in range(a.steps):
-        one_step(d_recs, evs[k])
+        if use_graph:
+            graph.replay()
+        else:
+            one_step(d_recs)
     t_end.record(stream)
     torch.cuda.synchronize()
     barrier()
     wall_dev = time.perf_counter() - wall0
-    launches = s.launch_count() - launches0
+    # graph replays do not pass through the library's launch counter: count
+    # the captured launches once per replay
+    launches = (s.launch_count() - launches0) if not use_graph else graph_launches * a.steps
     ms_total = t_start.elapsed_time(t_end)
-    ph = np.array([[e[i].elapsed_time(e[i + 1]) for i in range(4)] for e in evs])  # ms
-    ph_mean = ph.mean(axis=0)
     if world > 1:
         t = torch.tensor([ms_total] + ph_mean.tolist(), dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -366,6 +393,7 @@ def main():
                 "path": "Session.attribute(pinned host tensor) -> drgpum_trace_attribute_host; "
                         "object_stats + patterns (D2H)"},
         "gpu_launches": launches,
+        "step_exec": "cuda_graph_replay" if use_graph else "eager",
         "clocks": clocks,
         "counters": {k: int(ctr[k]) for k in ctr.dtype.names},
         "attribution_paths_tiles": paths,

@@ -360,7 +360,7 @@ __device__ __noinline__ void enqueue_range(RangeEntry* rq, uint32_t rq_cap, unsi
                                            uint32_t* orw, uint64_t gb0, uint64_t gb1, uint32_t& ovf) {
   const uint64_t wlo = gb0 >> 5, whi = gb1 >> 5;
   const uint64_t nch = (whi - wlo) / kRangeChunkWords + 1;
-  const unsigned long long slot = atomicAdd(&ctr[C_RQ_COUNT], (unsigned long long)nch);
+  const unsigned long long slot = atomicAdd(ctr, (unsigned long long)nch);
   for (uint64_t c = 0; c < nch; ++c) {
     const uint64_t cw0 = wlo + c * kRangeChunkWords;
     const uint64_t bl = c == 0 ? gb0 : cw0 * 32;
@@ -442,7 +442,7 @@ __device__ __noinline__ void process_slow(const AttrParams& p, uint4 r, bool pre
     const uint64_t gb1 = c->bm_word * 32 + ((off_end - 1) >> c->shift);
     const uint64_t w0 = gb0 >> 5, w1 = gb1 >> 5;
     if (w1 - w0 >= 2) {
-      enqueue_range(p.rq, p.rq_cap, p.ctr, p.orw, gb0, gb1, ovf);
+      enqueue_range(p.rq, p.rq_cap, p.ctr + p.rq_slot, p.orw, gb0, gb1, ovf);
     } else if (w1 == w0) {
       key0 = w0; m0 = bits_mask(gb0 & 31, gb1 & 31);
     } else {
@@ -800,9 +800,16 @@ __global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid
 // B2: expand queued ranges: one warp per <= kRangeChunkWords-word entry;
 // interior words get a plain all-ones store (idempotent with concurrent ORs),
 // edge words a RED.OR.
+// The counters the attribution kernel consumed are re-armed here for the next
+// call (no memset nodes between calls): the work cursor, and the queue count
+// of the OTHER parity -- this call's count is still being read by every block.
 __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
-    const unsigned long long* ctr, uint32_t cap, uint32_t* orw) {
-  const unsigned long long cnt_raw = ctr[C_RQ_COUNT];
+    unsigned long long* ctr, uint32_t slot, uint32_t cap, uint32_t* orw) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    ctr[C_WORK] = 0;
+    ctr[slot == C_RQ_COUNT ? C_RQ_COUNT_ALT : C_RQ_COUNT] = 0;
+  }
+  const unsigned long long cnt_raw = ctr[slot];
   const uint64_t cnt = cnt_raw < cap ? cnt_raw : cap;
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
@@ -833,8 +840,8 @@ __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
 
 int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s) {
   if (p.n == 0) return 0;
-  cudaMemsetAsync(p.ctr + C_RQ_COUNT, 0, sizeof(unsigned long long), s);
-  cudaMemsetAsync(p.ctr + C_WORK, 0, sizeof(unsigned long long), s);
+  // C_WORK and this call's queue count are zero here: zeroed by the reset,
+  // then re-armed by the previous call's range_expand_kernel
   static int occ = 0;
   if (!occ) {
     cudaFuncSetAttribute(attribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kAttrSmem));
@@ -847,7 +854,7 @@ int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s) {
   if (blocks > full) blocks = full;
   if (blocks < 1) blocks = 1;
   attribute_kernel<<<(unsigned)blocks, kAttrThreads, kAttrSmem, s>>>(p);
-  range_expand_kernel<<<num_sms * 4, 256, 0, s>>>(p.rq, p.ctr, p.rq_cap, p.orw);
+  range_expand_kernel<<<num_sms * 4, 256, 0, s>>>(p.rq, p.ctr, p.rq_slot, p.rq_cap, p.orw);
   return 2;
 }
 

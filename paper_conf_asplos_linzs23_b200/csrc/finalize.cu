@@ -131,8 +131,9 @@ __device__ __noinline__ uint32_t interior_zero_run(uint32_t u) {
 // runs are all shorter than 30 -- otherwise they cannot change its longest
 // run (dense strided sweeps need them; untouched or sparse regions do not).
 __global__ void __launch_bounds__(256, 4) tile_reduce_kernel(const uint32_t* __restrict__ orw,
-    const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out) {
+    const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr) {
   const int lane = threadIdx.x & 31;
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctr[C_CONSISTENCY] = 0;   // counted by object_finalize_kernel
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
   constexpr uint32_t kLaneWords = kTileWords / 32;          // 32 words = 1024 bits per lane
@@ -452,7 +453,7 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   if (p.n_obj == 0) return 0;
   const uint64_t tb = (p.n_tiles + 7) / 8;
   const unsigned g1 = (unsigned)(tb < uint64_t(num_sms) * 16 ? tb : uint64_t(num_sms) * 16);
-  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles, p.n_tiles, p.tile_part);
+  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles, p.n_tiles, p.tile_part, p.ctr);
   const uint64_t gb = (p.n_groups + 7) / 8;
   const unsigned g3 = (unsigned)(gb < uint64_t(num_sms) * 16 ? gb : uint64_t(num_sms) * 16);
   group_reduce_kernel<<<g3 ? g3 : 1, 256, 0, s>>>(p.groups, p.n_groups, p.tile_part, p.group_part);

@@ -77,6 +77,7 @@ struct drgpum_ctx {
   std::vector<drgpum_object_layout_t> layout;
   uint64_t bitmap_words = 0, hit_words = 0;
   uint32_t rq_cap = 1u << 20;
+  uint64_t attr_calls = 0;        // parity selects the range-queue count slot
   uint32_t features = 0;
   std::vector<uint64_t> elem_base, slot_base;
   uint64_t n_elem_total = 0, n_slots = 0;
@@ -422,6 +423,7 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   p.ctr = at<unsigned long long>(c, c->L.ctr);
   p.rq = at<RangeEntry>(c, c->L.rq);
   p.rq_cap = c->rq_cap;
+  p.rq_slot = (c->attr_calls & 1) ? C_RQ_COUNT_ALT : C_RQ_COUNT;
   return p;
 }
 
@@ -666,6 +668,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_re
     return fail(ctx, DRGPUM_EINVAL, "records must be non-NULL and 16-B aligned");
   AttrParams p = attr_params(ctx, d_recs, n);
   ctx->launches += launch_attribute(p, ctx->num_sms, as_stream(stream));
+  ctx->attr_calls++;
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     ctx->launches += launch_structured(sa_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
@@ -705,6 +708,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
     CK(cudaStreamWaitEvent(st, ctx->ev_copied[b], 0));
     AttrParams p = attr_params(ctx, stage[b], m);
     ctx->launches += launch_attribute(p, ctx->num_sms, st);
+    ctx->attr_calls++;
     if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
       ctx->launches += launch_structured(sa_params(ctx, stage[b], m), ctx->num_sms, st);
     if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
@@ -764,7 +768,6 @@ DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_threshold
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "finalize before workspace_bind");
   drgpum_thresholds_t t = th ? *th : drgpum_thresholds_t{2, 80, 80};
   cudaStream_t st = as_stream(stream);
-  CK(cudaMemsetAsync(at<unsigned long long>(ctx, ctx->L.ctr) + C_CONSISTENCY, 0, 8, st));
   FinalParams p;
   p.orw = at<uint32_t>(ctx, ctx->L.orw);
   p.tiles = at<Tile>(ctx, ctx->L.tiles);

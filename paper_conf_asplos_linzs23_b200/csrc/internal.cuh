@@ -59,7 +59,8 @@ enum : int { C_RECORDS = 0, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID,
              C_RQ_OVERFLOW, C_CONSISTENCY, C_RQ_COUNT,
              // diagnostics: 32-record tiles by attribution path
              C_TILES_AFFINE_UNION, C_TILES_AFFINE_WORDS, C_TILES_FAST, C_TILES_SLOW,
-             C_WORK,   // attribution work cursor (records handed out)
+             C_WORK,   // attribution work cursor (chunk tickets handed out)
+             C_RQ_COUNT_ALT,   // range-queue count of odd-numbered attribute calls
              C_SLOTS = 16 };
 
 struct AttrParams {
@@ -79,6 +80,7 @@ struct AttrParams {
   unsigned long long* ctr;
   RangeEntry* rq;
   uint32_t rq_cap;
+  uint32_t rq_slot;          // counter slot of this call's range-queue count (C_RQ_COUNT / _ALT)
 };
 
 // NEXT-3 structured access pass (optional feature).
@@ -164,7 +166,7 @@ struct FinalParams {
 };
 
 // Launchers (return the number of kernels enqueued).
-int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);
+int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);   // p.rq_slot alternates per call
 int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
 int launch_frequency(const FreqParams& p, uint64_t n_slots, int num_sms, cudaStream_t s);
 int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t s);
