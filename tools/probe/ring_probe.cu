@@ -74,12 +74,40 @@ void run(const uint4* d, uint64_t n, unsigned long long* cur, uint32_t* out, int
          pad >> 10, occ, (unsigned long long)chunk, best, n * 16.0 / best / 1e6);
 }
 
+__global__ void __launch_bounds__(256) ldg_read(const uint4* __restrict__ recs, uint64_t n, uint32_t* out) {
+  uint32_t acc = 0;
+  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
+  uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  for (; i + 3 * nth < n; i += 4 * nth) {
+    uint4 r[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) r[k] = __ldcs(recs + i + k * nth);
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc ^= r[k].x + r[k].y * 3 + r[k].z * 5 + r[k].w;
+  }
+  for (; i < n; i += nth) { uint4 r = __ldcs(recs + i); acc ^= r.x + r.y * 3 + r.z * 5 + r.w; }
+  if (acc == 0x12345678u) out[0] = acc;
+}
+
+void run_ldg(const uint4* d, uint64_t n, uint32_t* out, int blocks) {
+  cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
+  float best = 1e9;
+  for (int i = 0; i < 6; ++i) {
+    cudaEventRecord(a);
+    ldg_read<<<blocks, 256>>>(d, n, out);
+    cudaEventRecord(b); cudaEventSynchronize(b);
+    float ms; cudaEventElapsedTime(&ms, a, b); if (ms < best) best = ms;
+  }
+  printf("LDG.128 grid-stride x4, %d blocks: %.3f ms  %.0f GB/s\n", blocks, best, n * 16.0 / best / 1e6);
+}
+
 int main() {
   const uint64_t n = 100000000ull;
   uint4* d; cudaMalloc(&d, n * 16); cudaMemset(d, 1, n * 16);
   unsigned long long* cur; cudaMalloc(&cur, 8); uint32_t* out; cudaMalloc(&out, 4);
   int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
   run<3, 4>(d, n, cur, out, sms, 8192, 3);            // warm-up
+  for (int b : {sms * 4, sms * 8, sms * 16, sms * 32}) run_ldg(d, n, out, b);
   for (uint64_t ch : {1024ull, 2048ull, 4096ull, 8192ull}) {
     run<3, 4>(d, n, cur, out, sms, ch, 5, 20 << 10);     // current attribution layout (3 blocks/SM)
     run<4, 4>(d, n, cur, out, sms, ch, 5, 5 << 10);      // + 1 stage, slow caches out of smem (3/SM)
