@@ -30,10 +30,26 @@ namespace drgpum {
 
 #define FULL_MASK 0xFFFFFFFFu
 
-constexpr int kConsumerWarps = 8;
+// Geometry (macros only for A/B builds, tools/build_variant.sh).  Measured on
+// C2 (tools/ab.sh, one box): 8 warps x 3 stages x 4 tiles at 3 blocks/SM
+// 0.404 ms; 256-record stages (8 tiles; 2 stages, 4 or 8 warps) 0.414-0.417;
+// 4 stages with 6-8 warps 0.405-0.411; 5 stages x 5 warps 0.417.
+#ifndef DRGPUM_WARPS
+#define DRGPUM_WARPS 8
+#endif
+#ifndef DRGPUM_STAGES
+#define DRGPUM_STAGES 3
+#endif
+#ifndef DRGPUM_TILES
+#define DRGPUM_TILES 4
+#endif
+#ifndef DRGPUM_MINBLOCKS
+#define DRGPUM_MINBLOCKS 3
+#endif
+constexpr int kConsumerWarps = DRGPUM_WARPS;
 constexpr int kAttrThreads = kConsumerWarps * 32;
-constexpr int kStages = 3;                                   // per-warp ring depth
-constexpr int kTilesPerWarp = 4;                             // 32-record tiles per stage
+constexpr int kStages = DRGPUM_STAGES;                       // per-warp ring depth
+constexpr int kTilesPerWarp = DRGPUM_TILES;                  // 32-record tiles per stage
 constexpr int kWarpRecords = kTilesPerWarp * 32;             // 128 records = 2 KB per stage
 // Work units: chunk k of a launch covers records [chunk_start(k),
 // chunk_start(k+1)).  Big chunks (fewer cache warm-ups at chunk starts) cover
@@ -153,9 +169,22 @@ __device__ __forceinline__ uint32_t bits_mask(uint32_t b0, uint32_t b1) {  // bi
 
 // Fire-and-forget global reductions (SASS REDG): OR/MIN/MAX are idempotent and
 // commutative, results are only read after the kernel, so relaxed gpu scope.
+#ifdef DRGPUM_DIAG_NORED
+// Diagnostic build only (tools/build_variant.sh NAME -DDRGPUM_DIAG_NORED=1):
+// every OR-RED is issued under a predicate that is false at run time, so the
+// instruction stream is unchanged and only the RED traffic through L1TEX/L2
+// disappears.  C2: 0.404 -> 0.303 ms -- the price of ~28M scattered RED
+// sectors (profiles/r01_c2_r40.md).  Results are wrong by construction.
+__constant__ uint32_t c_red_on = 0;
+__device__ __forceinline__ void red_or(uint32_t* a, uint32_t v) {
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %2, 0; @q red.relaxed.gpu.global.or.b32 [%0], %1; }"
+               ::"l"(a), "r"(v), "r"(c_red_on) : "memory");
+}
+#else
 __device__ __forceinline__ void red_or(uint32_t* a, uint32_t v) {
   asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
 }
+#endif
 __device__ __forceinline__ void red_min(uint32_t* a, uint32_t v) {
   asm volatile("red.relaxed.gpu.global.min.u32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
 }
@@ -645,7 +674,7 @@ __device__ __noinline__ bool try_uniform_slow(const AttrParams& p, uint4 r, bool
   return true;
 }
 
-__global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid_constant__ AttrParams p) {
+__global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kernel(const __grid_constant__ AttrParams p) {
   extern __shared__ __align__(128) uint8_t smem[];
   const int lane = threadIdx.x & 31;
   // this warp's region (shared-window address): ring | barriers | fetch state | counters
@@ -733,7 +762,7 @@ __global__ void __launch_bounds__(kAttrThreads, 3) attribute_kernel(const __grid
     // would also wait for this lane's outstanding global REDs).
     uint32_t dep = 0;
 #pragma unroll
-    for (int t = 0; t < kTilesPerWarp; ++t) dep ^= r4[t].x ^ r4[t].w;
+    for (int t = 0; t < kTilesPerWarp; ++t) dep ^= r4[t].x;   // one register per LDS.128 suffices
     const bool never = __any_sync(FULL_MASK, dep == 0x9E3779B9u && lane == 32);
     if (lane == 0 && !never) fetch(s);
     __syncwarp();

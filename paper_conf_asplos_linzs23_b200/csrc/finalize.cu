@@ -183,6 +183,16 @@ __global__ void __launch_bounds__(256, 4) tile_reduce_kernel(const uint32_t* __r
     };
     // lane-uniform: does any of this lane's bits lie past the last element?
     const bool masked = (w0 + kLaneWords) * 32 > nbits;
+    // all-ones / all-zeros lanes (dense sweeps, untouched regions) in closed
+    // form: three-input ANDs / ORs over the 32 words instead of the fold
+    uint32_t all_and = 0xFFFFFFFFu, all_or = 0u;
+#pragma unroll
+    for (int k = 0; k < int(kLaneWords / 4); ++k) {
+      all_and &= v[k].x & v[k].y & v[k].z & v[k].w;
+      all_or |= v[k].x | v[k].y | v[k].z | v[k].w;
+    }
+    const bool full = !masked && all_and == 0xFFFFFFFFu;
+    const bool empty = !masked && all_or == 0u;
     auto views = [&](int j, uint32_t& real, uint32_t& run) {
       const uint4& q = v[j >> 2];
       const uint32_t x = (j & 3) == 0 ? q.x : (j & 3) == 1 ? q.y : (j & 3) == 2 ? q.z : q.w;
@@ -192,7 +202,11 @@ __global__ void __launch_bounds__(256, 4) tile_reduce_kernel(const uint32_t* __r
       real = masked ? x & vm : x;
       run = masked ? real | ~vm : x;
     };
-    if (!masked) {
+    if (full) {
+      pop = kLaneBits; nzr = 0xFFFFFFFFu; z = 0; pre = 0; seen = true;
+    } else if (empty) {
+      z = kLaneBits;
+    } else if (!masked) {
 #pragma unroll
       for (int k = 0; k < int(kLaneWords / 4); ++k) {
         step(4 * k, v[k].x, v[k].x);
@@ -265,10 +279,12 @@ __global__ void __launch_bounds__(256, 4) tile_reduce_kernel(const uint32_t* __r
     }
     // pass 2: zero runs inside single words (<= 30 bits) matter only if every
     // other run of the tile is shorter
-    if (acc.best < 30) {
+    const bool mixed = !(full || empty);
+    if (acc.best < 30 && __any_sync(FULL_MASK, mixed)) {
       uint32_t im = 0;
 #pragma unroll
       for (int j = 0; j < int(kLaneWords); ++j) {
+        if (!mixed) break;   // uniform lanes hold no word-interior zero run
         uint32_t real, u;
         views(j, real, u);
         if (u != 0u && u != 0xFFFFFFFFu) im = max(im, interior_zero_run(u));
