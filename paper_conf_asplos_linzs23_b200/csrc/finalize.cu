@@ -365,17 +365,24 @@ __device__ __forceinline__ HitM hit_shfl_down(const HitM& m, int d) {
 // looks them up once per accessing API, on a dependent chain).
 constexpr uint32_t kSmemAcc = 8192;
 
+constexpr int kFinThreads = 256;
+
 template <bool kStaged>
-__global__ void __launch_bounds__(128) object_finalize_kernel(const FinalParams p) {
-  extern __shared__ uint32_t s_acc[];   // [n_acc] ts, then [n_acc] cs bytes
+__global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const FinalParams p) {
+  extern __shared__ uint4 s_acc4[];     // [n_acc] ts (padded to 16 B), then [n_acc] cs bytes
   const uint32_t* acc_ts = p.acc_ts;
   const uint8_t* acc_cs = p.acc_cs;
   if (kStaged) {
-    uint8_t* s_cs = reinterpret_cast<uint8_t*>(s_acc + p.n_acc);
-    for (uint32_t i = threadIdx.x; i < p.n_acc; i += blockDim.x) { s_acc[i] = p.acc_ts[i]; s_cs[i] = p.acc_cs[i]; }
+    // 16-B copies (the workspace sections are 256-B aligned and padded, so
+    // the rounded-up tails stay inside them); independent loads, one round trip
+    const uint32_t nts = (p.n_acc + 3) / 4, ncs = (p.n_acc + 15) / 16;
+    const uint4* g_ts = reinterpret_cast<const uint4*>(p.acc_ts);
+    const uint4* g_cs = reinterpret_cast<const uint4*>(p.acc_cs);
+    for (uint32_t i = threadIdx.x; i < nts + ncs; i += blockDim.x)
+      s_acc4[i] = i < nts ? __ldg(g_ts + i) : __ldg(g_cs + (i - nts));
     __syncthreads();
-    acc_ts = s_acc;
-    acc_cs = s_cs;
+    acc_ts = reinterpret_cast<const uint32_t*>(s_acc4);
+    acc_cs = reinterpret_cast<const uint8_t*>(s_acc4 + nts);
   }
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
@@ -473,12 +480,13 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   const uint64_t gb = (p.n_groups + 7) / 8;
   const unsigned g3 = (unsigned)(gb < uint64_t(num_sms) * 16 ? gb : uint64_t(num_sms) * 16);
   group_reduce_kernel<<<g3 ? g3 : 1, 256, 0, s>>>(p.groups, p.n_groups, p.tile_part, p.group_part);
-  const uint64_t ob = (p.n_obj + 3) / 4;   // one warp per object, 4 warps per block
-  const unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 32 ? ob : uint64_t(num_sms) * 32);
+  constexpr unsigned wpb = kFinThreads / 32;   // one warp per object
+  const uint64_t ob = (p.n_obj + wpb - 1) / wpb;
+  const unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
   if (p.n_acc <= kSmemAcc)
-    object_finalize_kernel<true><<<g2, 128, p.n_acc * 5 + 16, s>>>(p);
+    object_finalize_kernel<true><<<g2, kFinThreads, 16 * ((p.n_acc + 3) / 4 + (p.n_acc + 15) / 16), s>>>(p);
   else
-    object_finalize_kernel<false><<<g2, 128, 0, s>>>(p);
+    object_finalize_kernel<false><<<g2, kFinThreads, 0, s>>>(p);
   return 3;
 }
 
