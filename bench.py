@@ -33,7 +33,18 @@ WORKLOADS = {
     "C1": "C1 synthetic (BASELINE configs[0]): 2^20 records, 4-8 B accesses, 64 objects (16 MiB), 100 access APIs",
     "C2": "C2 Rodinia-style HPC trace (BASELINE configs[1]): 1e8 records over 1000 objects (4 GiB), "
           "strided + partial-object access, 3700 access APIs",
+    "C3": "C3 ResNet-50 training-iteration-shaped trace (BASELINE configs[2]): 1e9 records over 20K tensors "
+          "in a 12 GiB best-fit caching pool (address reuse), short-lived activations",
+    "C4": "C4 LLM-inference-shaped trace (BASELINE configs[3]): 4e9 records over 100K objects "
+          "(120 GiB live footprint, reused 4 GiB activation arena), Zipf-skewed hot weights / KV blocks",
+    "C5": "C5 scaling sweep (BASELINE configs[4]): 1.6e10 records over 1M objects, streamed through HBM "
+          "in 2^28-record chunks generated on the device",
 }
+# configs whose records are generated on the device (tracegen/gen.cu) rather
+# than on the host; traces above RESIDENT_BYTES are streamed in GEN_CHUNK chunks
+DEVICE_GEN = ("C3", "C4", "C5")
+GEN_CHUNK = 1 << 28
+RESIDENT_BYTES = 96 << 30
 FALLBACK_HBM_GBS = 6650.0
 
 
@@ -51,7 +62,10 @@ def args_():
     ap.add_argument("--no-graph", action="store_true",
                     help="time eager launches instead of CUDA-graph replays of the step")
     ap.add_argument("--cpu-sample", type=int, default=None,
-                    help="records in the oracle's timed sample (default: whole workload up to 1e8)")
+                    help="records in the oracle's timed sample (default: whole workload up to 1e8; "
+                         "2e7 for the device-generated configs)")
+    ap.add_argument("--e2e-sample", type=int, default=1 << 26,
+                    help="records of the host-buffer (e2e) leg for the device-generated configs")
     ap.add_argument("--ref-sample", type=int, default=8_000_000,
                     help="records per reference-arm step")
     return ap.parse_args()
@@ -233,8 +247,27 @@ def main():
     N = prog.n_records
     lo, hi = shard_range(N, rank, world)
     n_local = hi - lo
-    recs = gen_records(prog, lo, hi)
-    d_recs = torch.from_numpy(recs.view(np.uint8)).cuda()
+    devgen = a.config in DEVICE_GEN
+    chunked = devgen and 16 * n_local > RESIDENT_BYTES
+    recs = None
+    if not devgen:
+        recs = gen_records(prog, lo, hi)
+        d_recs = torch.from_numpy(recs.view(np.uint8)).cuda()
+        chunks = [(0, n_local)]
+    else:
+        # device generation (never timed): the whole shard resident, or one
+        # GEN_CHUNK buffer refilled per chunk inside every step
+        from tracegen.device import DeviceProgram
+        dp = DeviceProgram(prog)
+        gen_chunks = [(c, min(c + GEN_CHUNK, n_local)) for c in range(0, n_local, GEN_CHUNK)]
+        d_recs = torch.empty(16 * (GEN_CHUNK if chunked else n_local), dtype=torch.uint8, device="cuda")
+        if chunked:
+            chunks = gen_chunks
+        else:
+            for c0, c1 in gen_chunks:
+                dp.gen(lo + c0, lo + c1, out=d_recs[16 * c0:16 * c1])
+            chunks = [(0, n_local)]
+        torch.cuda.synchronize()
     s = Session(prog.objects, prog.kinds)
     stream = torch.cuda.current_stream()
 
@@ -243,16 +276,32 @@ def main():
             dist.barrier()
 
     def one_step(src, ev=None):
-        if ev: ev[0].record(stream)
+        """ev: per-phase event pairs [reset, attribute, merge, finalize]; the
+        attribute pair is per chunk (generation of a chunk lies outside it)."""
+        if ev: ev["reset"][0].record(stream)
         s.reset()
-        if ev: ev[1].record(stream)
-        s.attribute(src)
-        if ev: ev[2].record(stream)
+        if ev: ev["reset"][1].record(stream)
+        for k, (c0, c1) in enumerate(chunks):
+            if chunked:
+                dp.gen(lo + c0, lo + c1, out=src)
+            if ev: ev["attr"][k][0].record(stream)
+            s.attribute(src[:16 * (c1 - c0)])
+            if ev: ev["attr"][k][1].record(stream)
+        if ev: ev["merge"][0].record(stream)
         if world > 1:
             merge_session(s)
-        if ev: ev[3].record(stream)
+        if ev: ev["merge"][1].record(stream)
+        if ev: ev["fin"][0].record(stream)
         s.finalize()
-        if ev: ev[4].record(stream)
+        if ev: ev["fin"][1].record(stream)
+
+    def events():
+        E = lambda: (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+        return {"reset": E(), "attr": [E() for _ in chunks], "merge": E(), "fin": E()}
+
+    def phases(ev):   # ms
+        el = lambda e: e[0].elapsed_time(e[1])
+        return [el(ev["reset"]), sum(el(e) for e in ev["attr"]), el(ev["merge"]), el(ev["fin"])]
 
     for _ in range(a.warmup):
         one_step(d_recs)
@@ -263,18 +312,19 @@ def main():
 
     # ---------------- device-resident timed region
     # Phase breakdown: eager launches with events between the phases.
-    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(a.steps)]
+    evs = [events() for _ in range(a.steps)]
     torch.cuda.synchronize()
     for k in range(a.steps):
         one_step(d_recs, evs[k])
     torch.cuda.synchronize()
-    ph = np.array([[e[i].elapsed_time(e[i + 1]) for i in range(4)] for e in evs])  # ms
+    ph = np.array([phases(e) for e in evs])  # ms
     ph_mean = ph.mean(axis=0)
     # The step itself: one CUDA graph of the library's launches (reset,
     # attribute + range expansion, finalize), replayed K times -- the same
     # kernels without per-launch host gaps.  Multi-rank steps (NCCL merge)
-    # run eagerly.
-    use_graph = world == 1 and not a.no_graph
+    # run eagerly; chunked traces (generation between the chunks) are timed
+    # as the sum of their phase events.
+    use_graph = world == 1 and not a.no_graph and not chunked
     if use_graph:
         graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(graph):
@@ -291,11 +341,12 @@ def main():
     torch.cuda.synchronize()
     wall0 = time.perf_counter()
     t_start.record(stream)
+    tev = [events() for _ in range(a.steps)] if chunked else None
     for k in range(a.steps):
         if use_graph:
             graph.replay()
         else:
-            one_step(d_recs)
+            one_step(d_recs, tev[k] if chunked else None)
     t_end.record(stream)
     torch.cuda.synchronize()
     barrier()
@@ -304,6 +355,8 @@ def main():
     # the captured launches once per replay
     launches = (s.launch_count() - launches0) if not use_graph else graph_launches * a.steps
     ms_total = t_start.elapsed_time(t_end)
+    if chunked:   # generation excluded: the steps are the sum of their phases
+        ms_total = float(sum(sum(phases(e)) for e in tev))
     if world > 1:
         t = torch.tensor([ms_total] + ph_mean.tolist(), dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -319,8 +372,9 @@ def main():
 
     # ---------------- end-to-end through the public API with HOST buffers
     e2e_steps = a.e2e_steps or min(a.steps, 10)
-    pinned = torch.empty(n_local * 16, dtype=torch.uint8, pin_memory=True)
-    pinned.numpy()[:] = recs.view(np.uint8)
+    n_e2e = n_local if not devgen else min(n_local, a.e2e_sample)
+    pinned = torch.empty(n_e2e * 16, dtype=torch.uint8, pin_memory=True)
+    pinned.numpy()[:] = (recs if recs is not None else gen_records(prog, lo, lo + n_e2e)).view(np.uint8)
     for _ in range(2):
         s.reset(); s.attribute(pinned); s.object_stats(); s.patterns()
     torch.cuda.synchronize()
@@ -341,7 +395,7 @@ def main():
         e2e_s = float(t[0])
     clocks = clk.stop()
     nxt = None
-    if world == 1 and not a.no_next:
+    if world == 1 and not a.no_next and not devgen:
         nxt = next_rows(prog, d_recs, float(ph_mean[1]))
 
     if rank != 0:
@@ -362,8 +416,8 @@ def main():
 
     cpu = None
     if world == 1 and not a.no_cpu_baseline:
-        m = min(a.cpu_sample or N, N, 100_000_000)
-        tcpu = time_oracle(prog.objects, prog.kinds, recs[:m])
+        m = min(a.cpu_sample or (20_000_000 if devgen else N), N, 100_000_000)
+        tcpu = time_oracle(prog.objects, prog.kinds, recs[:m] if recs is not None else gen_records(prog, 0, m))
         cpu = {"value": m / tcpu, "unit": "records/s", "cores": 1, "kind": "oracle",
                "sample": (f"{'all' if m == N else 'first'} {m} records of the {a.config} trace, "
                           f"one pass: load + attribute + stats + patterns (O1, single thread)"),
@@ -387,7 +441,8 @@ def main():
                      "bytes_rule": "16 B per record + 4 B per touched shadow word",
                      "peak_source": hbm_src},
         "cpu_baseline": cpu,
-        "e2e": {"value": N / e2e_s, "unit": "records/s", "h2d_bytes_per_step": 16 * n_local,
+        "e2e": {"value": n_e2e * world / e2e_s, "unit": "records/s", "h2d_bytes_per_step": 16 * n_e2e,
+                "records_per_rank": n_e2e,
                 "d2h_bytes_per_step": int(prog.n_obj * (56 + 32) + 40),
                 "ms_per_step": e2e_s * 1e3,
                 "path": "Session.attribute(pinned host tensor) -> drgpum_trace_attribute_host; "
