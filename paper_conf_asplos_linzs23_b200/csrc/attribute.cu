@@ -255,8 +255,24 @@ struct WarpCounts { uint32_t rec, attr, unattr, clip, inval, ovf, aff_u, aff_w, 
 // Per-warp shared region, addressed through ONE 32-bit shared address: the
 // ring stages, their barriers and record counts, lane 0's fetch position and
 // the counters.
+// Small objects (bitmap <= kScratchWords words, i.e. <= 4096 elements): the
+// fast tiers OR their per-record masks into a per-warp shared-memory copy of
+// the object's bitmap (RED.shared) instead of global REDs; the copy is
+// flushed -- one global RED per nonzero word, coalesced -- when the warp's
+// object changes and at the end of the kernel.  A burst of thousands of
+// scattered records over a small object then costs a handful of global RED
+// sectors instead of one per record.  Exact: OR is idempotent and
+// commutative, every scratch bit reaches global memory before the kernel ends.
+#ifndef DRGPUM_SCRATCH
+#define DRGPUM_SCRATCH 128
+#endif
+constexpr uint32_t kScratchWords = DRGPUM_SCRATCH;
+constexpr uint64_t kNoScratch = ~0ull;
+
 struct alignas(16) WarpSmem {
   uint4 ring[kStages][kWarpRecords];   // 3 x 2 KB stages
+  uint32_t scratch[kScratchWords > 0 ? kScratchWords : 4];   // small-object bitmap copy
+  uint64_t sc_base;                    // global word of scratch[0], kNoScratch if unbound
   uint64_t full[kStages];              // one mbarrier per stage
   uint64_t f_pos, f_hi;                // lane 0: rest of the current chunk [f_pos, f_hi)
   uint32_t cnt[kStages];               // records in each stage (0 = end of work)
@@ -265,7 +281,8 @@ struct alignas(16) WarpSmem {
 };
 constexpr uint32_t kOffFull = offsetof(WarpSmem, full), kOffPos = offsetof(WarpSmem, f_pos),
                    kOffHi = offsetof(WarpSmem, f_hi), kOffCnt = offsetof(WarpSmem, cnt),
-                   kOffWc = offsetof(WarpSmem, wc);
+                   kOffWc = offsetof(WarpSmem, wc), kOffScratch = offsetof(WarpSmem, scratch),
+                   kOffScBase = offsetof(WarpSmem, sc_base);
 static_assert(offsetof(WarpCounts, aff_w) == offsetof(WarpCounts, aff_u) + 4, "aff_u / aff_w adjacent");
 // block layout: 8 x WarpSmem | level-1 keys (4 KB) | 256 x 56-B lane caches
 // = ~66 KB: three blocks (24 warps) per SM with ~26 KB of L1
@@ -521,6 +538,47 @@ __device__ __forceinline__ void red_record(uint32_t* orw, uint64_t bm_word, uint
   }
 }
 
+// --- small-object scratch (warp-uniform calls)
+__device__ __forceinline__ bool scratch_ok(const FastCache& c) {
+  return kScratchWords > 0 && c.size <= (uint64_t(kScratchWords) * 32) << c.shift;
+}
+__device__ __forceinline__ void red_shared_or(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+// OR every nonzero scratch word into the global bitmap at sc_base and clear it
+__device__ __noinline__ void scratch_flush(uint32_t wsm, uint32_t* orw, uint64_t sc_base, int lane) {
+  __syncwarp();   // every lane's shared REDs are done
+#pragma unroll
+  for (uint32_t i = lane; i < kScratchWords; i += 32) {
+    const uint32_t a = wsm + kOffScratch + 4 * i;
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+    if (v) {
+      red_or(orw + sc_base + i, v);
+      sts32(a, 0);
+    }
+  }
+  __syncwarp();
+}
+// bind the scratch to the object whose bitmap starts at bm_word (flushing the
+// previous object's bits)
+__device__ __forceinline__ void scratch_bind(uint32_t wsm, uint32_t* orw, uint64_t bm_word, int lane) {
+  const uint64_t cur = lds64(wsm + kOffScBase);
+  if (cur == bm_word) return;   // warp-uniform
+  if (cur != kNoScratch) scratch_flush(wsm, orw, cur, lane);
+  if (lane == 0) sts64(wsm + kOffScBase, bm_word);
+  __syncwarp();
+}
+__device__ __forceinline__ void scratch_record(uint32_t wsm, uint32_t e0, uint32_t e1) {
+  const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
+  if (w1 == w0) {
+    red_shared_or(wsm + kOffScratch + 4 * w0, bits_mask(e0 & 31, e1 & 31));
+  } else {
+    red_shared_or(wsm + kOffScratch + 4 * w0, 0xFFFFFFFFu << (e0 & 31));
+    red_shared_or(wsm + kOffScratch + 4 * w1, 0xFFFFFFFFu >> (31 - (e1 & 31)));
+  }
+}
+
 __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_t e0, uint32_t e1, int lane) {
   // contiguous union: intervals chain (start within or right after the
   // previous interval, monotone ends) -> union = [e0 of lane 0, e1 of lane 31]
@@ -542,6 +600,22 @@ __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_
   }
   red_record(orw, bm_word, e0, e1);   // irregular: each record ORs its own word(s)
 }
+// fast_or for the warp's cached object c: irregular tiles of a small object
+// go through the scratch
+__device__ __forceinline__ void fast_or_c(uint32_t wsm, uint32_t* orw, const FastCache& c, uint32_t e0,
+                                          uint32_t e1, int lane) {
+  if (scratch_ok(c)) {
+    const uint32_t pe0 = __shfl_up_sync(FULL_MASK, e0, 1);
+    const uint32_t pe1 = __shfl_up_sync(FULL_MASK, e1, 1);
+    const bool chain = lane == 0 || (e0 >= pe0 && e0 <= pe1 + 1 && e1 >= pe1);
+    if (!__all_sync(FULL_MASK, chain)) {
+      scratch_bind(wsm, orw, c.bm_word, lane);
+      scratch_record(wsm, e0, e1);
+      return;
+    }
+  }
+  fast_or(orw, c.bm_word, e0, e1, lane);
+}
 
 // Affine tier: the warp's 128 consecutive records (4 tiles, lane l holds
 // records l, 32+l, 64+l, 96+l) are one constant-stride run of one size and one
@@ -553,7 +627,7 @@ __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_
 // with one RED.OR per word; otherwise each record ORs its own word(s).
 // Returns false (no side effect) when the precondition does not hold.
 __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const FastCache& c,
-                                           uint32_t* orw, int lane) {
+                                           uint32_t* orw, uint32_t wsm, int lane) {
   // predicted record j = 32k + lane: {lo(a0) + j*st, hi(a0), sz, meta}; the
   // mismatch bits of all four words of all records are ORed with 3-input
   // LOP3s (about 5 instructions per record)
@@ -594,8 +668,18 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
     return 1;
   }
   if (((sz - 1) >> c.shift) >= 32) return 0;   // records wider than a word: tile path
-  // not one range: every record ORs its own word(s) (offsets in 32 bits)
+  // not one range: every record ORs its own word(s) (offsets in 32 bits),
+  // through the scratch for a small object
   uint32_t off = o0 + uint32_t(lane) * st32;
+  if (scratch_ok(c)) {
+    scratch_bind(wsm, orw, c.bm_word, lane);
+#pragma unroll
+    for (int k = 0; k < kTilesPerWarp; ++k) {
+      scratch_record(wsm, off >> c.shift, (off + sz - 1) >> c.shift);
+      off += 32u * st32;
+    }
+    return 2;
+  }
 #pragma unroll
   for (int k = 0; k < kTilesPerWarp; ++k) {
     red_record(orw, c.bm_word, off >> c.shift, (off + sz - 1) >> c.shift);
@@ -610,20 +694,31 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
 // word(s): no warp analysis, OR is idempotent.  Returns false without side
 // effects otherwise.
 __device__ __forceinline__ bool try_in_object(const uint4 (&r)[kTilesPerWarp], const FastCache& c,
-                                              uint32_t* orw) {
+                                              uint32_t* orw, uint32_t wsm, int lane) {
   const uint32_t osz = uint32_t(c.size);
   uint32_t e0[kTilesPerWarp], e1[kTilesPerWarp];
   bool ok = true;
+  uint32_t nclip = 0;
 #pragma unroll
   for (int k = 0; k < kTilesPerWarp; ++k) {
     const uint64_t off = ((uint64_t(r[k].y) << 32) | r[k].x) - c.base;
-    const uint32_t off32 = uint32_t(off), size = r[k].z;
+    const uint32_t off32 = uint32_t(off), size = r[k].z, room = osz - off32;
+    const bool clip = size > room;   // runs past the object's end: clipped there (R3)
     e0[k] = off32 >> c.shift;
-    e1[k] = (off32 + size - 1) >> c.shift;
+    e1[k] = (off32 + (clip ? room : size) - 1) >> c.shift;
     ok = ok && r[k].w == c.meta && (off >> 32) == 0 && off32 < osz && size != 0 &&
-         size <= osz - off32 && (e1[k] >> 5) - (e0[k] >> 5) < 2;
+         (e1[k] >> 5) - (e0[k] >> 5) < 2;
+    nclip += clip;
   }
   if (!__all_sync(FULL_MASK, ok)) return false;
+  nclip = __reduce_add_sync(FULL_MASK, nclip);
+  if (nclip && lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, clip)>(wsm, nclip);
+  if (scratch_ok(c)) {
+    scratch_bind(wsm, orw, c.bm_word, lane);
+#pragma unroll
+    for (int k = 0; k < kTilesPerWarp; ++k) scratch_record(wsm, e0[k], e1[k]);
+    return true;
+  }
 #pragma unroll
   for (int k = 0; k < kTilesPerWarp; ++k) red_record(orw, c.bm_word, e0[k], e1[k]);
   return true;
@@ -718,6 +813,7 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
     }
   };
 
+  for (uint32_t i = lane; i < kScratchWords; i += 32) sts32(wsm + kOffScratch + 4 * i, 0);
   SlowCache* my = slow_cache();
   my->base = 0; my->size = 0; my->bm_word = 0; my->hit_word = 0;
   my->t_alloc = 0; my->t_free = 0; my->r_lo = 0; my->shift = 0; my->obj = kNone; my->meta = kNever;
@@ -725,6 +821,7 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
     *slow_counts() = WarpCounts{0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     sts64(wsm + kOffPos, 0);
     sts64(wsm + kOffHi, 0);
+    sts64(wsm + kOffScBase, kNoScratch);
     for (int s = 0; s < kStages; ++s) mbar_init(wsm + kOffFull + 8 * s, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     for (int s = 0; s < kStages; ++s) fetch(s);
@@ -767,13 +864,13 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
     if (lane == 0 && !never) fetch(s);
     __syncwarp();
     if (uni && ntiles == kTilesPerWarp) {
-      const int how = try_affine(r4, c, p.orw, lane);
+      const int how = try_affine(r4, c, p.orw, wsm, lane);
       if (how) {
         fast_rec += kTilesPerWarp;
         if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, aff_u)>(wsm + (how == 1 ? 0 : 4), kTilesPerWarp);
         continue;
       }
-      if (try_in_object(r4, c, p.orw)) {
+      if (try_in_object(r4, c, p.orw, wsm, lane)) {
         fast_rec += kTilesPerWarp;
         if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, fast)>(wsm, kTilesPerWarp);
         continue;
@@ -788,13 +885,16 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
       if (uni) {
         // fast check in 32-bit object-relative arithmetic
         const uint64_t off = ((uint64_t(r.y) << 32) | r.x) - c.base;
-        const uint32_t off32 = uint32_t(off), size = r.z, osz = uint32_t(c.size);
+        const uint32_t off32 = uint32_t(off), size = r.z, osz = uint32_t(c.size), room = osz - off32;
+        const bool clip = size > room;   // runs past the object's end: clipped there (R3)
         const uint32_t e0 = off32 >> c.shift;
-        const uint32_t e1 = (off32 + size - 1) >> c.shift;
+        const uint32_t e1 = (off32 + (clip ? room : size) - 1) >> c.shift;
         const bool ok = present && r.w == c.meta && (off >> 32) == 0 && off32 < osz &&
-                        size != 0 && size <= osz - off32 && (e1 >> 5) - (e0 >> 5) < 2;
+                        size != 0 && (e1 >> 5) - (e0 >> 5) < 2;
         if (__all_sync(FULL_MASK, ok)) {
-          fast_or(p.orw, c.bm_word, e0, e1, lane);
+          const uint32_t nclip = __popc(__ballot_sync(FULL_MASK, clip));
+          if (nclip && lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, clip)>(wsm, nclip);
+          fast_or_c(wsm, p.orw, c, e0, e1, lane);
           ++fast_rec;
           if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, fast)>(wsm, 1);
           continue;
@@ -808,6 +908,10 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
       const uint32_t o0 = __shfl_sync(FULL_MASK, my->obj, 0);
       uni = __all_sync(FULL_MASK, c.meta == m0 && my->obj == o0 && m0 != kNever && c.size <= 0xFFFFFFFFull);
     }
+  }
+  if (kScratchWords > 0) {   // the small-object scratch's last bits
+    const uint64_t sc = lds64(wsm + kOffScBase);
+    if (sc != kNoScratch) scratch_flush(wsm, p.orw, sc, lane);
   }
   // A5: counters -- fast-path records per lane plus the warp's slow-path sums
   const uint32_t fr = __reduce_add_sync(FULL_MASK, fast_rec);
