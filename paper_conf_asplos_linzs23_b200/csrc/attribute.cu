@@ -495,7 +495,12 @@ __device__ __noinline__ void process_slow(const AttrParams& p, uint4 r, bool pre
     const uint64_t gb1 = c->bm_word * 32 + ((off_end - 1) >> c->shift);
     const uint64_t w0 = gb0 >> 5, w1 = gb1 >> 5;
     if (w1 - w0 >= 2) {
-      enqueue_range(p.rq, p.rq_cap, p.ctr + p.rq_slot, p.orw, gb0, gb1, ovf);
+      // a whole-object memcpy / memset range is expanded once per trace: the
+      // first such record of the object queues it, later ones (memset then
+      // memcpy-in then memcpy-out ...) set no new bit (OR is idempotent)
+      const bool whole = addr == c->base && off_end == c->size;
+      if (!whole || atomicOr(p.rfull + obj, 1u) == 0)
+        enqueue_range(p.rq, p.rq_cap, p.ctr + p.rq_slot, p.orw, gb0, gb1, ovf);
     } else if (w1 == w0) {
       key0 = w0; m0 = bits_mask(gb0 & 31, gb1 & 31);
     } else {

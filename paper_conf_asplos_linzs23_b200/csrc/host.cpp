@@ -35,6 +35,7 @@ struct Layout {
   uint64_t orw, first, last, ctr;           // dynamic (reset per trace)
   uint64_t dyn_end;
   uint64_t objs, seg_start, seg_cand_off, seg, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
+  uint64_t rfull;                 // per object: a whole-object range was queued in this trace
   uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage;
   // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
@@ -303,6 +304,7 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   L.first = put(4 * n);
   L.last = put(4 * n);
   L.ctr = put(8 * C_SLOTS);
+  L.rfull = put(4 * n);
   L.dyn_end = off;
   L.objs = put(sizeof(DevObj) * n);
   L.seg_start = put(8 * S);
@@ -421,6 +423,7 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   p.first = at<uint32_t>(c, c->L.first);
   p.last = at<uint32_t>(c, c->L.last);
   p.ctr = at<unsigned long long>(c, c->L.ctr);
+  p.rfull = at<uint32_t>(c, c->L.rfull);
   p.rq = at<RangeEntry>(c, c->L.rq);
   p.rq_cap = c->rq_cap;
   p.rq_slot = (c->attr_calls & 1) ? C_RQ_COUNT_ALT : C_RQ_COUNT;

@@ -78,6 +78,7 @@ struct AttrParams {
   uint32_t* first;
   uint32_t* last;
   unsigned long long* ctr;
+  uint32_t* rfull;           // [n_obj] 1 once a whole-object range was queued (zeroed by the reset)
   RangeEntry* rq;
   uint32_t rq_cap;
   uint32_t rq_slot;          // counter slot of this call's range-queue count (C_RQ_COUNT / _ALT)
