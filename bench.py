@@ -365,6 +365,25 @@ def main():
     ms_step = ms_total / a.steps
     value = N / (ms_step / 1e3)
 
+    # calibration: attainable streaming-read bandwidth over the same record
+    # buffer (a torch reduction, not part of the path), so that the
+    # attribution can also be read as a fraction of "just reading the records"
+    cal = None
+    if not chunked:
+        v64 = d_recs.view(torch.int64)
+        for _ in range(3):
+            v64.sum()
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        c0.record(stream)
+        for _ in range(5):
+            v64.sum()
+        c1.record(stream)
+        torch.cuda.synchronize()
+        rd_ms = c0.elapsed_time(c1) / 5
+        cal = {"read_gbs": 16.0 * n_local / (rd_ms / 1e3) / 1e9, "ms": rd_ms,
+               "how": "torch.sum over the resident record buffer viewed as int64 (read-only stream)"}
+
     # touched shadow words of the last step (algorithmic write-back of A3/A4)
     touched = int(torch.count_nonzero(s.or_words()).item())
     stats, ctr = s.object_stats()
@@ -440,6 +459,8 @@ def main():
                      "algorithmic_bytes": alg_bytes,
                      "bytes_rule": "16 B per record + 4 B per touched shadow word",
                      "peak_source": hbm_src},
+        "calibration": None if cal is None else dict(cal, attribution_frac_of_read=cal["read_gbs"] and
+                                                     (16.0 * n_local / (attr_ms / 1e3) / 1e9) / cal["read_gbs"]),
         "cpu_baseline": cpu,
         "e2e": {"value": n_e2e * world / e2e_s, "unit": "records/s", "h2d_bytes_per_step": 16 * n_e2e,
                 "records_per_rank": n_e2e,
