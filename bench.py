@@ -57,6 +57,9 @@ def args_():
     ap.add_argument("--config", default="C2", choices=sorted(WORKLOADS))
     ap.add_argument("--records", type=int, default=None, help="override the record count")
     ap.add_argument("--e2e-steps", type=int, default=None)
+    ap.add_argument("--merge", default="peers", choices=["peers", "nccl"],
+                    help="N>1 exchange step: drgpum_merge_peers over torch symmetric memory (one "
+                         "kernel per rank, NVLink P2P) or NCCL all-to-all + merge_or + all-gather")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-next", action="store_true", help="skip the SURVEY §8(f) NEXT-row timings")
     ap.add_argument("--no-graph", action="store_true",
@@ -268,7 +271,20 @@ def main():
                 dp.gen(lo + c0, lo + c1, out=d_recs[16 * c0:16 * c1])
             chunks = [(0, n_local)]
         torch.cuda.synchronize()
-    s = Session(prog.objects, prog.kinds)
+    sm, merge_note = None, "none (1 rank)"
+    if world > 1 and a.merge == "peers":
+        from paper_conf_asplos_linzs23_b200.parallel import SymmetricMerge
+        try:
+            sm = SymmetricMerge()
+            s = Session(prog.objects, prog.kinds, workspace_alloc=sm.alloc)
+            merge_note = "drgpum_merge_peers over torch symmetric memory (one kernel per rank, NVLink P2P)"
+        except Exception as e:   # symmetric memory unavailable: the NCCL exchange instead, said so
+            sm = None
+            merge_note = f"NCCL all_to_all + merge_or + all_gather (symmetric memory unavailable: {e})"
+    if sm is None:
+        s = Session(prog.objects, prog.kinds)
+        if world > 1 and a.merge == "nccl":
+            merge_note = "NCCL all_to_all + merge_or + all_gather"
     stream = torch.cuda.current_stream()
 
     def barrier():
@@ -289,7 +305,7 @@ def main():
             if ev: ev["attr"][k][1].record(stream)
         if ev: ev["merge"][0].record(stream)
         if world > 1:
-            merge_session(s)
+            sm.merge(s) if sm is not None else merge_session(s)
         if ev: ev["merge"][1].record(stream)
         if ev: ev["fin"][0].record(stream)
         s.finalize()
@@ -403,7 +419,7 @@ def main():
         s.reset()
         s.attribute(pinned)                 # drgpum_trace_attribute_host: H2D inside
         if world > 1:
-            merge_session(s)
+            sm.merge(s) if sm is not None else merge_session(s)
         st_h, ctr_h = s.object_stats()      # D2H of the result
         rep_h = s.patterns()
     torch.cuda.synchronize()
@@ -448,7 +464,7 @@ def main():
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
         "data": f"synthetic (tracegen {prog.name}, seed {prog.seed:#x})",
         "config": {"workload": WORKLOADS[a.config], "records": N, "objects": prog.n_obj,
-                   "n_api": prog.n_api, "parallelism": f"record-range x{world}",
+                   "n_api": prog.n_api, "parallelism": f"record-range x{world}", "merge": merge_note,
                    "l2": f"inputs larger than L2 ({16 * N / 2**30:.2f} GiB of records streamed per step)",
                    "shadow_words": int(s.view.or_words), "touched_words": touched},
         "phases_ms": {"reset": float(ph_mean[0]), "attribute": attr_ms,

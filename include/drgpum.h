@@ -34,7 +34,7 @@
  *     two tiny event/stream objects for drgpum_trace_attribute_host.
  *   - One context per device (per rank).  A context is not thread-safe.
  *   - Call order: create -> objects_load -> workspace_bind ->
- *     { trace_attribute | trace_attribute_host }* -> [merge_or ...] ->
+ *     { trace_attribute | trace_attribute_host }* -> [merge_or ... | merge_peers] ->
  *     finalize / object_stats / patterns.  drgpum_reset starts a new trace on
  *     the same objects.  Out-of-order calls return DRGPUM_ESTATE.
  */
@@ -239,6 +239,26 @@ DRGPUM_API drgpum_status drgpum_object_layout(const drgpum_ctx *ctx, drgpum_obje
 DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx *ctx, const uint32_t *d_in,
     uint32_t n_src, uint64_t src_stride_words, uint64_t word_lo,
     uint64_t word_hi, void *stream);
+
+/* Peer-memory merge ("P2P intermediate"; the exchange step of
+ * the record-range sharding, §5.2 l.266-268 bitmaps and §5.1 l.242
+ * first/last, merged by OR / MIN / MAX / SUM): ONE kernel per rank, over
+ * NVLink peer pointers, instead of all-to-all + merge_or + all-gather.
+ * h_peer_ws is a HOST array of n_peers device pointers: the workspace base of
+ * every rank (index = rank; h_peer_ws[rank] must be this context's own
+ * workspace), each bound to a context loaded with the same objects and
+ * timeline (identical layouts) and addressable from this device -- the same
+ * device, or mapped through NVLink (CUDA IPC / torch symmetric memory).
+ * Rank r owns the r-th of n_peers equal slices of the OR words and of the
+ * objects: it reads its slices from every peer, combines them and stores the
+ * result into every peer's slices; rank 0 also sums the counters.  After ALL
+ * ranks' calls have completed (the caller's barrier), every workspace holds
+ * the merged shadow, bit-identical to a single-GPU run.  The caller must also
+ * barrier BEFORE the call (every rank's attribution done).  Asynchronous.
+ * EINVAL: n_peers == 0 or > 64, rank >= n_peers, a NULL / unaligned pointer,
+ * or h_peer_ws[rank] != this workspace. */
+DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx *ctx, void *const *h_peer_ws,
+    uint32_t n_peers, uint32_t rank, void *stream);
 
 /* Enqueue the per-object reductions and the pattern classification on the
  * device (thresholds NULL = defaults).  Asynchronous; the results stay on

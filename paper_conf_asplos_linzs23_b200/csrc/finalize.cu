@@ -537,6 +537,58 @@ __global__ void __launch_bounds__(256) merge_or_kernel(uint32_t* __restrict__ ds
   }
 }
 
+// B7' (peer memory): the one exchange step as ONE kernel per rank over
+// NVLink peer pointers (symmetric memory / CUDA IPC).  Rank r owns the word
+// slice [w_lo, w_hi) of the OR words and the object slice [o_lo, o_hi): it
+// reads its slice from every peer's shadow (its own included), ORs /
+// MINs / MAXes them, and stores the result into every peer's slice, so that
+// after a barrier every rank holds the merged shadow.  Slices of different
+// ranks are disjoint, so the ranks' kernels never touch the same word.  Rank
+// 0 also sums the counters.  OR / MIN / MAX / SUM are associative and
+// commutative: the result is bit-exact for any number of ranks.
+__global__ void __launch_bounds__(256) merge_peers_kernel(const MergePeersParams q) {
+  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
+  // OR words, 16 B at a time (the slice bounds are multiples of 4 words)
+  const uint64_t v_lo = q.w_lo / 4, v_hi = q.w_hi / 4;
+  for (uint64_t i = v_lo + tid; i < v_hi; i += nth) {
+    uint4 v = make_uint4(0, 0, 0, 0);
+    for (uint32_t r = 0; r < q.n_peers; ++r) {
+      const uint4 x = __ldcg(reinterpret_cast<const uint4*>(q.peer[r] + q.or_off) + i);
+      v.x |= x.x; v.y |= x.y; v.z |= x.z; v.w |= x.w;
+    }
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      __stcg(reinterpret_cast<uint4*>(q.peer[r] + q.or_off) + i, v);
+  }
+  for (uint64_t o = q.o_lo + tid; o < q.o_hi; o += nth) {
+    uint32_t f = 0xFFFFFFFFu, l = 0;
+    for (uint32_t r = 0; r < q.n_peers; ++r) {
+      f = min(f, __ldcg(reinterpret_cast<const uint32_t*>(q.peer[r] + q.first_off) + o));
+      l = max(l, __ldcg(reinterpret_cast<const uint32_t*>(q.peer[r] + q.last_off) + o));
+    }
+    for (uint32_t r = 0; r < q.n_peers; ++r) {
+      __stcg(reinterpret_cast<uint32_t*>(q.peer[r] + q.first_off) + o, f);
+      __stcg(reinterpret_cast<uint32_t*>(q.peer[r] + q.last_off) + o, l);
+    }
+  }
+  if (q.rank == 0 && tid < 5) {   // records, attributed, unattributed, clipped, invalid
+    unsigned long long sum = 0;
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      sum += __ldcg(reinterpret_cast<const unsigned long long*>(q.peer[r] + q.ctr_off) + tid);
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      __stcg(reinterpret_cast<unsigned long long*>(q.peer[r] + q.ctr_off) + tid, sum);
+  }
+}
+
+int launch_merge_peers(const MergePeersParams& q, int num_sms, cudaStream_t s) {
+  const uint64_t work = max((q.w_hi - q.w_lo) / 4, q.o_hi - q.o_lo);
+  uint64_t b = (work + 255) / 256;
+  if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
+  if (b < 1) b = 1;
+  merge_peers_kernel<<<(unsigned)b, 256, 0, s>>>(q);
+  return 1;
+}
+
 int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src, uint64_t src_stride,
                     uint64_t n_words, int num_sms, cudaStream_t s) {
   if (!n_words || !n_src) return 0;

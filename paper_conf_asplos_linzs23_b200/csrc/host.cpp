@@ -766,6 +766,41 @@ DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx* ctx, const uint32_t* d_in, 
   return DRGPUM_OK;
 }
 
+DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx* ctx, void* const* h_peer_ws, uint32_t n_peers,
+                                            uint32_t rank, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers before workspace_bind");
+  if (!h_peer_ws || n_peers == 0 || n_peers > kMaxPeers || rank >= n_peers)
+    return fail(ctx, DRGPUM_EINVAL, "merge_peers: need 1 <= n_peers <= %u and rank < n_peers", kMaxPeers);
+  if (h_peer_ws[rank] != ctx->ws)
+    return fail(ctx, DRGPUM_EINVAL, "merge_peers: h_peer_ws[rank] is not this context's workspace");
+  MergePeersParams q{};
+  for (uint32_t r = 0; r < n_peers; ++r) {
+    if (!h_peer_ws[r] || reinterpret_cast<uintptr_t>(h_peer_ws[r]) % kAlign)
+      return fail(ctx, DRGPUM_EINVAL, "merge_peers: peer %u workspace NULL or not 256-B aligned", r);
+    q.peer[r] = static_cast<uint8_t*>(h_peer_ws[r]);
+  }
+  q.n_peers = n_peers;
+  q.rank = rank;
+  q.or_off = ctx->L.orw;
+  q.first_off = ctx->L.first;
+  q.last_off = ctx->L.last;
+  q.ctr_off = ctx->L.ctr;
+  // the OR-word section is padded to 256 B (zero in every shadow), so the
+  // slices can be rounded to whole 16-B vectors
+  const uint64_t w4 = (ctx->bitmap_words + ctx->hit_words + 3) / 4 * 4;
+  const uint64_t sw = ((w4 + n_peers - 1) / n_peers + 3) / 4 * 4;
+  q.w_lo = std::min<uint64_t>(uint64_t(rank) * sw, w4);
+  q.w_hi = std::min<uint64_t>(q.w_lo + sw, w4);
+  const uint64_t so = (ctx->n_obj + n_peers - 1) / n_peers;
+  q.o_lo = std::min<uint64_t>(uint64_t(rank) * so, ctx->n_obj);
+  q.o_hi = std::min<uint64_t>(q.o_lo + so, ctx->n_obj);
+  ctx->launches += launch_merge_peers(q, ctx->num_sms, as_stream(stream));
+  ctx->final_valid = false;
+  CK(cudaGetLastError());
+  return DRGPUM_OK;
+}
+
 DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_thresholds_t* th, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "finalize before workspace_bind");

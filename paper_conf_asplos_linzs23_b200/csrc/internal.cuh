@@ -166,6 +166,16 @@ struct FinalParams {
   unsigned long long* ctr;
 };
 
+// Peer-memory merge (B7'): workspace base pointers of every rank, indexed by rank.
+constexpr uint32_t kMaxPeers = 64;
+struct MergePeersParams {
+  uint8_t* peer[kMaxPeers];
+  uint32_t n_peers, rank;
+  uint64_t or_off, first_off, last_off, ctr_off;   // byte offsets inside a workspace
+  uint64_t w_lo, w_hi;                             // owned OR-word slice (multiples of 4)
+  uint64_t o_lo, o_hi;                             // owned object slice
+};
+
 // Launchers (return the number of kernels enqueued).
 int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);   // p.rq_slot alternates per call
 int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
@@ -174,6 +184,7 @@ int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
 int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_bytes, int num_sms, cudaStream_t s);
+int launch_merge_peers(const MergePeersParams& q, int num_sms, cudaStream_t s);
 int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src,
                     uint64_t src_stride, uint64_t n_words, int num_sms, cudaStream_t s);
 

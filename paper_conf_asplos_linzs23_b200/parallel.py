@@ -14,6 +14,13 @@ are small: all_reduce MIN / MAX / SUM.
 The collective choreography (``merge_shadow``) takes the OR step as a
 callable so the same code is exercised with gloo on CPU tensors in the tests;
 on the GPU path ``Session`` passes its merge_or kernel.
+
+``SymmetricMerge`` is the NVLink-native alternative: every rank's workspace
+lives in torch symmetric memory, and ONE library kernel per rank
+(``drgpum_merge_peers``) reads its owned slice from every peer, combines it
+and stores the result into every peer -- no NCCL staging buffers, no second
+pass.  Barriers before and after it (the symmetric-memory handle's device
+barrier) order it against the peers' attribution and finalize.
 """
 import torch
 import torch.distributed as dist
@@ -80,3 +87,31 @@ def merge_session(session, group=None):
         session.merge_or(recv, recv.shape[0], S, lo, hi)
 
     merge_shadow(orw, first, last, ctr, group, or_reduce)
+
+
+class SymmetricMerge:
+    """Workspace allocator + merge over torch symmetric memory (NVLink P2P).
+
+    usage:  sm = SymmetricMerge(group); s = Session(objs, kinds, workspace_alloc=sm.alloc)
+            ... s.attribute(...) ...; sm.merge(s)
+    """
+
+    def __init__(self, group=None):
+        self.group = group if group is not None else dist.group.WORLD
+        self.handle = None
+
+    def alloc(self, nbytes, device):
+        import torch.distributed._symmetric_memory as symm_mem
+        buf = symm_mem.empty(nbytes, dtype=torch.uint8, device=device)
+        self.handle = symm_mem.rendezvous(buf, self.group)
+        self.buf = buf
+        return buf
+
+    def peer_ptrs(self):
+        return [int(p) for p in self.handle.buffer_ptrs]
+
+    def merge(self, session, stream=None):
+        h = self.handle
+        h.barrier(channel=0)            # every rank's attribution is done
+        session.merge_peers(self.peer_ptrs(), h.rank, stream)
+        h.barrier(channel=0)            # every slice is merged everywhere

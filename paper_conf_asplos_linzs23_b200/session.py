@@ -38,7 +38,7 @@ class Session:
     kinds:   uint8 array, the GPU-API kind of every timestamp.
     """
 
-    def __init__(self, objects, kinds, device=None, structured=False, frequency=False):
+    def __init__(self, objects, kinds, device=None, structured=False, frequency=False, workspace_alloc=None):
         if not torch.cuda.is_available():
             raise RuntimeError("drgpum Session needs a CUDA device (there is no CPU fallback)")
         self.L = _lib.load()
@@ -61,8 +61,10 @@ class Session:
             check(self._h, self.L.drgpum_set_features(self._h, feats))
         nbytes = ctypes.c_uint64()
         check(self._h, self.L.drgpum_workspace_size(self._h, ctypes.byref(nbytes)))
-        self.workspace = torch.empty(max(int(nbytes.value), 256), dtype=torch.uint8,
-                                     device=self.device)
+        # workspace_alloc(nbytes, device) -> uint8 CUDA tensor (e.g. torch
+        # symmetric memory for merge_peers); default torch.empty
+        alloc = workspace_alloc or (lambda nb, dev: torch.empty(nb, dtype=torch.uint8, device=dev))
+        self.workspace = alloc(max(int(nbytes.value), 256), self.device)
         with torch.cuda.device(self.device):
             check(self._h, self.L.drgpum_workspace_bind(
                 self._h, ctypes.c_void_p(self.workspace.data_ptr()), self.workspace.numel(),
@@ -238,6 +240,13 @@ class Session:
         check(self._h, self.L.drgpum_merge_or(self._h, ctypes.c_void_p(src.data_ptr()), n_src,
                                               src_stride_words, word_lo, word_hi,
                                               _stream_handle(stream)))
+
+    def merge_peers(self, peer_ptrs, rank, stream=None):
+        """drgpum_merge_peers: peer_ptrs = workspace base pointers (ints) of every
+        rank, index = rank (this session's own at ``rank``)."""
+        arr = (ctypes.c_void_p * len(peer_ptrs))(*[ctypes.c_void_p(int(x)) for x in peer_ptrs])
+        check(self._h, self.L.drgpum_merge_peers(self._h, arr, len(peer_ptrs), rank,
+                                                 _stream_handle(stream)))
 
     def bitmap(self, o):
         """Object o's bitmap as a bool numpy array (copies from the device)."""

@@ -1,0 +1,127 @@
+"""drgpum_merge_peers -- the exchange step as one kernel per rank over peer
+pointers -- checked on one GPU with VIRTUAL peers: P sessions
+of the same program on cuda:0 each attribute one record-range shard, then
+every rank's merge kernel runs over the P workspaces (the pointers a
+symmetric-memory rendezvous would hand out on an NVLink box).  Afterwards
+EVERY session must hold the single-GPU shadow: stats, patterns, counters and
+bitmaps equal to the oracle over the whole trace, bit for bit.  The slices of
+different ranks are disjoint, so running the P kernels one after the other on
+one device is the same computation as running them concurrently on P GPUs.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from oracle import Oracle  # noqa: E402
+from tracegen import build_config, build_tiny, gen_all_records  # noqa: E402
+from tests.test_gpu_parity import expected_or_words  # noqa: E402
+
+
+def _check_against_oracle(s, objs, kinds, recs, orc=None):
+    if orc is None:
+        orc = Oracle(objs, kinds)
+        orc.attribute(recs)
+    ost, octr = orc.stats()
+    orep = orc.patterns()
+    st, ctr = s.object_stats()
+    rep = s.patterns()
+    assert s.consistency_errors() == 0
+    for k in octr.dtype.names:
+        assert int(ctr[k]) == int(octr[k]), k
+    for k in ost.dtype.names:
+        if k != "_pad":
+            assert np.array_equal(st[k], ost[k]), k
+    for k in orep.dtype.names:
+        assert np.array_equal(rep[k], orep[k]), k
+    orw = s.or_words().cpu().numpy().view(np.uint32)
+    assert np.array_equal(orw, expected_or_words(s, orc, objs, kinds))
+    return orc
+
+
+def _virtual_peers(objs, kinds, recs, P):
+    from paper_conf_asplos_linzs23_b200 import Session
+    from paper_conf_asplos_linzs23_b200.parallel import shard_range
+    sessions = [Session(objs, kinds) for _ in range(P)]
+    d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
+    for r, s in enumerate(sessions):
+        lo, hi = shard_range(len(recs), r, P)
+        s.attribute(d[16 * lo: 16 * hi])
+    torch.cuda.synchronize()
+    ptrs = [s.workspace.data_ptr() for s in sessions]
+    for r, s in enumerate(sessions):
+        s.merge_peers(ptrs, r)
+    torch.cuda.synchronize()
+    return sessions
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+def test_virtual_peers_c1(P):
+    p = build_config("C1")
+    recs = gen_all_records(p)
+    orc = None
+    for s in _virtual_peers(p.objects, p.kinds, recs, P):
+        orc = _check_against_oracle(s, p.objects, p.kinds, recs, orc)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_virtual_peers_tiny_reuse(seed):
+    p = build_tiny(4100 + seed)
+    recs = gen_all_records(p)
+    P = 2 + seed % 5
+    orc = None
+    for s in _virtual_peers(p.objects, p.kinds, recs, P):
+        orc = _check_against_oracle(s, p.objects, p.kinds, recs, orc)
+
+
+def test_merge_peers_rejects_bad_arguments():
+    from paper_conf_asplos_linzs23_b200 import Session
+    from paper_conf_asplos_linzs23_b200._lib import DrgpumError
+    p = build_tiny(4200)
+    a, b = Session(p.objects, p.kinds), Session(p.objects, p.kinds)
+    ptrs = [a.workspace.data_ptr(), b.workspace.data_ptr()]
+    with pytest.raises(DrgpumError):
+        a.merge_peers(ptrs, 1)          # ptrs[1] is not a's workspace
+    with pytest.raises(DrgpumError):
+        a.merge_peers(ptrs, 2)          # rank out of range
+    with pytest.raises(DrgpumError):
+        a.merge_peers([], 0)
+    with pytest.raises(DrgpumError):
+        a.merge_peers([ptrs[0], ptrs[1] + 16], 0)   # unaligned peer
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def test_symmetric_memory_single_rank():
+    """The torch symmetric-memory plumbing (allocation, rendezvous, device
+    barrier, peer pointers) around drgpum_merge_peers, with one rank."""
+    import torch.distributed as dist
+    from paper_conf_asplos_linzs23_b200 import Session
+    from paper_conf_asplos_linzs23_b200.parallel import SymmetricMerge
+    if not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ["MASTER_PORT"] = str(_free_port())
+        dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        sm = SymmetricMerge()
+        p = build_config("C1")
+        recs = gen_all_records(p)
+        try:
+            s = Session(p.objects, p.kinds, workspace_alloc=sm.alloc)
+        except Exception as e:   # symmetric memory unavailable in this torch / driver
+            pytest.skip(f"torch symmetric memory unavailable: {e}")
+        s.attribute(torch.from_numpy(recs.view(np.uint8)).cuda())
+        sm.merge(s)
+        torch.cuda.synchronize()
+        assert sm.peer_ptrs() == [s.workspace.data_ptr()]
+        _check_against_oracle(s, p.objects, p.kinds, recs)
+    finally:
+        dist.destroy_process_group()
