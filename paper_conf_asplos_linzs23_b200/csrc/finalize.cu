@@ -130,7 +130,14 @@ __device__ __noinline__ uint32_t interior_zero_run(uint32_t u) {
 // in the first pass and computed in a second pass only when the tile's other
 // runs are all shorter than 30 -- otherwise they cannot change its longest
 // run (dense strided sweeps need them; untouched or sparse regions do not).
-__global__ void __launch_bounds__(256, 4) tile_reduce_kernel(const uint32_t* __restrict__ orw,
+// Blocks per SM (A/B on C2, tools/ab.sh): 4 (64 registers) 60.6 us of
+// finalize; 5 (48, spills) 67.7; 6 (40, spills) 91.2.  Persistent variants
+// with register prefetch (3 and 2 blocks/SM) 79.5 / 75.8, with a 3-stage
+// cp.async ring (2 blocks/SM) 49.8 us of tile_reduce alone vs 40.8.
+#ifndef DRGPUM_TR_BLOCKS
+#define DRGPUM_TR_BLOCKS 4
+#endif
+__global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(const uint32_t* __restrict__ orw,
     const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr) {
   const int lane = threadIdx.x & 31;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctr[C_CONSISTENCY] = 0;   // counted by object_finalize_kernel
