@@ -38,12 +38,12 @@ WORKLOADS = {
     "C4": "C4 LLM-inference-shaped trace (BASELINE configs[3]): 4e9 records over 100K objects "
           "(120 GiB live footprint, reused 4 GiB activation arena), Zipf-skewed hot weights / KV blocks",
     "C5": "C5 scaling sweep (BASELINE configs[4]): 1.6e10 records over 1M objects, streamed through HBM "
-          "in 2^28-record chunks generated on the device",
+          "in 2^30-record chunks generated on the device",
 }
 # configs whose records are generated on the device (tracegen/gen.cu) rather
 # than on the host; traces above RESIDENT_BYTES are streamed in GEN_CHUNK chunks
 DEVICE_GEN = ("C3", "C4", "C5")
-GEN_CHUNK = 1 << 28
+GEN_CHUNK = 1 << 30
 RESIDENT_BYTES = 96 << 30
 FALLBACK_HBM_GBS = 6650.0
 
