@@ -12,10 +12,15 @@ from tracegen import build_config, gen_records
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
 ap.add_argument("--steps", type=int, default=10)
+ap.add_argument("--records", type=int, default=None)
 a = ap.parse_args()
-prog = build_config(a.config)
-recs = gen_records(prog, 0, prog.n_records)
-d = torch.from_numpy(recs.view(np.uint8)).cuda()
+prog = build_config(a.config, **({"n_records": a.records} if a.records else {}))
+if a.config in ("C3", "C4", "C5"):   # device generation (tracegen/gen.cu)
+    from tracegen.device import DeviceProgram
+    d = DeviceProgram(prog).gen(0, prog.n_records)
+else:
+    recs = gen_records(prog, 0, prog.n_records)
+    d = torch.from_numpy(recs.view(np.uint8)).cuda()
 s = Session(prog.objects, prog.kinds)
 for _ in range(3):
     s.reset(); s.attribute(d); s.finalize()
