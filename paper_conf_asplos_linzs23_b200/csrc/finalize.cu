@@ -134,8 +134,16 @@ __device__ __noinline__ uint32_t interior_zero_run(uint32_t u) {
 // finalize; 5 (48, spills) 67.7; 6 (40, spills) 91.2.  Persistent variants
 // with register prefetch (3 and 2 blocks/SM) 79.5 / 75.8, with a 3-stage
 // cp.async ring (2 blocks/SM) 49.8 us of tile_reduce alone vs 40.8.
+// r43 (ncu source page: 20.9M warp-instructions, stalls mostly long_sb on the
+// tile loads): skipping pass-2 words equal to the last searched one or whose
+// inner zeros cannot beat the running max 61.8 vs 60.5 us of finalize (not
+// adopted); grid cap per SM (DRGPUM_TR_GRID_PER_SM) 4 / 8 / 16 / 64 blocks:
+// 66.9 / 67.3 / 60.7 / 62.8 us of finalize -- 16 stays.
 #ifndef DRGPUM_TR_BLOCKS
 #define DRGPUM_TR_BLOCKS 4
+#endif
+#ifndef DRGPUM_TR_GRID_PER_SM
+#define DRGPUM_TR_GRID_PER_SM 16
 #endif
 __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(const uint32_t* __restrict__ orw,
     const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr) {
@@ -482,7 +490,8 @@ __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const Fina
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   if (p.n_obj == 0) return 0;
   const uint64_t tb = (p.n_tiles + 7) / 8;
-  const unsigned g1 = (unsigned)(tb < uint64_t(num_sms) * 16 ? tb : uint64_t(num_sms) * 16);
+  const uint64_t cap1 = uint64_t(num_sms) * DRGPUM_TR_GRID_PER_SM;
+  const unsigned g1 = (unsigned)(tb < cap1 ? tb : cap1);
   tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles, p.n_tiles, p.tile_part, p.ctr);
   const uint64_t gb = (p.n_groups + 7) / 8;
   const unsigned g3 = (unsigned)(gb < uint64_t(num_sms) * 16 ? gb : uint64_t(num_sms) * 16);
