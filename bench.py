@@ -57,9 +57,12 @@ def args_():
     ap.add_argument("--config", default="C2", choices=sorted(WORKLOADS))
     ap.add_argument("--records", type=int, default=None, help="override the record count")
     ap.add_argument("--e2e-steps", type=int, default=None)
-    ap.add_argument("--merge", default="peers", choices=["peers", "nccl"],
-                    help="N>1 exchange step: drgpum_merge_peers over torch symmetric memory (one "
-                         "kernel per rank, NVLink P2P) or NCCL all-to-all + merge_or + all-gather")
+    ap.add_argument("--merge", default="owned", choices=["owned", "peers", "nccl"],
+                    help="N>1 exchange step over torch symmetric memory (NVLink P2P): owned = "
+                         "drgpum_merge_peers_owned + per-rank finalize of its objects + "
+                         "drgpum_gather_peers; peers = drgpum_merge_peers (every rank gets the "
+                         "whole merged shadow, finalizes everything); nccl = all-to-all + "
+                         "merge_or + all-gather")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-next", action="store_true", help="skip the SURVEY §8(f) NEXT-row timings")
     ap.add_argument("--no-graph", action="store_true",
@@ -272,12 +275,14 @@ def main():
             chunks = [(0, n_local)]
         torch.cuda.synchronize()
     sm, merge_note = None, "none (1 rank)"
-    if world > 1 and a.merge == "peers":
+    if world > 1 and a.merge in ("peers", "owned"):
         from paper_conf_asplos_linzs23_b200.parallel import SymmetricMerge
         try:
             sm = SymmetricMerge()
             s = Session(prog.objects, prog.kinds, workspace_alloc=sm.alloc)
-            merge_note = "drgpum_merge_peers over torch symmetric memory (one kernel per rank, NVLink P2P)"
+            merge_note = ("drgpum_merge_peers_owned + finalize of the owned objects + drgpum_gather_peers "
+                          "over torch symmetric memory (NVLink P2P)" if a.merge == "owned" else
+                          "drgpum_merge_peers over torch symmetric memory (one kernel per rank, NVLink P2P)")
         except Exception as e:   # symmetric memory unavailable: the NCCL exchange instead, said so
             sm = None
             merge_note = f"NCCL all_to_all + merge_or + all_gather (symmetric memory unavailable: {e})"
@@ -286,6 +291,21 @@ def main():
         if world > 1 and a.merge == "nccl":
             merge_note = "NCCL all_to_all + merge_or + all_gather"
     stream = torch.cuda.current_stream()
+    owned = sm is not None and a.merge == "owned"
+
+    def do_merge():
+        if world > 1:
+            if owned:
+                sm.merge_owned(s)
+            elif sm is not None:
+                sm.merge(s)
+            else:
+                merge_session(s)
+
+    def do_finalize():
+        s.finalize()
+        if owned:
+            sm.gather(s)
 
     def barrier():
         if world > 1:
@@ -304,11 +324,10 @@ def main():
             s.attribute(src[:16 * (c1 - c0)])
             if ev: ev["attr"][k][1].record(stream)
         if ev: ev["merge"][0].record(stream)
-        if world > 1:
-            sm.merge(s) if sm is not None else merge_session(s)
+        do_merge()
         if ev: ev["merge"][1].record(stream)
         if ev: ev["fin"][0].record(stream)
-        s.finalize()
+        do_finalize()
         if ev: ev["fin"][1].record(stream)
 
     def events():
@@ -418,8 +437,9 @@ def main():
     for _ in range(e2e_steps):
         s.reset()
         s.attribute(pinned)                 # drgpum_trace_attribute_host: H2D inside
-        if world > 1:
-            sm.merge(s) if sm is not None else merge_session(s)
+        do_merge()
+        if owned:
+            do_finalize()
         st_h, ctr_h = s.object_stats()      # D2H of the result
         rep_h = s.patterns()
     torch.cuda.synchronize()

@@ -260,6 +260,37 @@ DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx *ctx, const uint32_t *d_in,
 DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx *ctx, void *const *h_peer_ws,
     uint32_t n_peers, uint32_t rank, void *stream);
 
+/* Owned merge (the exchange step of the record-range sharding
+ * with the finalize sharded by object, §5.2 l.266-268 bitmaps and
+ * §5.1 l.242 first/last): rank r owns the objects [o_lo, o_hi) whose
+ * boundaries split (bitmap words + objects) into n_peers near-equal parts;
+ * ONE kernel reads those objects' bitmaps, hit rows and first/last from every
+ * peer (h_peer_ws as for drgpum_merge_peers) and stores the OR / MIN / MAX
+ * into THIS workspace only; rank 0 also sums the counters into every peer.
+ * Then drgpum_finalize reduces and classifies only the owned objects, and
+ * drgpum_gather_peers shares their stats and reports.  Compared with
+ * drgpum_merge_peers, nothing is written to the peers' shadows (half the
+ * NVLink traffic) and the finalize work is 1/n_peers per rank; the price is
+ * that afterwards this workspace's shadow (bitmaps, hit rows, first/last) is
+ * merged for the owned objects only.  Barriers as for drgpum_merge_peers
+ * (before: all attribution done; after: all merges done).  Asynchronous.
+ * EINVAL as for drgpum_merge_peers. */
+DRGPUM_API drgpum_status drgpum_merge_peers_owned(drgpum_ctx *ctx, void *const *h_peer_ws,
+    uint32_t n_peers, uint32_t rank, void *stream);
+
+/* After drgpum_merge_peers_owned + drgpum_finalize on every rank (and a
+ * barrier): stores this rank's objects' stats and pattern reports into every
+ * peer's workspace and adds its consistency-violation count into every peer's
+ * total.  After all ranks' calls have completed (barrier), object_stats,
+ * patterns and consistency_errors return the single-GPU results on every
+ * rank.  Asynchronous.  ESTATE without a preceding owned merge + finalize;
+ * EINVAL for bad peers or an n_peers / rank different from the merge's.
+ * object_stats / patterns after an owned merge return ESTATE until the
+ * gather is done, and patterns with other thresholds than the finalize's
+ * return ESTATE (a re-finalize would cover the owned objects only). */
+DRGPUM_API drgpum_status drgpum_gather_peers(drgpum_ctx *ctx, void *const *h_peer_ws,
+    uint32_t n_peers, uint32_t rank, void *stream);
+
 /* Enqueue the per-object reductions and the pattern classification on the
  * device (thresholds NULL = defaults).  Asynchronous; the results stay on
  * the device until object_stats / patterns copy them out. */

@@ -404,7 +404,7 @@ __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const Fina
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
   drgpum_object_stats_t* stats = static_cast<drgpum_object_stats_t*>(p.stats);
   drgpum_pattern_report_t* reps = static_cast<drgpum_pattern_report_t*>(p.reports);
-  for (uint64_t o = gwarp; o < p.n_obj; o += nwarps) {
+  for (uint64_t o = p.o_lo + gwarp; o < p.o_hi; o += nwarps) {
     // ---- bitmap groups of o, in order
     const uint32_t t0 = p.group_off[o], t1 = p.group_off[o + 1];
     BitMonoid bm = bm_identity();
@@ -489,16 +489,18 @@ __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const Fina
 
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   if (p.n_obj == 0) return 0;
-  const uint64_t tb = (p.n_tiles + 7) / 8;
+  const uint64_t nt = p.t_hi - p.t_lo, ng = p.g_hi - p.g_lo, no = p.o_hi - p.o_lo;
+  const uint64_t tb = (nt + 7) / 8;
   const uint64_t cap1 = uint64_t(num_sms) * DRGPUM_TR_GRID_PER_SM;
   const unsigned g1 = (unsigned)(tb < cap1 ? tb : cap1);
-  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles, p.n_tiles, p.tile_part, p.ctr);
-  const uint64_t gb = (p.n_groups + 7) / 8;
+  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles + p.t_lo, nt, p.tile_part + p.t_lo, p.ctr);
+  const uint64_t gb = (ng + 7) / 8;
   const unsigned g3 = (unsigned)(gb < uint64_t(num_sms) * 16 ? gb : uint64_t(num_sms) * 16);
-  group_reduce_kernel<<<g3 ? g3 : 1, 256, 0, s>>>(p.groups, p.n_groups, p.tile_part, p.group_part);
+  group_reduce_kernel<<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
   constexpr unsigned wpb = kFinThreads / 32;   // one warp per object
-  const uint64_t ob = (p.n_obj + wpb - 1) / wpb;
-  const unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
+  const uint64_t ob = (no + wpb - 1) / wpb;
+  unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
+  if (g2 == 0) g2 = 1;
   if (p.n_acc <= kSmemAcc)
     object_finalize_kernel<true><<<g2, kFinThreads, 16 * ((p.n_acc + 3) / 4 + (p.n_acc + 15) / 16), s>>>(p);
   else
@@ -602,6 +604,85 @@ int launch_merge_peers(const MergePeersParams& q, int num_sms, cudaStream_t s) {
   if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
   if (b < 1) b = 1;
   merge_peers_kernel<<<(unsigned)b, 256, 0, s>>>(q);
+  return 1;
+}
+
+// B7'': owned merge.  Reads rank r's objects' shadow from every peer and
+// stores the OR / MIN / MAX into rank r's workspace only (no write-back to
+// the peers: each rank finalizes its own objects, gather_peers shares the
+// results).  NVLink traffic per rank: (P-1)/P of the shadow read, nothing
+// written remotely -- half of merge_peers_kernel's.
+__global__ void __launch_bounds__(256) merge_owned_kernel(const MergeOwnedParams q) {
+  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
+  uint8_t* const own = q.peer[q.rank];
+  for (uint64_t i = q.b_lo / 4 + tid; i < q.b_hi / 4; i += nth) {   // bitmaps: 4-word aligned per object
+    uint4 v = make_uint4(0, 0, 0, 0);
+    for (uint32_t r = 0; r < q.n_peers; ++r) {
+      const uint4 x = __ldcg(reinterpret_cast<const uint4*>(q.peer[r] + q.or_off) + i);
+      v.x |= x.x; v.y |= x.y; v.z |= x.z; v.w |= x.w;
+    }
+    __stcg(reinterpret_cast<uint4*>(own + q.or_off) + i, v);
+  }
+  for (uint64_t w = q.h_lo + tid; w < q.h_hi; w += nth) {           // hit rows
+    uint32_t v = 0;
+    for (uint32_t r = 0; r < q.n_peers; ++r) v |= __ldcg(reinterpret_cast<const uint32_t*>(q.peer[r] + q.or_off) + w);
+    __stcg(reinterpret_cast<uint32_t*>(own + q.or_off) + w, v);
+  }
+  for (uint64_t o = q.o_lo + tid; o < q.o_hi; o += nth) {
+    uint32_t f = 0xFFFFFFFFu, l = 0;
+    for (uint32_t r = 0; r < q.n_peers; ++r) {
+      f = min(f, __ldcg(reinterpret_cast<const uint32_t*>(q.peer[r] + q.first_off) + o));
+      l = max(l, __ldcg(reinterpret_cast<const uint32_t*>(q.peer[r] + q.last_off) + o));
+    }
+    __stcg(reinterpret_cast<uint32_t*>(own + q.first_off) + o, f);
+    __stcg(reinterpret_cast<uint32_t*>(own + q.last_off) + o, l);
+  }
+  if (q.rank == 0 && tid < 5) {   // records, attributed, unattributed, clipped, invalid
+    unsigned long long sum = 0;
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      sum += __ldcg(reinterpret_cast<const unsigned long long*>(q.peer[r] + q.ctr_off) + tid);
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      __stcg(reinterpret_cast<unsigned long long*>(q.peer[r] + q.ctr_off) + tid, sum);
+  }
+}
+
+int launch_merge_owned(const MergeOwnedParams& q, int num_sms, cudaStream_t s) {
+  const uint64_t work = max(max((q.b_hi - q.b_lo) / 4, q.h_hi - q.h_lo), max(q.o_hi - q.o_lo, uint64_t(5)));
+  uint64_t b = (work + 255) / 256;
+  if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
+  merge_owned_kernel<<<(unsigned)b, 256, 0, s>>>(q);
+  return 1;
+}
+
+// B7'': gather of the finalized stats / reports of rank r's objects into
+// every peer (u32 copies; both sections are 4-B multiples per object).
+__global__ void __launch_bounds__(256) gather_peers_kernel(const GatherParams q) {
+  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
+  const uint8_t* const own = q.peer[q.rank];
+  for (uint32_t r = 0; r < q.n_peers; ++r) {
+    if (r == q.rank) continue;
+    for (uint64_t i = q.s_lo / 4 + tid; i < q.s_hi / 4; i += nth)
+      reinterpret_cast<uint32_t*>(q.peer[r] + q.stats_off)[i] =
+          reinterpret_cast<const uint32_t*>(own + q.stats_off)[i];
+    for (uint64_t i = q.r_lo / 4 + tid; i < q.r_hi / 4; i += nth)
+      reinterpret_cast<uint32_t*>(q.peer[r] + q.reports_off)[i] =
+          reinterpret_cast<const uint32_t*>(own + q.reports_off)[i];
+  }
+  if (tid == 0) {
+    const unsigned long long mine = reinterpret_cast<const unsigned long long*>(own + q.ctr_off)[C_CONSISTENCY];
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      atomicAdd(reinterpret_cast<unsigned long long*>(q.peer[r] + q.ctr_off) + C_CONSISTENCY_ALL, mine);
+  }
+}
+
+int launch_gather_peers(const GatherParams& q, int num_sms, cudaStream_t s) {
+  const uint64_t work = max((q.s_hi - q.s_lo) / 4, (q.r_hi - q.r_lo) / 4);
+  uint64_t b = (work + 255) / 256;
+  if (b > uint64_t(num_sms) * 4) b = uint64_t(num_sms) * 4;
+  if (b < 1) b = 1;
+  gather_peers_kernel<<<(unsigned)b, 256, 0, s>>>(q);
   return 1;
 }
 

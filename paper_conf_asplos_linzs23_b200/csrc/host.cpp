@@ -89,6 +89,10 @@ struct drgpum_ctx {
   // finalize cache
   bool final_valid = false;
   drgpum_thresholds_t final_th{2, 80, 80};
+  // owned merge: this rank holds the merged shadow of objects [own_lo, own_hi) only
+  bool owned = false, gathered = false;
+  uint64_t own_lo = 0, own_hi = 0;
+  uint32_t own_P = 0, own_rank = 0;
   // host ingest
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_used[2] = {nullptr, nullptr};
@@ -401,6 +405,7 @@ drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s) {
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
     CK(cudaMemsetAsync(ctx->ws + ctx->L.fq_cells, 0, ctx->L.fq_end - ctx->L.fq_cells, s));
   ctx->final_valid = false;
+  ctx->owned = ctx->gathered = false;
   return DRGPUM_OK;
 }
 
@@ -766,20 +771,42 @@ DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx* ctx, const uint32_t* d_in, 
   return DRGPUM_OK;
 }
 
+static drgpum_status check_peers(drgpum_ctx* ctx, const char* what, void* const* h_peer_ws,
+                                 uint32_t n_peers, uint32_t rank, uint8_t** out) {
+  if (!h_peer_ws || n_peers == 0 || n_peers > kMaxPeers || rank >= n_peers)
+    return fail(ctx, DRGPUM_EINVAL, "%s: need 1 <= n_peers <= %u and rank < n_peers", what, kMaxPeers);
+  if (h_peer_ws[rank] != ctx->ws)
+    return fail(ctx, DRGPUM_EINVAL, "%s: h_peer_ws[rank] is not this context's workspace", what);
+  for (uint32_t r = 0; r < n_peers; ++r) {
+    if (!h_peer_ws[r] || reinterpret_cast<uintptr_t>(h_peer_ws[r]) % kAlign)
+      return fail(ctx, DRGPUM_EINVAL, "%s: peer %u workspace NULL or not 256-B aligned", what, r);
+    out[r] = static_cast<uint8_t*>(h_peer_ws[r]);
+  }
+  return DRGPUM_OK;
+}
+
+// Object boundary k of P: the first object o with bitmap_word(o) + o >= k/P of
+// (bitmap words + objects) -- balances the merge (words) and the finalize
+// (tiles + one warp per object).
+static uint64_t owned_cut(const drgpum_ctx* c, uint32_t k, uint32_t P) {
+  if (k == 0) return 0;
+  if (k >= P) return c->n_obj;
+  const uint64_t total = c->bitmap_words + c->n_obj;
+  const uint64_t target = (uint64_t)((unsigned __int128)total * k / P);
+  uint64_t lo = 0, hi = c->n_obj;   // f(n_obj) = total >= target
+  while (lo < hi) {
+    const uint64_t m = (lo + hi) / 2;
+    if (c->layout[m].bitmap_word + m >= target) hi = m; else lo = m + 1;
+  }
+  return lo;
+}
+
 DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx* ctx, void* const* h_peer_ws, uint32_t n_peers,
                                             uint32_t rank, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers before workspace_bind");
-  if (!h_peer_ws || n_peers == 0 || n_peers > kMaxPeers || rank >= n_peers)
-    return fail(ctx, DRGPUM_EINVAL, "merge_peers: need 1 <= n_peers <= %u and rank < n_peers", kMaxPeers);
-  if (h_peer_ws[rank] != ctx->ws)
-    return fail(ctx, DRGPUM_EINVAL, "merge_peers: h_peer_ws[rank] is not this context's workspace");
   MergePeersParams q{};
-  for (uint32_t r = 0; r < n_peers; ++r) {
-    if (!h_peer_ws[r] || reinterpret_cast<uintptr_t>(h_peer_ws[r]) % kAlign)
-      return fail(ctx, DRGPUM_EINVAL, "merge_peers: peer %u workspace NULL or not 256-B aligned", r);
-    q.peer[r] = static_cast<uint8_t*>(h_peer_ws[r]);
-  }
+  if (drgpum_status e = check_peers(ctx, "merge_peers", h_peer_ws, n_peers, rank, q.peer)) return e;
   q.n_peers = n_peers;
   q.rank = rank;
   q.or_off = ctx->L.orw;
@@ -797,7 +824,62 @@ DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx* ctx, void* const* h_peer
   q.o_hi = std::min<uint64_t>(q.o_lo + so, ctx->n_obj);
   ctx->launches += launch_merge_peers(q, ctx->num_sms, as_stream(stream));
   ctx->final_valid = false;
+  ctx->owned = ctx->gathered = false;
   CK(cudaGetLastError());
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_merge_peers_owned(drgpum_ctx* ctx, void* const* h_peer_ws,
+                                                  uint32_t n_peers, uint32_t rank, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers_owned before workspace_bind");
+  MergeOwnedParams q{};
+  if (drgpum_status e = check_peers(ctx, "merge_peers_owned", h_peer_ws, n_peers, rank, q.peer)) return e;
+  q.n_peers = n_peers;
+  q.rank = rank;
+  q.or_off = ctx->L.orw;
+  q.first_off = ctx->L.first;
+  q.last_off = ctx->L.last;
+  q.ctr_off = ctx->L.ctr;
+  const uint64_t lo = owned_cut(ctx, rank, n_peers), hi = owned_cut(ctx, rank + 1, n_peers);
+  auto bw = [&](uint64_t o) { return o < ctx->n_obj ? ctx->layout[o].bitmap_word : ctx->bitmap_words; };
+  auto hw = [&](uint64_t o) { return ctx->bitmap_words + (o < ctx->n_obj ? ctx->layout[o].hit_word : ctx->hit_words); };
+  q.b_lo = bw(lo); q.b_hi = bw(hi);   // multiples of 4 (every bitmap is padded to 4 words)
+  q.h_lo = hw(lo); q.h_hi = hw(hi);
+  q.o_lo = lo; q.o_hi = hi;
+  ctx->launches += launch_merge_owned(q, ctx->num_sms, as_stream(stream));
+  CK(cudaGetLastError());
+  ctx->final_valid = false;
+  ctx->owned = true;
+  ctx->gathered = false;
+  ctx->own_lo = lo; ctx->own_hi = hi; ctx->own_P = n_peers; ctx->own_rank = rank;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_gather_peers(drgpum_ctx* ctx, void* const* h_peer_ws,
+                                             uint32_t n_peers, uint32_t rank, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "gather_peers before workspace_bind");
+  GatherParams q{};
+  if (drgpum_status e = check_peers(ctx, "gather_peers", h_peer_ws, n_peers, rank, q.peer)) return e;
+  if (!ctx->owned || !ctx->final_valid)
+    return fail(ctx, DRGPUM_ESTATE, "gather_peers needs merge_peers_owned then finalize");
+  if (n_peers != ctx->own_P || rank != ctx->own_rank)
+    return fail(ctx, DRGPUM_EINVAL, "gather_peers: n_peers / rank differ from merge_peers_owned");
+  static_assert(sizeof(drgpum_object_stats_t) % 4 == 0 && sizeof(drgpum_pattern_report_t) % 4 == 0,
+                "gather copies u32 words");
+  q.n_peers = n_peers;
+  q.rank = rank;
+  q.stats_off = ctx->L.stats;
+  q.s_lo = ctx->own_lo * sizeof(drgpum_object_stats_t);
+  q.s_hi = ctx->own_hi * sizeof(drgpum_object_stats_t);
+  q.reports_off = ctx->L.reports;
+  q.r_lo = ctx->own_lo * sizeof(drgpum_pattern_report_t);
+  q.r_hi = ctx->own_hi * sizeof(drgpum_pattern_report_t);
+  q.ctr_off = ctx->L.ctr;
+  ctx->launches += launch_gather_peers(q, ctx->num_sms, as_stream(stream));
+  CK(cudaGetLastError());
+  ctx->gathered = true;
   return DRGPUM_OK;
 }
 
@@ -829,7 +911,14 @@ DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_threshold
   p.stats = ctx->ws + ctx->L.stats;
   p.reports = ctx->ws + ctx->L.reports;
   p.ctr = at<unsigned long long>(ctx, ctx->L.ctr);
+  p.o_lo = ctx->owned ? ctx->own_lo : 0;
+  p.o_hi = ctx->owned ? ctx->own_hi : ctx->n_obj;
+  p.t_lo = ctx->tile_off[p.o_lo];
+  p.t_hi = ctx->tile_off[p.o_hi];
+  p.g_lo = ctx->group_off[p.o_lo];
+  p.g_hi = ctx->group_off[p.o_hi];
   ctx->launches += launch_finalize(p, ctx->num_sms, st);
+  ctx->gathered = false;
   CK(cudaGetLastError());
   ctx->final_valid = true;
   ctx->final_th = t;
@@ -846,6 +935,8 @@ DRGPUM_API drgpum_status drgpum_object_stats(drgpum_ctx* ctx, drgpum_object_stat
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "object_stats before workspace_bind");
   cudaStream_t st = as_stream(stream);
+  if (ctx->owned && !(ctx->final_valid && ctx->gathered))
+    return fail(ctx, DRGPUM_ESTATE, "object_stats after merge_peers_owned needs finalize + gather_peers");
   if (!ctx->final_valid) {
     drgpum_status s = drgpum_finalize(ctx, &ctx->final_th, stream);
     if (s != DRGPUM_OK) return s;
@@ -872,6 +963,8 @@ DRGPUM_API drgpum_status drgpum_patterns(drgpum_ctx* ctx, const drgpum_threshold
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "patterns before workspace_bind");
   drgpum_thresholds_t t = th ? *th : drgpum_thresholds_t{2, 80, 80};
   cudaStream_t st = as_stream(stream);
+  if (ctx->owned && !(ctx->final_valid && ctx->gathered && same_th(t, ctx->final_th)))
+    return fail(ctx, DRGPUM_ESTATE, "patterns after merge_peers_owned needs finalize (same thresholds) + gather_peers");
   if (!ctx->final_valid || !same_th(t, ctx->final_th)) {
     drgpum_status s = drgpum_finalize(ctx, &t, stream);
     if (s != DRGPUM_OK) return s;
@@ -890,7 +983,7 @@ DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx* ctx, uint64_t* h_
   unsigned long long c[C_SLOTS];
   CK(cudaMemcpyAsync(c, ctx->ws + ctx->L.ctr, sizeof c, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
-  *h_errors = c[C_CONSISTENCY];
+  *h_errors = ctx->owned && ctx->gathered ? c[C_CONSISTENCY_ALL] : c[C_CONSISTENCY];
   return DRGPUM_OK;
 }
 

@@ -61,6 +61,7 @@ enum : int { C_RECORDS = 0, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID,
              C_TILES_AFFINE_UNION, C_TILES_AFFINE_WORDS, C_TILES_FAST, C_TILES_SLOW,
              C_WORK,   // attribution work cursor (chunk tickets handed out)
              C_RQ_COUNT_ALT,   // range-queue count of odd-numbered attribute calls
+             C_CONSISTENCY_ALL,   // sum of every rank's C_CONSISTENCY after gather_peers
              C_SLOTS = 16 };
 
 struct AttrParams {
@@ -164,6 +165,9 @@ struct FinalParams {
   void* stats;               // drgpum_object_stats[n_obj]
   void* reports;             // drgpum_pattern_report[n_obj]
   unsigned long long* ctr;
+  // the objects this call finalizes ([0, n_obj) unless an owned merge
+  // narrowed it) and their tiles / groups
+  uint64_t o_lo, o_hi, t_lo, t_hi, g_lo, g_hi;
 };
 
 // Peer-memory merge (B7'): workspace base pointers of every rank, indexed by rank.
@@ -176,6 +180,26 @@ struct MergePeersParams {
   uint64_t o_lo, o_hi;                             // owned object slice
 };
 
+// Owned merge (B7''): rank r combines only the shadow of ITS objects
+// [o_lo, o_hi) -- bitmap words [b_lo, b_hi) (16-B vectors [b_lo/4, b_hi/4)),
+// hit-row words [h_lo, h_hi) of the OR section, first/last -- from every
+// peer into its own workspace; rank 0 sums the counters into every peer.
+struct MergeOwnedParams {
+  uint8_t* peer[kMaxPeers];
+  uint32_t n_peers, rank;
+  uint64_t or_off, first_off, last_off, ctr_off;
+  uint64_t b_lo, b_hi, h_lo, h_hi, o_lo, o_hi;
+};
+
+// Gather (B7''): rank r stores bytes [lo, hi) of the stats and of the
+// reports sections (its objects) into every peer, and adds its consistency
+// count into every peer's C_CONSISTENCY_ALL.
+struct GatherParams {
+  uint8_t* peer[kMaxPeers];
+  uint32_t n_peers, rank;
+  uint64_t stats_off, s_lo, s_hi, reports_off, r_lo, r_hi, ctr_off;
+};
+
 // Launchers (return the number of kernels enqueued).
 int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);   // p.rq_slot alternates per call
 int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
@@ -185,6 +209,8 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
 int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_bytes, int num_sms, cudaStream_t s);
 int launch_merge_peers(const MergePeersParams& q, int num_sms, cudaStream_t s);
+int launch_merge_owned(const MergeOwnedParams& q, int num_sms, cudaStream_t s);
+int launch_gather_peers(const GatherParams& q, int num_sms, cudaStream_t s);
 int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src,
                     uint64_t src_stride, uint64_t n_words, int num_sms, cudaStream_t s);
 

@@ -115,3 +115,17 @@ class SymmetricMerge:
         h.barrier(channel=0)            # every rank's attribution is done
         session.merge_peers(self.peer_ptrs(), h.rank, stream)
         h.barrier(channel=0)            # every slice is merged everywhere
+
+    def merge_owned(self, session, stream=None):
+        """Owned merge: afterwards this rank holds the merged shadow of its
+        objects only; follow with session.finalize() and gather()."""
+        h = self.handle
+        h.barrier(channel=0)            # every rank's attribution is done
+        session.merge_peers_owned(self.peer_ptrs(), h.rank, stream)
+        h.barrier(channel=0)            # every rank's objects are merged
+
+    def gather(self, session, stream=None):
+        h = self.handle
+        h.barrier(channel=0)            # every rank's finalize is done
+        session.gather_peers(self.peer_ptrs(), h.rank, stream)
+        h.barrier(channel=0)            # every rank holds all stats / reports

@@ -248,6 +248,19 @@ class Session:
         check(self._h, self.L.drgpum_merge_peers(self._h, arr, len(peer_ptrs), rank,
                                                  _stream_handle(stream)))
 
+    def merge_peers_owned(self, peer_ptrs, rank, stream=None):
+        """drgpum_merge_peers_owned: merge this rank's objects only (then
+        finalize + gather_peers)."""
+        arr = (ctypes.c_void_p * len(peer_ptrs))(*[ctypes.c_void_p(int(x)) for x in peer_ptrs])
+        check(self._h, self.L.drgpum_merge_peers_owned(self._h, arr, len(peer_ptrs), rank,
+                                                       _stream_handle(stream)))
+
+    def gather_peers(self, peer_ptrs, rank, stream=None):
+        """drgpum_gather_peers: share this rank's finalized stats / reports."""
+        arr = (ctypes.c_void_p * len(peer_ptrs))(*[ctypes.c_void_p(int(x)) for x in peer_ptrs])
+        check(self._h, self.L.drgpum_gather_peers(self._h, arr, len(peer_ptrs), rank,
+                                                  _stream_handle(stream)))
+
     def bitmap(self, o):
         """Object o's bitmap as a bool numpy array (copies from the device)."""
         lay = self.layout()[o]

@@ -123,5 +123,117 @@ def test_symmetric_memory_single_rank():
         torch.cuda.synchronize()
         assert sm.peer_ptrs() == [s.workspace.data_ptr()]
         _check_against_oracle(s, p.objects, p.kinds, recs)
+        # the owned path through the same plumbing (bench.py's N>1 default)
+        s.reset()
+        s.attribute(torch.from_numpy(recs.view(np.uint8)).cuda())
+        sm.merge_owned(s)
+        s.finalize()
+        sm.gather(s)
+        torch.cuda.synchronize()
+        _check_against_oracle(s, p.objects, p.kinds, recs)
     finally:
         dist.destroy_process_group()
+
+
+# ---------------------------------------------------------------- owned merge
+def _virtual_peers_owned(objs, kinds, recs, P, th=None):
+    """drgpum_merge_peers_owned + finalize + drgpum_gather_peers over P virtual
+    peers on cuda:0 (each phase for every rank, then a device sync = the
+    barrier between phases on P GPUs)."""
+    from paper_conf_asplos_linzs23_b200 import Session
+    from paper_conf_asplos_linzs23_b200.parallel import shard_range
+    sessions = [Session(objs, kinds) for _ in range(P)]
+    d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
+    for r, s in enumerate(sessions):
+        lo, hi = shard_range(len(recs), r, P)
+        s.attribute(d[16 * lo: 16 * hi])
+    torch.cuda.synchronize()
+    ptrs = [s.workspace.data_ptr() for s in sessions]
+    for r, s in enumerate(sessions):
+        s.merge_peers_owned(ptrs, r)
+    torch.cuda.synchronize()
+    for s in sessions:
+        s.finalize(th)
+    torch.cuda.synchronize()
+    for r, s in enumerate(sessions):
+        s.gather_peers(ptrs, r)
+    torch.cuda.synchronize()
+    return sessions, ptrs
+
+
+def _check_owned(sessions, objs, kinds, recs):
+    orc = Oracle(objs, kinds)
+    orc.attribute(recs)
+    ost, octr = orc.stats()
+    orep = orc.patterns()
+    for s in sessions:
+        st, ctr = s.object_stats()
+        rep = s.patterns()
+        assert s.consistency_errors() == 0
+        for k in octr.dtype.names:
+            assert int(ctr[k]) == int(octr[k]), k
+        for k in ost.dtype.names:
+            if k != "_pad":
+                assert np.array_equal(st[k], ost[k]), k
+        for k in orep.dtype.names:
+            assert np.array_equal(rep[k], orep[k]), k
+    # every object's bitmap is merged on (at least) its owner
+    exp = expected_or_words(sessions[0], orc, objs, kinds)
+    lay = sessions[0].layout()
+    have = [s.or_words().cpu().numpy().view(np.uint32) for s in sessions]
+    for o in range(len(objs)):
+        w0 = int(lay["bitmap_word"][o])
+        nw = (int(objs["size"][o] // objs["elem_size"][o]) + 31) // 32
+        assert any(np.array_equal(h[w0:w0 + nw], exp[w0:w0 + nw]) for h in have), o
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+def test_virtual_peers_owned_c1(P):
+    p = build_config("C1")
+    recs = gen_all_records(p)
+    sessions, _ = _virtual_peers_owned(p.objects, p.kinds, recs, P)
+    _check_owned(sessions, p.objects, p.kinds, recs)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_virtual_peers_owned_tiny_reuse(seed):
+    p = build_tiny(4300 + seed)
+    recs = gen_all_records(p)
+    P = 2 + seed % 7            # up to 8 ranks: some own no object at all
+    sessions, _ = _virtual_peers_owned(p.objects, p.kinds, recs, P)
+    _check_owned(sessions, p.objects, p.kinds, recs)
+
+
+def test_owned_state_rules():
+    """object_stats before the gather, patterns with other thresholds, and a
+    gather without an owned merge are refused (ESTATE), not answered from a
+    partially merged shadow."""
+    from paper_conf_asplos_linzs23_b200 import Session
+    from paper_conf_asplos_linzs23_b200._lib import DrgpumError
+    p = build_tiny(4400)
+    recs = gen_all_records(p)
+    a, b = Session(p.objects, p.kinds), Session(p.objects, p.kinds)
+    ptrs = [a.workspace.data_ptr(), b.workspace.data_ptr()]
+    with pytest.raises(DrgpumError):
+        a.gather_peers(ptrs, 0)                     # no owned merge yet
+    d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
+    a.attribute(d[: 16 * (len(recs) // 2)])
+    b.attribute(d[16 * (len(recs) // 2):])
+    torch.cuda.synchronize()
+    a.merge_peers_owned(ptrs, 0)
+    b.merge_peers_owned(ptrs, 1)
+    torch.cuda.synchronize()
+    with pytest.raises(DrgpumError):
+        a.object_stats()                            # not finalized + gathered
+    a.finalize(); b.finalize()
+    torch.cuda.synchronize()
+    with pytest.raises(DrgpumError):
+        a.gather_peers(ptrs[::-1], 1)               # rank differs from the merge's
+    a.gather_peers(ptrs, 0); b.gather_peers(ptrs, 1)
+    torch.cuda.synchronize()
+    a.object_stats()
+    with pytest.raises(DrgpumError):
+        a.patterns((3, 80, 80))
+    a.reset()                                       # a new trace: ordinary rules again
+    a.attribute(d)
+    a.patterns((3, 80, 80))
