@@ -104,3 +104,40 @@ def test_shard_range_partitions():
             assert rs[0][0] == 0 and rs[-1][1] == n
             assert all(a[1] == b[0] for a, b in zip(rs, rs[1:]))
             assert max(b - a for a, b in rs) - min(b - a for a, b in rs) <= 1
+
+
+def test_symmetric_merge_call_order():
+    """SymmetricMerge's host sequencing (no GPU): every library call of the
+    exchange sits between two device barriers of the symmetric-memory
+    handle, with this rank's index and every rank's workspace pointer."""
+    from paper_conf_asplos_linzs23_b200.parallel import SymmetricMerge
+    log = []
+
+    class Handle:
+        rank = 1
+        buffer_ptrs = [4096, 8192, 12288]
+
+        def barrier(self, channel=0):
+            log.append(("barrier", channel))
+
+    class Sess:
+        def merge_peers(self, ptrs, rank, stream=None):
+            log.append(("merge_peers", tuple(ptrs), rank))
+
+        def merge_peers_owned(self, ptrs, rank, stream=None):
+            log.append(("merge_peers_owned", tuple(ptrs), rank))
+
+        def gather_peers(self, ptrs, rank, stream=None):
+            log.append(("gather_peers", tuple(ptrs), rank))
+
+    sm = SymmetricMerge.__new__(SymmetricMerge)
+    sm.handle = Handle()
+    s = Sess()
+    ptrs = (4096, 8192, 12288)
+    sm.merge(s)
+    assert log == [("barrier", 0), ("merge_peers", ptrs, 1), ("barrier", 0)]
+    log.clear()
+    sm.merge_owned(s)
+    sm.gather(s)
+    assert log == [("barrier", 0), ("merge_peers_owned", ptrs, 1), ("barrier", 0),
+                   ("barrier", 0), ("gather_peers", ptrs, 1), ("barrier", 0)]
