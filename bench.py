@@ -419,8 +419,21 @@ def main():
         cal = {"read_gbs": 16.0 * n_local / (rd_ms / 1e3) / 1e9, "ms": rd_ms,
                "how": "torch.sum over the resident record buffer viewed as int64 (read-only stream)"}
 
-    # touched shadow words of the last step (algorithmic write-back of A3/A4)
-    touched = int(torch.count_nonzero(s.or_words()).item())
+    # touched shadow words (algorithmic write-back of A3/A4) of THIS rank's
+    # attribution: at N>1 the merged shadow is not what the rank's kernel
+    # wrote, so the shard is attributed once more alone, counted, and the
+    # merged step re-run (collectively) for the stats below
+    if world > 1:
+        s.reset()
+        for c0, c1 in chunks:
+            if chunked:
+                dp.gen(lo + c0, lo + c1, out=d_recs)
+            s.attribute(d_recs[:16 * (c1 - c0)])
+        touched = int(torch.count_nonzero(s.or_words()).item())
+        barrier()
+        one_step(d_recs)
+    else:
+        touched = int(torch.count_nonzero(s.or_words()).item())
     stats, ctr = s.object_stats()
     paths = s.path_stats()
 
