@@ -385,11 +385,32 @@ __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(cons
 
 // B4b: one warp per group (<= 32 consecutive tiles of one object): ordered
 // shuffle tree over the tile monoids.
+template <bool kBatch>
 __global__ void __launch_bounds__(256) group_reduce_kernel(const Group* __restrict__ groups,
     uint64_t n_groups, const BitMonoid* __restrict__ tile_part, BitMonoid* __restrict__ out) {
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  if (kBatch) {
+  // 32 consecutive groups per warp: single-tile groups (small objects) are
+  // copied lane-parallel, the others reduced one by one by the whole warp
+  for (uint64_t g0 = gwarp * 32; g0 < n_groups; g0 += nwarps * 32) {
+    const uint64_t g = g0 + lane;
+    const Group gr = g < n_groups ? groups[g] : Group{0, 0};
+    if (gr.n_tiles == 1) out[g] = tile_part[gr.tile_lo];
+    uint32_t multi = __ballot_sync(FULL_MASK, gr.n_tiles > 1);
+    while (multi) {
+      const int j = __ffs(multi) - 1;
+      multi &= multi - 1;
+      const uint32_t tlo = __shfl_sync(FULL_MASK, gr.tile_lo, j), nt = __shfl_sync(FULL_MASK, gr.n_tiles, j);
+      BitMonoid m = uint32_t(lane) < nt ? tile_part[tlo + lane] : bm_identity();
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) m = bm_cat(m, bm_shfl_down(m, d));
+      if (lane == 0) out[g0 + j] = m;
+    }
+  }
+  return;
+  }
   for (uint64_t g = gwarp; g < n_groups; g += nwarps) {
     const Group gr = groups[g];
     BitMonoid m = uint32_t(lane) < gr.n_tiles ? tile_part[gr.tile_lo + lane] : bm_identity();
@@ -559,9 +580,16 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   const uint64_t cap1 = uint64_t(num_sms) * DRGPUM_TR_GRID_PER_SM;
   const unsigned g1 = (unsigned)(tb < cap1 ? tb : cap1);
   tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles + p.t_lo, nt, p.tile_part + p.t_lo, p.ctr);
-  const uint64_t gb = (ng + 7) / 8;
+  // mostly single-tile groups (many small objects, C5): 32 groups per warp,
+  // single-tile ones copied lane-parallel (C5 finalize 2.77 -> 2.37 ms);
+  // otherwise one warp per group (C2: the batched form 83 vs 58 us)
+  const bool batch = nt < 2 * ng;
+  const uint64_t gb = batch ? (ng + 255) / 256 : (ng + 7) / 8;
   const unsigned g3 = (unsigned)(gb < uint64_t(num_sms) * 16 ? gb : uint64_t(num_sms) * 16);
-  group_reduce_kernel<<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
+  if (batch)
+    group_reduce_kernel<true><<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
+  else
+    group_reduce_kernel<false><<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
   constexpr unsigned wpb = kFinThreads / 32;   // one warp per object
   const uint64_t ob = (no + wpb - 1) / wpb;
   unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
