@@ -1,22 +1,37 @@
 #!/usr/bin/env python
 """Benchmark: DrGPUM per-access attribution on B200 (BASELINE.json metric).
 
-One *step* is one pass of the whole hot path over the workload's records,
-already resident in HBM: reset the shadow (bitmaps / hit rows / first / last /
-counters), attribute every record (A1-A5), [merge across ranks], and the
-per-object reductions + pattern classification (A6-A7), all on the device.
+One *step* is one pass of the whole hot path over the workload's records:
+reset the shadow (bitmaps / hit rows / first / last / counters), attribute
+every record (A1-A5), [merge across ranks], and the per-object reductions +
+pattern classification (A6-A7), all on the device.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5]
   python bench.py --impl reference ...   # the CPU oracle as the reference arm
+  python bench.py --gpus 2 --dry-run     # rank plumbing only (gloo, no GPU)
 
-N>1 runs under torchrun (one rank per GPU, NCCL): rank r attributes records
-[r*N/P, (r+1)*N/P) of the same trace, then the one exchange step merges the
-shadows (paper_conf_asplos_linzs23_b200/parallel.py) -- strong scaling.
-Rank 0 prints ONE JSON line.
+Default workload: C5, BASELINE.json's scaling sweep (1.6e10 records over 10^6
+objects), the largest config; it does not fit one GPU's HBM (256 GB of
+records), so at N=1 it is streamed through HBM in 2^30-record chunks generated
+on the device (generation outside the timed events), and at N>=4 every rank's
+shard is resident.  Extra key ``other_configs``: C4 (the largest config that
+is resident on one GPU) and C2, measured in the same run.
+
+--gpus N > 1 without torchrun in the environment re-launches this script
+under ``torch.distributed.run`` with N ranks (one per GPU, NCCL): rank r
+attributes records [r*N/P, (r+1)*N/P) of the same trace, then the one
+exchange step merges the shadows (paper_conf_asplos_linzs23_b200/parallel.py)
+-- strong scaling.  Rank 0 prints ONE JSON line.
+
+Every run checks its results against the oracle's golden digests
+(tests/golden/digests/<config>.json, written by tools/make_golden_digests.py
+from oracle/ alone) when they exist for the measured record count: key
+``parity``.
 """
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -37,15 +52,14 @@ WORKLOADS = {
           "in a 12 GiB best-fit caching pool (address reuse), short-lived activations",
     "C4": "C4 LLM-inference-shaped trace (BASELINE configs[3]): 4e9 records over 100K objects "
           "(120 GiB live footprint, reused 4 GiB activation arena), Zipf-skewed hot weights / KV blocks",
-    "C5": "C5 scaling sweep (BASELINE configs[4]): 1.6e10 records over 1M objects, streamed through HBM "
-          "in 2^30-record chunks generated on the device",
+    "C5": "C5 scaling sweep (BASELINE configs[4]): 1.6e10 records over 1M objects, record-range sharded; "
+          "streamed through HBM in 2^30-record chunks generated on the device when a shard exceeds 96 GiB",
 }
-# configs whose records are generated on the device (tracegen/gen.cu) rather
-# than on the host; traces above RESIDENT_BYTES are streamed in GEN_CHUNK chunks
-DEVICE_GEN = ("C3", "C4", "C5")
+# traces above RESIDENT_BYTES per rank are streamed in GEN_CHUNK chunks
 GEN_CHUNK = 1 << 30
 RESIDENT_BYTES = 96 << 30
 FALLBACK_HBM_GBS = 6650.0
+GOLDEN_DIR = os.path.join(ROOT, "tests", "golden", "digests")
 
 
 def args_():
@@ -54,7 +68,7 @@ def args_():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C2", choices=sorted(WORKLOADS))
+    ap.add_argument("--config", default="C5", choices=sorted(WORKLOADS))
     ap.add_argument("--records", type=int, default=None, help="override the record count")
     ap.add_argument("--e2e-steps", type=int, default=None)
     ap.add_argument("--merge", default="owned", choices=["owned", "peers", "nccl"],
@@ -67,13 +81,17 @@ def args_():
     ap.add_argument("--no-next", action="store_true", help="skip the SURVEY §8(f) NEXT-row timings")
     ap.add_argument("--no-graph", action="store_true",
                     help="time eager launches instead of CUDA-graph replays of the step")
-    ap.add_argument("--cpu-sample", type=int, default=None,
-                    help="records in the oracle's timed sample (default: whole workload up to 1e8; "
-                         "2e7 for the device-generated configs)")
-    ap.add_argument("--e2e-sample", type=int, default=1 << 26,
-                    help="records of the host-buffer (e2e) leg for the device-generated configs")
-    ap.add_argument("--ref-sample", type=int, default=8_000_000,
-                    help="records per reference-arm step")
+    ap.add_argument("--no-parity", action="store_true", help="skip the golden-digest check")
+    ap.add_argument("--extra-configs", default="C4,C2",
+                    help="comma list of configs measured after the main one at N=1 (key other_configs); '' = none")
+    ap.add_argument("--cpu-sample", type=int, default=30_000_000,
+                    help="target records of the oracle's timed sample (an object_sample of the workload)")
+    ap.add_argument("--e2e-sample", type=int, default=1 << 28,
+                    help="records per step of the host-buffer (e2e) leg")
+    ap.add_argument("--ref-sample", type=int, default=4_000_000,
+                    help="target records per reference-arm step (an object_sample of the workload)")
+    ap.add_argument("--dry-run", action="store_true",
+                    help="launch the ranks and check the process-group plumbing only (gloo; no GPU)")
     return ap.parse_args()
 
 
@@ -137,6 +155,63 @@ def cpu_model():
     return "unknown"
 
 
+def free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def relaunch(a):
+    """--gpus N > 1 outside torchrun: run this script under
+    torch.distributed.run with N ranks on this node and pass its exit code on."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()),
+           os.path.abspath(__file__)] + sys.argv[1:]
+    print(f"bench.py: launching {a.gpus} ranks: {' '.join(cmd)}", file=sys.stderr, flush=True)
+    return subprocess.call(cmd)
+
+
+def world_env():
+    return (int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")),
+            int(os.environ.get("LOCAL_RANK", "0")))
+
+
+def dry_run(a):
+    """The rank plumbing of an N-GPU run without a GPU: every rank joins a
+    gloo process group, the ranks are counted with an all_reduce, rank 0
+    prints one line."""
+    import torch
+    import torch.distributed as dist
+    world, rank, _ = world_env()
+    if world != a.gpus:
+        raise SystemExit(f"bench.py: WORLD_SIZE={world} but --gpus {a.gpus}")
+    if world > 1:
+        dist.init_process_group("gloo")
+    t = torch.tensor([1, rank], dtype=torch.int64)
+    if world > 1:
+        dist.all_reduce(t)
+    if rank == 0:
+        print(json.dumps({"dry_run": True, "n_gpus": world, "ranks_reporting": int(t[0]),
+                          "rank_sum": int(t[1]), "backend": "gloo" if world > 1 else "none",
+                          "config": {"workload": WORKLOADS[a.config]}}), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# ---------------------------------------------------------------- CPU oracle
+def oracle_sample(prog, target):
+    """A bounded sample of the workload for the CPU oracle: 1/k of the objects
+    (index % k == 0) with every record that targets them, over the full
+    timeline (tracegen.object_sample), k chosen for ~target records."""
+    from tracegen import object_sample
+    k = max(1, int(round(prog.n_records / max(1, target))))
+    sub = object_sample(prog, k, 0) if k > 1 else prog
+    desc = (f"1/{k} of the {prog.name} objects (index % {k} == 0, {sub.n_obj} of {prog.n_obj}) with every "
+            f"record that targets them: {sub.n_records} of {prog.n_records} records, the full {prog.n_api}-API "
+            f"timeline; one pass: load + attribute + stats + patterns (O1, single thread)")
+    return sub, desc
+
+
 def time_oracle(objs, kinds, recs):
     """The oracle as it stands (single-threaded C++), one full pass."""
     from oracle import Oracle
@@ -149,30 +224,350 @@ def time_oracle(objs, kinds, recs):
 
 
 def reference_arm(a):
-    """--impl reference: the CPU oracle, timed on the host cores, on our config."""
-    rank = int(os.environ.get("RANK", "0"))
+    """--impl reference: the CPU oracle, timed on the host cores, on our
+    config (a bounded object sample of it per step)."""
+    world, rank, _ = world_env()
     if rank != 0:
         return
     from tracegen import build_config, gen_records
     prog = build_config(a.config, **({"n_records": a.records} if a.records else {}))
-    m = min(a.ref_sample, prog.n_records)
-    recs = gen_records(prog, 0, m)
+    sub, desc = oracle_sample(prog, a.ref_sample)
+    recs = gen_records(sub, 0, sub.n_records)
     for _ in range(a.warmup):
-        time_oracle(prog.objects, prog.kinds, recs)
-    ts = [time_oracle(prog.objects, prog.kinds, recs) for _ in range(a.steps)]
+        time_oracle(sub.objects, sub.kinds, recs)
+    ts = [time_oracle(sub.objects, sub.kinds, recs) for _ in range(a.steps)]
     t = sum(ts) / len(ts)
-    v = m / t
-    sample = (f"first {m} records of the {prog.n_records}-record {a.config} trace per step "
-              f"(prefix-timed; oracle = O1 std::map replay, single thread)")
+    v = sub.n_records / t
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": v, "unit": "records/s",
         "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup, "ms_per_step": t * 1e3,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
-        "data": "synthetic", "config": {"workload": WORKLOADS[a.config], "records": m},
+        "data": f"synthetic (tracegen {prog.name}, seed {prog.seed:#x})",
+        "config": {"workload": WORKLOADS[a.config], "records": prog.n_records, "objects": prog.n_obj,
+                   "sample_records": sub.n_records, "sample_objects": sub.n_obj},
+        "same_config": True,
         "cpu_baseline": {"value": v, "unit": "records/s", "cores": 1, "kind": "oracle",
-                         "sample": sample, "cpu": cpu_model()},
+                         "sample": desc, "cpu": cpu_model()},
         "e2e": {"value": v, "unit": "records/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
+
+
+# ---------------------------------------------------------------- GPU workload
+class Workload:
+    """One config's records (resident, or regenerated chunk by chunk on the
+    device), its Session, and the step that bench.py times.  The GPU parity
+    tests (tests/test_gpu_fullsize.py) run exactly this step."""
+
+    def __init__(self, cfg, records=None, rank=0, world=1, merge="owned", resident_bytes=RESIDENT_BYTES):
+        import torch
+        from paper_conf_asplos_linzs23_b200 import Session
+        from tracegen import build_config
+        from tracegen.device import DeviceProgram
+        from paper_conf_asplos_linzs23_b200.parallel import shard_range
+        self.torch = torch
+        self.cfg, self.rank, self.world = cfg, rank, world
+        self.prog = build_config(cfg, **({"n_records": records} if records else {}))
+        self.N = self.prog.n_records
+        self.lo, self.hi = shard_range(self.N, rank, world)
+        self.n_local = self.hi - self.lo
+        self.chunked = 16 * self.n_local > resident_bytes
+        self.dp = DeviceProgram(self.prog)
+        gen = [(c, min(c + GEN_CHUNK, self.n_local)) for c in range(0, self.n_local, GEN_CHUNK)]
+        self.d_recs = torch.empty(16 * max(1, GEN_CHUNK if self.chunked else self.n_local),
+                                  dtype=torch.uint8, device="cuda")
+        if self.chunked:
+            self.chunks = gen
+        else:
+            for c0, c1 in gen:   # device generation, never timed
+                self.dp.gen(self.lo + c0, self.lo + c1, out=self.d_recs[16 * c0:16 * c1])
+            self.chunks = [(0, self.n_local)]
+        torch.cuda.synchronize()
+        self.sm, self.merge_note = None, "none (1 rank)"
+        if world > 1 and merge in ("peers", "owned"):
+            from paper_conf_asplos_linzs23_b200.parallel import SymmetricMerge
+            try:
+                self.sm = SymmetricMerge()
+                self.s = Session(self.prog.objects, self.prog.kinds, workspace_alloc=self.sm.alloc)
+                self.merge_note = ("drgpum_merge_peers_owned + finalize of the owned objects + "
+                                   "drgpum_gather_peers over torch symmetric memory (NVLink P2P)"
+                                   if merge == "owned" else
+                                   "drgpum_merge_peers over torch symmetric memory (one kernel per rank, NVLink P2P)")
+            except Exception as e:   # symmetric memory unavailable: the NCCL exchange instead, said so
+                self.sm = None
+                self.merge_note = f"NCCL all_to_all + merge_or + all_gather (symmetric memory unavailable: {e})"
+        if self.sm is None:
+            self.s = Session(self.prog.objects, self.prog.kinds)
+            if world > 1 and merge == "nccl":
+                self.merge_note = "NCCL all_to_all + merge_or + all_gather"
+        self.owned = self.sm is not None and merge == "owned"
+        self.stream = torch.cuda.current_stream()
+        self.graph = None
+
+    # -- the step ------------------------------------------------------------
+    def do_merge(self):
+        if self.world > 1:
+            from paper_conf_asplos_linzs23_b200.parallel import merge_session
+            if self.owned:
+                self.sm.merge_owned(self.s)
+            elif self.sm is not None:
+                self.sm.merge(self.s)
+            else:
+                merge_session(self.s)
+
+    def do_finalize(self):
+        self.s.finalize()
+        if self.owned:
+            self.sm.gather(self.s)
+
+    def step(self, ev=None):
+        """ev: per-phase event pairs [reset, attribute (per chunk), merge,
+        finalize]; generation of a chunk lies outside its attribute pair."""
+        st = self.stream
+        if ev: ev["reset"][0].record(st)
+        self.s.reset()
+        if ev: ev["reset"][1].record(st)
+        for k, (c0, c1) in enumerate(self.chunks):
+            if self.chunked:
+                self.dp.gen(self.lo + c0, self.lo + c1, out=self.d_recs)
+            if ev: ev["attr"][k][0].record(st)
+            self.s.attribute(self.d_recs[:16 * (c1 - c0)])
+            if ev: ev["attr"][k][1].record(st)
+        if ev: ev["merge"][0].record(st)
+        self.do_merge()
+        if ev: ev["merge"][1].record(st)
+        if ev: ev["fin"][0].record(st)
+        self.do_finalize()
+        if ev: ev["fin"][1].record(st)
+
+    def events(self):
+        E = lambda: (self.torch.cuda.Event(enable_timing=True), self.torch.cuda.Event(enable_timing=True))
+        return {"reset": E(), "attr": [E() for _ in self.chunks], "merge": E(), "fin": E()}
+
+    @staticmethod
+    def phases(ev):   # ms
+        el = lambda e: e[0].elapsed_time(e[1])
+        return [el(ev["reset"]), sum(el(e) for e in ev["attr"]), el(ev["merge"]), el(ev["fin"])]
+
+    def capture(self, warmup):
+        """The step as one CUDA graph (resident traces only): reset, attribute
+        + range expansion, [barrier, merge, barrier, finalize, barrier,
+        gather, barrier -- the symmetric-memory device barriers], finalize.
+        Every rank agrees on graph vs eager before any replay."""
+        torch = self.torch
+        ok, why = not self.chunked, "chunked trace (device generation between the chunks)"
+        if ok and self.world > 1 and self.sm is None:
+            ok, why = False, "NCCL exchange (host-side collectives)"
+        g = None
+        if ok:
+            try:
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g):
+                    self.step()
+                why = None
+            except Exception as e:   # noqa: BLE001 -- reported in the JSON line
+                g, ok, why = None, False, f"capture failed: {type(e).__name__}: {e}"
+        if self.world > 1:
+            import torch.distributed as dist
+            t = torch.tensor([1 if g is not None else 0], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MIN)
+            if int(t) == 0 and g is not None:
+                g, why = None, "another rank could not capture"
+        self.graph = g
+        self.graph_note = why
+        if g is not None:
+            for _ in range(warmup):
+                g.replay()
+            torch.cuda.synchronize()
+        return g is not None
+
+    def run(self):
+        if self.graph is not None:
+            self.graph.replay()
+        else:
+            self.step()
+
+    def close(self):
+        self.graph = None
+        self.s.close()
+        del self.s, self.d_recs, self.dp
+        self.torch.cuda.synchronize()
+        self.torch.cuda.empty_cache()
+
+
+def golden(cfg, n_records):
+    path = os.path.join(GOLDEN_DIR, f"{cfg}.json")
+    if not os.path.exists(path):
+        return None, path
+    with open(path) as f:
+        g = json.load(f)
+    return (g if int(g.get("records", -1)) == int(n_records) else None), path
+
+
+def parity_check(w, full):
+    """Compare this run's results with the oracle's golden digests (stats,
+    reports, counters; with full=True also every bitmap and accessing-API
+    set).  After an owned merge every rank holds all stats / reports."""
+    from tests.digest_util import compare, results_digest, session_digest
+    g, path = golden(w.cfg, w.N)
+    if g is None:
+        return {"checked": False, "why": f"no golden digest for {w.cfg} at {w.N} records ({os.path.relpath(path, ROOT)})"}
+    t0 = time.perf_counter()
+    if full:
+        d = session_digest(w.s)
+        keys = ("counters", "stats_sha", "reports_sha", "bitmap_sha", "access_sha")
+    else:
+        stats, ctr = w.s.object_stats()
+        d = results_digest(w.s.objects, ctr, stats, w.s.patterns())
+        keys = ("counters", "stats_sha", "reports_sha")
+    bad = compare(d, g, keys)
+    return {"checked": True, "golden": os.path.relpath(path, ROOT), "compared": list(keys),
+            "ok": not bad, "mismatches": bad[:20], "seconds": time.perf_counter() - t0}
+
+
+def measure(w, a, steps, warmup, clocks=False, use_graph=True):
+    """Warm up, phase breakdown (eager, events between phases), then the timed
+    region: K steps (graph replays when the trace is resident) bracketed by
+    barrier + synchronize, device time from events on the launching stream
+    (chunked traces: the sum of the steps' phase events, generation excluded)."""
+    import torch
+    import torch.distributed as dist
+    world = w.world
+    barrier = (lambda: dist.barrier()) if world > 1 else (lambda: None)
+    for _ in range(warmup):
+        w.step()
+    torch.cuda.synchronize()
+    l0 = w.s.launch_count()
+    w.step()
+    step_launches = w.s.launch_count() - l0
+    evs = [w.events() for _ in range(steps)]
+    torch.cuda.synchronize()
+    for k in range(steps):
+        w.step(evs[k])
+    torch.cuda.synchronize()
+    ph_mean = np.array([w.phases(e) for e in evs]).mean(axis=0)
+    graphed = use_graph and w.capture(warmup)
+    clk = ClockSampler(int(os.environ.get("LOCAL_RANK", "0"))) if clocks else None
+    if clk:
+        time.sleep(0.3)
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    launches0 = w.s.launch_count()
+    barrier()
+    torch.cuda.synchronize()
+    wall0 = time.perf_counter()
+    t_start.record(w.stream)
+    tev = [w.events() for _ in range(steps)] if w.chunked else None
+    for k in range(steps):
+        if graphed:
+            w.graph.replay()
+        else:
+            w.step(tev[k] if w.chunked else None)
+    t_end.record(w.stream)
+    torch.cuda.synchronize()
+    barrier()
+    wall = time.perf_counter() - wall0
+    clocks_v = clk.stop() if clk else None
+    # graph replays do not pass through the library's launch counter
+    launches = step_launches * steps if graphed else w.s.launch_count() - launches0
+    ms_total = t_start.elapsed_time(t_end)
+    if w.chunked:
+        ms_total = float(sum(sum(w.phases(e)) for e in tev))
+    if world > 1:
+        t = torch.tensor([ms_total] + ph_mean.tolist(), dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t[0])
+        ph_mean = t[1:].cpu().numpy()
+    return {"ms_step": ms_total / steps, "phases": ph_mean, "launches": launches, "graphed": graphed,
+            "wall": wall, "clocks": clocks_v, "step_launches": step_launches}
+
+
+def touched_words(w):
+    """Touched shadow words of THIS rank's attribution (the algorithmic
+    write-back of A3/A4).  At N>1 the merged shadow is not what the rank's
+    kernel wrote, so the shard is attributed once more alone, counted, and
+    the merged step re-run (collectively) for the results read afterwards."""
+    import torch
+    if w.world > 1:
+        import torch.distributed as dist
+        w.s.reset()
+        for c0, c1 in w.chunks:
+            if w.chunked:
+                w.dp.gen(w.lo + c0, w.lo + c1, out=w.d_recs)
+            w.s.attribute(w.d_recs[:16 * (c1 - c0)])
+        n = int(torch.count_nonzero(w.s.or_words()).item())
+        dist.barrier()
+        w.step()
+        torch.cuda.synchronize()
+        return n
+    return int(torch.count_nonzero(w.s.or_words()).item())
+
+
+def roofline(w, m, touched, hbm, hbm_src):
+    attr_ms = float(m["phases"][1])
+    alg_bytes = 16.0 * w.n_local + 4.0 * touched
+    achieved = alg_bytes / (attr_ms / 1e3) / 1e9
+    traffic = None
+    tfile = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tfile):
+        try:
+            t = json.load(open(tfile)).get(w.cfg)
+            traffic = None if t is None else int(t["bytes_per_launch"])
+        except Exception:
+            traffic = None
+    return {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+            "frac": achieved / hbm, "traffic": traffic,
+            "kernel": "drgpum_trace_attribute (attribute_kernel + range_expand_kernel)",
+            "algorithmic_bytes": alg_bytes, "records_per_rank": w.n_local,
+            "bytes_rule": "16 B per record + 4 B per touched shadow word",
+            "peak_source": hbm_src}
+
+
+def e2e_leg(w, a, steps):
+    """The same metric through the public API with HOST buffers: every step
+    copies its records from pinned host memory (drgpum_trace_attribute_host,
+    pipelined H2D staging) and reads the results back (object_stats +
+    patterns).  The sample is the first e2e_sample records of the rank's
+    shard (generated on the device, copied into the pinned buffer once)."""
+    import torch
+    import torch.distributed as dist
+    n = min(w.n_local, a.e2e_sample)
+    pinned = torch.empty(n * 16, dtype=torch.uint8, pin_memory=True)
+    tmp = torch.empty(16 * min(n, GEN_CHUNK), dtype=torch.uint8, device="cuda")
+    for c0 in range(0, n, GEN_CHUNK):
+        c1 = min(n, c0 + GEN_CHUNK)
+        w.dp.gen(w.lo + c0, w.lo + c1, out=tmp)
+        pinned[16 * c0:16 * c1].copy_(tmp[:16 * (c1 - c0)])
+    del tmp
+    torch.cuda.synchronize()
+
+    def one():
+        w.s.reset()
+        w.s.attribute(pinned)                 # drgpum_trace_attribute_host: H2D inside
+        w.do_merge()
+        if w.owned:
+            w.do_finalize()
+        w.s.object_stats()                    # D2H of the results
+        w.s.patterns()
+
+    for _ in range(2):
+        one()
+    torch.cuda.synchronize()
+    if w.world > 1:
+        dist.barrier()
+    w0 = time.perf_counter()
+    for _ in range(steps):
+        one()
+    torch.cuda.synchronize()
+    e2e_s = (time.perf_counter() - w0) / steps
+    if w.world > 1:
+        t = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = float(t[0])
+    return {"value": n * w.world / e2e_s, "unit": "records/s", "h2d_bytes_per_step": 16 * n,
+            "records_per_rank": n, "d2h_bytes_per_step": int(w.prog.n_obj * (56 + 32) + 40),
+            "ms_per_step": e2e_s * 1e3,
+            "path": "Session.attribute(pinned host tensor) -> drgpum_trace_attribute_host; "
+                    "object_stats + patterns (D2H)",
+            "sample": f"first {n} records of the rank's shard per step"}
 
 
 def next_rows(prog, d_recs, plain_attr_ms, reps=5):
@@ -212,6 +607,7 @@ def next_rows(prog, d_recs, plain_attr_ms, reps=5):
                      "pass_gbs_records_only": 16.0 * N / ((m - plain_attr_ms) / 1e3) / 1e9
                      if m > plain_attr_ms else None,
                      "query_ms": q_ms}
+        s.close()
         del s
         torch.cuda.empty_cache()
     s = Session(prog.objects, prog.kinds)
@@ -230,302 +626,118 @@ def next_rows(prog, d_recs, plain_attr_ms, reps=5):
     out["NEXT-4 multi-stream graph + Kahn"] = {
         "graph_and_levels_ms": g_ms, "patterns_topo_ms": (time.perf_counter() - w0) * 1e3,
         "streams": 8, "edges": int(src.shape[0]), "levels": int(T.max()) + 1 if T.size else 0}
+    s.close()
+    return out
+
+
+def other_config(cfg, a, hbm, hbm_src):
+    """One extra config at N=1: value, phases, roofline, parity (stats /
+    reports / counters), and for C2 the NEXT rows."""
+    import torch
+    w = Workload(cfg)
+    steps = max(3, min(a.steps, 10))
+    m = measure(w, a, steps, max(2, min(a.warmup, 3)), use_graph=not a.no_graph)
+    touched = touched_words(w)
+    out = {"workload": WORKLOADS[cfg], "records": w.N, "value": w.N / (m["ms_step"] / 1e3),
+           "unit": "records/s", "ms_per_step": m["ms_step"], "steps": steps,
+           "phases_ms": dict(zip(("reset", "attribute", "merge", "finalize"), map(float, m["phases"]))),
+           "step_exec": "cuda_graph_replay" if m["graphed"] else "eager",
+           "gpu_launches": m["launches"], "roofline": roofline(w, m, touched, hbm, hbm_src),
+           "resident": not w.chunked}
+    if not a.no_parity:
+        out["parity"] = parity_check(w, full=False)
+    if cfg == "C2" and not a.no_next:
+        out["next"] = next_rows(w.prog, w.d_recs[:16 * w.n_local], float(m["phases"][1]))
+    w.close()
+    torch.cuda.empty_cache()
     return out
 
 
 def main():
     a = args_()
+    world, rank, local = world_env()
+    if a.gpus > 1 and "WORLD_SIZE" not in os.environ and a.impl == "ours":
+        sys.exit(relaunch(a))
+    if a.dry_run:
+        return dry_run(a)
     if a.impl == "reference":
         return reference_arm(a)
+    if world != a.gpus:
+        raise SystemExit(f"bench.py: WORLD_SIZE={world} but --gpus {a.gpus}")
     import torch
     import torch.distributed as dist
-    from paper_conf_asplos_linzs23_b200 import Session
-    from paper_conf_asplos_linzs23_b200.parallel import shard_range, merge_session
-    from tracegen import build_config, gen_records
-
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
+    ranks = None
     if world > 1:
+        os.environ.setdefault("NCCL_DEBUG", "INFO")   # communicator lines on stderr (rank evidence)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    prog = build_config(a.config, **({"n_records": a.records} if a.records else {}))
-    N = prog.n_records
-    lo, hi = shard_range(N, rank, world)
-    n_local = hi - lo
-    devgen = a.config in DEVICE_GEN
-    chunked = devgen and 16 * n_local > RESIDENT_BYTES
-    recs = None
-    if not devgen:
-        recs = gen_records(prog, lo, hi)
-        d_recs = torch.from_numpy(recs.view(np.uint8)).cuda()
-        chunks = [(0, n_local)]
-    else:
-        # device generation (never timed): the whole shard resident, or one
-        # GEN_CHUNK buffer refilled per chunk inside every step
-        from tracegen.device import DeviceProgram
-        dp = DeviceProgram(prog)
-        gen_chunks = [(c, min(c + GEN_CHUNK, n_local)) for c in range(0, n_local, GEN_CHUNK)]
-        d_recs = torch.empty(16 * (GEN_CHUNK if chunked else n_local), dtype=torch.uint8, device="cuda")
-        if chunked:
-            chunks = gen_chunks
-        else:
-            for c0, c1 in gen_chunks:
-                dp.gen(lo + c0, lo + c1, out=d_recs[16 * c0:16 * c1])
-            chunks = [(0, n_local)]
-        torch.cuda.synchronize()
-    sm, merge_note = None, "none (1 rank)"
-    if world > 1 and a.merge in ("peers", "owned"):
-        from paper_conf_asplos_linzs23_b200.parallel import SymmetricMerge
-        try:
-            sm = SymmetricMerge()
-            s = Session(prog.objects, prog.kinds, workspace_alloc=sm.alloc)
-            merge_note = ("drgpum_merge_peers_owned + finalize of the owned objects + drgpum_gather_peers "
-                          "over torch symmetric memory (NVLink P2P)" if a.merge == "owned" else
-                          "drgpum_merge_peers over torch symmetric memory (one kernel per rank, NVLink P2P)")
-        except Exception as e:   # symmetric memory unavailable: the NCCL exchange instead, said so
-            sm = None
-            merge_note = f"NCCL all_to_all + merge_or + all_gather (symmetric memory unavailable: {e})"
-    if sm is None:
-        s = Session(prog.objects, prog.kinds)
-        if world > 1 and a.merge == "nccl":
-            merge_note = "NCCL all_to_all + merge_or + all_gather"
-    stream = torch.cuda.current_stream()
-    owned = sm is not None and a.merge == "owned"
-
-    def do_merge():
-        if world > 1:
-            if owned:
-                sm.merge_owned(s)
-            elif sm is not None:
-                sm.merge(s)
-            else:
-                merge_session(s)
-
-    def do_finalize():
-        s.finalize()
-        if owned:
-            sm.gather(s)
-
-    def barrier():
-        if world > 1:
-            dist.barrier()
-
-    def one_step(src, ev=None):
-        """ev: per-phase event pairs [reset, attribute, merge, finalize]; the
-        attribute pair is per chunk (generation of a chunk lies outside it)."""
-        if ev: ev["reset"][0].record(stream)
-        s.reset()
-        if ev: ev["reset"][1].record(stream)
-        for k, (c0, c1) in enumerate(chunks):
-            if chunked:
-                dp.gen(lo + c0, lo + c1, out=src)
-            if ev: ev["attr"][k][0].record(stream)
-            s.attribute(src[:16 * (c1 - c0)])
-            if ev: ev["attr"][k][1].record(stream)
-        if ev: ev["merge"][0].record(stream)
-        do_merge()
-        if ev: ev["merge"][1].record(stream)
-        if ev: ev["fin"][0].record(stream)
-        do_finalize()
-        if ev: ev["fin"][1].record(stream)
-
-    def events():
-        E = lambda: (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-        return {"reset": E(), "attr": [E() for _ in chunks], "merge": E(), "fin": E()}
-
-    def phases(ev):   # ms
-        el = lambda e: e[0].elapsed_time(e[1])
-        return [el(ev["reset"]), sum(el(e) for e in ev["attr"]), el(ev["merge"]), el(ev["fin"])]
-
-    for _ in range(a.warmup):
-        one_step(d_recs)
-    torch.cuda.synchronize()
-    l0 = s.launch_count()
-    one_step(d_recs)
-    graph_launches = s.launch_count() - l0   # kernels of the library per step
-
-    # ---------------- device-resident timed region
-    # Phase breakdown: eager launches with events between the phases.
-    evs = [events() for _ in range(a.steps)]
-    torch.cuda.synchronize()
-    for k in range(a.steps):
-        one_step(d_recs, evs[k])
-    torch.cuda.synchronize()
-    ph = np.array([phases(e) for e in evs])  # ms
-    ph_mean = ph.mean(axis=0)
-    # The step itself: one CUDA graph of the library's launches (reset,
-    # attribute + range expansion, finalize), replayed K times -- the same
-    # kernels without per-launch host gaps.  Multi-rank steps (NCCL merge)
-    # run eagerly; chunked traces (generation between the chunks) are timed
-    # as the sum of their phase events.
-    use_graph = world == 1 and not a.no_graph and not chunked
-    if use_graph:
-        graph = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(graph):
-            one_step(d_recs)
-        for _ in range(a.warmup):
-            graph.replay()
-        torch.cuda.synchronize()
-    clk = ClockSampler(local)
-    time.sleep(0.3)
-    t_start = torch.cuda.Event(enable_timing=True)
-    t_end = torch.cuda.Event(enable_timing=True)
-    launches0 = s.launch_count()
-    barrier()
-    torch.cuda.synchronize()
-    wall0 = time.perf_counter()
-    t_start.record(stream)
-    tev = [events() for _ in range(a.steps)] if chunked else None
-    for k in range(a.steps):
-        if use_graph:
-            graph.replay()
-        else:
-            one_step(d_recs, tev[k] if chunked else None)
-    t_end.record(stream)
-    torch.cuda.synchronize()
-    barrier()
-    wall_dev = time.perf_counter() - wall0
-    # graph replays do not pass through the library's launch counter: count
-    # the captured launches once per replay
-    launches = (s.launch_count() - launches0) if not use_graph else graph_launches * a.steps
-    ms_total = t_start.elapsed_time(t_end)
-    if chunked:   # generation excluded: the steps are the sum of their phases
-        ms_total = float(sum(sum(phases(e)) for e in tev))
-    if world > 1:
-        t = torch.tensor([ms_total] + ph_mean.tolist(), dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_total = float(t[0])
-        ph_mean = t[1:].cpu().numpy()
-    ms_step = ms_total / a.steps
-    value = N / (ms_step / 1e3)
-
-    # calibration: attainable streaming-read bandwidth over the same record
-    # buffer (a torch reduction, not part of the path), so that the
-    # attribution can also be read as a fraction of "just reading the records"
-    cal = None
-    if not chunked:
-        v64 = d_recs.view(torch.int64)
-        for _ in range(3):
-            v64.sum()
-        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        torch.cuda.synchronize()
-        c0.record(stream)
-        for _ in range(5):
-            v64.sum()
-        c1.record(stream)
-        torch.cuda.synchronize()
-        rd_ms = c0.elapsed_time(c1) / 5
-        cal = {"read_gbs": 16.0 * n_local / (rd_ms / 1e3) / 1e9, "ms": rd_ms,
-               "how": "torch.sum over the resident record buffer viewed as int64 (read-only stream)"}
-
-    # touched shadow words (algorithmic write-back of A3/A4) of THIS rank's
-    # attribution: at N>1 the merged shadow is not what the rank's kernel
-    # wrote, so the shard is attributed once more alone, counted, and the
-    # merged step re-run (collectively) for the stats below
-    if world > 1:
-        s.reset()
-        for c0, c1 in chunks:
-            if chunked:
-                dp.gen(lo + c0, lo + c1, out=d_recs)
-            s.attribute(d_recs[:16 * (c1 - c0)])
-        touched = int(torch.count_nonzero(s.or_words()).item())
-        barrier()
-        one_step(d_recs)
-    else:
-        touched = int(torch.count_nonzero(s.or_words()).item())
-    stats, ctr = s.object_stats()
-    paths = s.path_stats()
-
-    # ---------------- end-to-end through the public API with HOST buffers
-    e2e_steps = a.e2e_steps or min(a.steps, 10)
-    n_e2e = n_local if not devgen else min(n_local, a.e2e_sample)
-    pinned = torch.empty(n_e2e * 16, dtype=torch.uint8, pin_memory=True)
-    pinned.numpy()[:] = (recs if recs is not None else gen_records(prog, lo, lo + n_e2e)).view(np.uint8)
-    for _ in range(2):
-        s.reset(); s.attribute(pinned); s.object_stats(); s.patterns()
-    torch.cuda.synchronize()
-    barrier()
-    w0 = time.perf_counter()
-    for _ in range(e2e_steps):
-        s.reset()
-        s.attribute(pinned)                 # drgpum_trace_attribute_host: H2D inside
-        do_merge()
-        if owned:
-            do_finalize()
-        st_h, ctr_h = s.object_stats()      # D2H of the result
-        rep_h = s.patterns()
-    torch.cuda.synchronize()
-    e2e_s = (time.perf_counter() - w0) / e2e_steps
-    if world > 1:
-        t = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_s = float(t[0])
-    clocks = clk.stop()
-    nxt = None
-    if world == 1 and not a.no_next and not devgen:
-        nxt = next_rows(prog, d_recs, float(ph_mean[1]))
-
-    if rank != 0:
-        dist.destroy_process_group()
-        return
+        t = torch.tensor([1, rank], dtype=torch.int64, device="cuda")
+        dist.all_reduce(t)
+        ranks = {"world": world, "backend": dist.get_backend(), "ranks_reporting": int(t[0]),
+                 "nccl_version": ".".join(map(str, torch.cuda.nccl.version()))}
+    w = Workload(a.config, a.records, rank, world, a.merge)
+    if ranks is not None and w.sm is not None:
+        ranks["symmetric_memory_peers"] = len(w.sm.peer_ptrs())
+    m = measure(w, a, a.steps, a.warmup, clocks=True, use_graph=not a.no_graph)
+    value = w.N / (m["ms_step"] / 1e3)
+    touched = touched_words(w)
+    parity = None if a.no_parity else parity_check(w, full=(world == 1))
+    if world > 1:   # every rank's verdict: all must hold the whole-trace results
+        ok = torch.tensor([1 if (parity or {}).get("ok", True) else 0], device="cuda")
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if parity is not None:
+            parity["all_ranks_ok"] = bool(int(ok))
+    stats, ctr = w.s.object_stats()     # the whole trace's (before the e2e leg resets it)
+    paths = w.s.path_stats()
+    e2e = e2e_leg(w, a, a.e2e_steps or min(a.steps, 5))
     hbm, hbm_src = peaks()
-    attr_ms = float(ph_mean[1])
-    alg_bytes = 16.0 * n_local + 4.0 * touched
-    achieved = alg_bytes / (attr_ms / 1e3) / 1e9
-    traffic = None
-    tfile = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tfile):
-        try:
-            t = json.load(open(tfile)).get(a.config)
-            traffic = None if t is None else int(t["bytes_per_launch"])
-        except Exception:
-            traffic = None
-
-    cpu = None
-    if world == 1 and not a.no_cpu_baseline:
-        m = min(a.cpu_sample or (20_000_000 if devgen else N), N, 100_000_000)
-        tcpu = time_oracle(prog.objects, prog.kinds, recs[:m] if recs is not None else gen_records(prog, 0, m))
-        cpu = {"value": m / tcpu, "unit": "records/s", "cores": 1, "kind": "oracle",
-               "sample": (f"{'all' if m == N else 'first'} {m} records of the {a.config} trace, "
-                          f"one pass: load + attribute + stats + patterns (O1, single thread)"),
-               "seconds": tcpu, "cpu": cpu_model(), "host_cores": os.cpu_count()}
-
+    rl = roofline(w, m, touched, hbm, hbm_src)
     line = {
         "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world,
-        "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms_step,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": m["ms_step"],
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
-        "data": f"synthetic (tracegen {prog.name}, seed {prog.seed:#x})",
-        "config": {"workload": WORKLOADS[a.config], "records": N, "objects": prog.n_obj,
-                   "n_api": prog.n_api, "parallelism": f"record-range x{world}", "merge": merge_note,
-                   "l2": f"inputs larger than L2 ({16 * N / 2**30:.2f} GiB of records streamed per step)",
-                   "shadow_words": int(s.view.or_words), "touched_words": touched},
-        "phases_ms": {"reset": float(ph_mean[0]), "attribute": attr_ms,
-                      "merge": float(ph_mean[2]), "finalize": float(ph_mean[3])},
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                     "frac": achieved / hbm, "traffic": traffic,
-                     "kernel": "drgpum_trace_attribute (attribute_kernel + range_expand_kernel)",
-                     "algorithmic_bytes": alg_bytes,
-                     "bytes_rule": "16 B per record + 4 B per touched shadow word",
-                     "peak_source": hbm_src},
-        "calibration": None if cal is None else dict(cal, attribution_frac_of_read=cal["read_gbs"] and
-                                                     (16.0 * n_local / (attr_ms / 1e3) / 1e9) / cal["read_gbs"]),
-        "cpu_baseline": cpu,
-        "e2e": {"value": n_e2e * world / e2e_s, "unit": "records/s", "h2d_bytes_per_step": 16 * n_e2e,
-                "records_per_rank": n_e2e,
-                "d2h_bytes_per_step": int(prog.n_obj * (56 + 32) + 40),
-                "ms_per_step": e2e_s * 1e3,
-                "path": "Session.attribute(pinned host tensor) -> drgpum_trace_attribute_host; "
-                        "object_stats + patterns (D2H)"},
-        "gpu_launches": launches,
-        "step_exec": "cuda_graph_replay" if use_graph else "eager",
-        "clocks": clocks,
+        "data": f"synthetic (tracegen {w.prog.name}, seed {w.prog.seed:#x}; records generated on the device)",
+        "config": {"workload": WORKLOADS[a.config], "records": w.N, "objects": w.prog.n_obj,
+                   "n_api": w.prog.n_api, "parallelism": f"record-range x{world}", "merge": w.merge_note,
+                   "records_per_rank": w.n_local,
+                   "residency": (f"streamed: {len(w.chunks)} chunks of <= {GEN_CHUNK} records generated on the "
+                                 f"device per step, outside the timed events (value = records / sum of the "
+                                 f"steps' reset + attribute + merge + finalize events)") if w.chunked
+                   else "resident in HBM for the whole timed region",
+                   "l2": f"inputs larger than L2 ({16 * w.n_local / 2**30:.2f} GiB of records per rank per step)",
+                   "shadow_words": int(w.s.view.or_words), "touched_words": touched},
+        "phases_ms": dict(zip(("reset", "attribute", "merge", "finalize"), map(float, m["phases"]))),
+        "roofline": rl,
+        "parity": parity,
+        "ranks": ranks,
+        "e2e": e2e,
+        "gpu_launches": m["launches"],
+        "step_exec": "cuda_graph_replay" if m["graphed"] else f"eager ({w.graph_note})",
+        "clocks": m["clocks"],
         "counters": {k: int(ctr[k]) for k in ctr.dtype.names},
         "attribution_paths_tiles": paths,
-        "wall_s_device_region": wall_dev,
-        "next": nxt,
+        "wall_s_device_region": m["wall"],
     }
-    print(json.dumps(line), flush=True)
+    cpu = None
+    if world == 1 and not a.no_cpu_baseline:
+        from tracegen import gen_records
+        sub, desc = oracle_sample(w.prog, a.cpu_sample)
+        recs = gen_records(sub, 0, sub.n_records)
+        tcpu = time_oracle(sub.objects, sub.kinds, recs)
+        del recs
+        cpu = {"value": sub.n_records / tcpu, "unit": "records/s", "cores": 1, "kind": "oracle",
+               "sample": desc, "seconds": tcpu, "cpu": cpu_model(), "host_cores": os.cpu_count()}
+    line["cpu_baseline"] = cpu
+    w.close()
+    if world == 1 and a.extra_configs:
+        line["other_configs"] = {}
+        for cfg in [c for c in a.extra_configs.split(",") if c and c != a.config]:
+            try:
+                line["other_configs"][cfg] = other_config(cfg, a, hbm, hbm_src)
+            except Exception as e:   # noqa: BLE001 -- an extra must not lose the main line
+                line["other_configs"][cfg] = {"error": f"{type(e).__name__}: {e}"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
 

@@ -33,10 +33,27 @@
  *     uses lives inside it.  The library never allocates device memory except
  *     two tiny event/stream objects for drgpum_trace_attribute_host.
  *   - One context per device (per rank).  A context is not thread-safe.
- *   - Call order: create -> objects_load -> workspace_bind ->
- *     { trace_attribute | trace_attribute_host }* -> [merge_or ... | merge_peers] ->
- *     finalize / object_stats / patterns.  drgpum_reset starts a new trace on
- *     the same objects.  Out-of-order calls return DRGPUM_ESTATE.
+ *   - Call order: create -> objects_load -> [set_features] [set_queue_capacity]
+ *     -> workspace_bind -> { trace_attribute | trace_attribute_host }* ->
+ *     one of the merges (multi-rank only):
+ *       (a) merge_or ... (after an all-to-all) or merge_peers, between two
+ *           barriers: afterwards every rank holds the whole merged shadow;
+ *       (b) barrier, merge_peers_owned, barrier, finalize, barrier,
+ *           gather_peers, barrier: afterwards every rank holds every
+ *           object's stats and reports, but its shadow (bitmaps, hit rows,
+ *           first/last) is merged for ITS OWN objects only;
+ *     -> finalize / object_stats / patterns / NEXT-row queries.
+ *     drgpum_reset starts a new trace on the same objects (and clears the
+ *     owned-merge state).  Out-of-order calls return DRGPUM_ESTATE.
+ *   - What a rank can read after an owned merge (b): object_stats, patterns
+ *     (with the finalize's thresholds), consistency_errors and
+ *     redundant_alloc are whole-trace results once gather_peers is done;
+ *     dependency_graph and patterns_topo return ESTATE (they read every
+ *     object's hit row); the bitmap / hit-row words, first/last of the other
+ *     ranks' objects in the shadow view are this rank's partial ones.  The
+ *     NEXT-2 / NEXT-3 results (drgpum_frequency, drgpum_structured) are never
+ *     merged by any of the merges: they cover the records this rank
+ *     attributed.
  */
 #ifndef DRGPUM_H
 #define DRGPUM_H
@@ -194,6 +211,18 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx *ctx,
  * access pass over its records. */
 enum { DRGPUM_FEATURE_STRUCTURED = 1, DRGPUM_FEATURE_FREQUENCY = 2 };
 DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx *ctx, uint32_t features);
+
+/* Capacity of the device work queues, in entries (0 = keep the current
+ * value; defaults 2^20 each).  range_entries sizes the A3b range-expansion
+ * queue (16 B per entry, <= 4096 words each); aux_entries the wide-record
+ * queues of the NEXT-2 / NEXT-3 passes.  A queue that fills up is never an
+ * error: the records that do not fit are expanded in place by the warp that
+ * found them (exact, slower), and the range-queue overflow is counted.
+ * Smaller queues shrink the workspace; tests use tiny ones to drive the
+ * overflow paths.  Set after objects_load and before workspace_size /
+ * workspace_bind (ESTATE otherwise); EINVAL above 2^24 entries. */
+DRGPUM_API drgpum_status drgpum_set_queue_capacity(drgpum_ctx *ctx, uint32_t range_entries,
+                                                   uint32_t aux_entries);
 
 /* Bytes of device workspace the loaded program needs (ESTATE before load). */
 DRGPUM_API drgpum_status drgpum_workspace_size(const drgpum_ctx *ctx, uint64_t *bytes);

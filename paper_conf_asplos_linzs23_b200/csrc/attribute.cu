@@ -1052,16 +1052,17 @@ __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
   }
 }
 
-int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s) {
+int attribute_occupancy() {
+  int occ = 0;
+  cudaFuncSetAttribute(attribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kAttrSmem));
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, attribute_kernel, kAttrThreads, kAttrSmem);
+  return occ < 1 ? 1 : occ;
+}
+
+int launch_attribute(const AttrParams& p, int num_sms, int occ, cudaStream_t s) {
   if (p.n == 0) return 0;
   // C_WORK and this call's queue count are zero here: zeroed by the reset,
   // then re-armed by the previous call's range_expand_kernel
-  static int occ = 0;
-  if (!occ) {
-    cudaFuncSetAttribute(attribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kAttrSmem));
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, attribute_kernel, kAttrThreads, kAttrSmem);
-    if (occ < 1) occ = 1;
-  }
   // enough stages per block to keep the ring busy, at most one wave
   uint64_t blocks = (p.n + 4ull * kConsumerWarps * kWarpRecords - 1) / (4ull * kConsumerWarps * kWarpRecords);
   const uint64_t full = uint64_t(num_sms) * occ;

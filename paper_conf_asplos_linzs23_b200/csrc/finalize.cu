@@ -766,7 +766,7 @@ __global__ void __launch_bounds__(256) gather_peers_kernel(const GatherParams q)
   if (tid == 0) {
     const unsigned long long mine = reinterpret_cast<const unsigned long long*>(own + q.ctr_off)[C_CONSISTENCY];
     for (uint32_t r = 0; r < q.n_peers; ++r)
-      atomicAdd(reinterpret_cast<unsigned long long*>(q.peer[r] + q.ctr_off) + C_CONSISTENCY_ALL, mine);
+      reinterpret_cast<unsigned long long*>(q.peer[r] + q.cons_off)[q.rank] = mine;
   }
 }
 

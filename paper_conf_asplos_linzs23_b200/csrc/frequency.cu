@@ -577,7 +577,14 @@ __global__ void __launch_bounds__(256) frequency_reduce_kernel(const FreqReduceP
   }
 }
 
-int launch_frequency(const FreqParams& q, uint64_t n_slots, int num_sms, cudaStream_t s) {
+int frequency_occupancy() {
+  int occ = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, freq_apply_kernel, kFreqThreads, 0);
+  if (occ < 1) occ = 1;
+  return occ > 2 ? 2 : occ;
+}
+
+int launch_frequency(const FreqParams& q, uint64_t n_slots, int num_sms, int occ, cudaStream_t s) {
   if (q.a.n == 0) return 0;
   const uint64_t n_api = q.a.n_api;
   cudaMemsetAsync(q.ctl, 0, sizeof(FreqCtl), s);
@@ -596,12 +603,6 @@ int launch_frequency(const FreqParams& q, uint64_t n_slots, int num_sms, cudaStr
   freq_count_kernel<<<(unsigned)b, 256, 0, s>>>(q);
   freq_slotseg_kernel<<<num_sms, 256, 0, s>>>(q);
   freq_table_plan_kernel<<<1, 1024, 0, s>>>(q);
-  static int occ = 0;
-  if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, freq_apply_kernel, kFreqThreads, 0);
-    if (occ < 1) occ = 1;
-    if (occ > 2) occ = 2;
-  }
   void* args[] = {const_cast<FreqParams*>(&q)};
   cudaLaunchCooperativeKernel((void*)freq_apply_kernel, dim3(num_sms * occ), dim3(kFreqThreads), args, 0, s);
   return 6;

@@ -32,7 +32,7 @@ namespace {
 enum State { S_CREATED = 0, S_LOADED = 1, S_BOUND = 2 };
 
 struct Layout {
-  uint64_t orw, first, last, ctr;           // dynamic (reset per trace)
+  uint64_t orw, first, last, ctr, cons;     // dynamic (reset per trace)
   uint64_t dyn_end;
   uint64_t objs, seg_start, seg_cand_off, seg, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
   uint64_t rfull;                 // per object: a whole-object range was queued in this trace
@@ -53,6 +53,7 @@ inline uint64_t align_up(uint64_t x, uint64_t a = kAlign) { return (x + a - 1) /
 struct drgpum_ctx {
   int device = 0;
   int num_sms = 148;
+  int attr_occ = 1, freq_occ = 1;   // blocks per SM of the persistent kernels, on this device
   State state = S_CREATED;
   std::string err;
   uint64_t launches = 0;
@@ -125,7 +126,14 @@ template <typename T> T* at(drgpum_ctx* c, uint64_t off) { return reinterpret_ca
 
 cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
 
-drgpum_status set_device(drgpum_ctx* ctx) { CK(cudaSetDevice(ctx->device)); return DRGPUM_OK; }
+// Every launching / copying entry point runs on the context's device,
+// whichever device the calling thread has current.
+drgpum_status set_device(drgpum_ctx* ctx) {
+  int cur = -1;
+  if (cudaGetDevice(&cur) == cudaSuccess && cur == ctx->device) return DRGPUM_OK;
+  CK(cudaSetDevice(ctx->device));
+  return DRGPUM_OK;
+}
 
 uint32_t ilog2(uint32_t e) { uint32_t s = 0; while ((1u << s) < e) ++s; return s; }
 
@@ -308,6 +316,7 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   L.first = put(4 * n);
   L.last = put(4 * n);
   L.ctr = put(8 * C_SLOTS);
+  L.cons = put(8 * kMaxPeers);   // per-rank consistency counts after gather_peers
   L.rfull = put(4 * n);
   L.dyn_end = off;
   L.objs = put(sizeof(DevObj) * n);
@@ -535,9 +544,22 @@ DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx* ctx, uint32_t features)
   return compute_layout(ctx);
 }
 
+DRGPUM_API drgpum_status drgpum_set_queue_capacity(drgpum_ctx* ctx, uint32_t range_entries,
+                                                   uint32_t aux_entries) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state != S_LOADED)
+    return fail(ctx, DRGPUM_ESTATE, "set_queue_capacity must follow objects_load and precede workspace_bind");
+  if (range_entries > (1u << 24) || aux_entries > (1u << 24))
+    return fail(ctx, DRGPUM_EINVAL, "queue capacity above 2^24 entries");
+  if (range_entries) ctx->rq_cap = range_entries;
+  if (aux_entries) ctx->sa_q_cap = aux_entries;
+  return compute_layout(ctx);
+}
+
 DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx* ctx, uint8_t* h_sa, uint8_t* h_overlap, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "structured before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   if (!(ctx->features & DRGPUM_FEATURE_STRUCTURED))
     return fail(ctx, DRGPUM_ESTATE, "DRGPUM_FEATURE_STRUCTURED was not enabled");
   std::vector<drgpum_object_stats_t> st(ctx->n_obj);
@@ -558,6 +580,7 @@ DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx* ctx, uint8_t* h_sa, uint8
 
 static drgpum_status frequency_ready(drgpum_ctx* ctx, cudaStream_t st) {
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "frequency before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   if (!(ctx->features & DRGPUM_FEATURE_FREQUENCY))
     return fail(ctx, DRGPUM_ESTATE, "DRGPUM_FEATURE_FREQUENCY was not enabled");
   uint32_t state[2];
@@ -625,6 +648,10 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
                 (unsigned long long)bytes, (unsigned long long)ctx->L.total);
   drgpum_status s = set_device(ctx);
   if (s != DRGPUM_OK) return s;
+  // per-device kernel attributes and occupancy, kept in the context
+  ctx->attr_occ = attribute_occupancy();
+  ctx->freq_occ = frequency_occupancy();
+  CK(cudaGetLastError());
   cudaStream_t st = as_stream(stream);
   ctx->ws = static_cast<uint8_t*>(d_ws);
   ctx->ws_bytes = bytes;
@@ -664,6 +691,7 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
 DRGPUM_API drgpum_status drgpum_reset(drgpum_ctx* ctx, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "reset before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   return enqueue_reset(ctx, as_stream(stream));
 }
 
@@ -671,16 +699,17 @@ DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_re
                                                 uint64_t n, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "trace_attribute before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   if (n == 0) return DRGPUM_OK;
   if (!d_recs || reinterpret_cast<uintptr_t>(d_recs) % 16)
     return fail(ctx, DRGPUM_EINVAL, "records must be non-NULL and 16-B aligned");
   AttrParams p = attr_params(ctx, d_recs, n);
-  ctx->launches += launch_attribute(p, ctx->num_sms, as_stream(stream));
+  ctx->launches += launch_attribute(p, ctx->num_sms, ctx->attr_occ, as_stream(stream));
   ctx->attr_calls++;
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     ctx->launches += launch_structured(sa_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
-    ctx->launches += launch_frequency(fq_params(ctx, d_recs, n), ctx->n_slots, ctx->num_sms, as_stream(stream));
+    ctx->launches += launch_frequency(fq_params(ctx, d_recs, n), ctx->n_slots, ctx->num_sms, ctx->freq_occ, as_stream(stream));
   ctx->final_valid = false;
   CK(cudaGetLastError());
   return DRGPUM_OK;
@@ -690,6 +719,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
                                                      uint64_t n, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "trace_attribute_host before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   if (n == 0) return DRGPUM_OK;
   if (!h_recs) return fail(ctx, DRGPUM_EINVAL, "records is NULL");
   cudaStream_t st = as_stream(stream);
@@ -715,12 +745,12 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
     CK(cudaEventRecord(ctx->ev_copied[b], ctx->copy_stream));
     CK(cudaStreamWaitEvent(st, ctx->ev_copied[b], 0));
     AttrParams p = attr_params(ctx, stage[b], m);
-    ctx->launches += launch_attribute(p, ctx->num_sms, st);
+    ctx->launches += launch_attribute(p, ctx->num_sms, ctx->attr_occ, st);
     ctx->attr_calls++;
     if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
       ctx->launches += launch_structured(sa_params(ctx, stage[b], m), ctx->num_sms, st);
     if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
-      ctx->launches += launch_frequency(fq_params(ctx, stage[b], m), ctx->n_slots, ctx->num_sms, st);
+      ctx->launches += launch_frequency(fq_params(ctx, stage[b], m), ctx->n_slots, ctx->num_sms, ctx->freq_occ, st);
     CK(cudaEventRecord(ctx->ev_used[b], st));
   }
   CK(cudaStreamSynchronize(ctx->copy_stream));
@@ -755,6 +785,7 @@ DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx* ctx, const uint32_t* d_in, 
                                          uint64_t word_hi, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_or before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   const uint64_t total = ctx->bitmap_words + ctx->hit_words;
   ctx->final_valid = false;  // the caller is merging state into this shadow
   if (word_lo > word_hi || word_hi > total)
@@ -805,6 +836,7 @@ DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx* ctx, void* const* h_peer
                                             uint32_t rank, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   MergePeersParams q{};
   if (drgpum_status e = check_peers(ctx, "merge_peers", h_peer_ws, n_peers, rank, q.peer)) return e;
   q.n_peers = n_peers;
@@ -833,6 +865,7 @@ DRGPUM_API drgpum_status drgpum_merge_peers_owned(drgpum_ctx* ctx, void* const* 
                                                   uint32_t n_peers, uint32_t rank, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers_owned before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   MergeOwnedParams q{};
   if (drgpum_status e = check_peers(ctx, "merge_peers_owned", h_peer_ws, n_peers, rank, q.peer)) return e;
   q.n_peers = n_peers;
@@ -860,6 +893,7 @@ DRGPUM_API drgpum_status drgpum_gather_peers(drgpum_ctx* ctx, void* const* h_pee
                                              uint32_t n_peers, uint32_t rank, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "gather_peers before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   GatherParams q{};
   if (drgpum_status e = check_peers(ctx, "gather_peers", h_peer_ws, n_peers, rank, q.peer)) return e;
   if (!ctx->owned || !ctx->final_valid)
@@ -877,6 +911,7 @@ DRGPUM_API drgpum_status drgpum_gather_peers(drgpum_ctx* ctx, void* const* h_pee
   q.r_lo = ctx->own_lo * sizeof(drgpum_pattern_report_t);
   q.r_hi = ctx->own_hi * sizeof(drgpum_pattern_report_t);
   q.ctr_off = ctx->L.ctr;
+  q.cons_off = ctx->L.cons;
   ctx->launches += launch_gather_peers(q, ctx->num_sms, as_stream(stream));
   CK(cudaGetLastError());
   ctx->gathered = true;
@@ -886,6 +921,7 @@ DRGPUM_API drgpum_status drgpum_gather_peers(drgpum_ctx* ctx, void* const* h_pee
 DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_thresholds_t* th, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "finalize before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   drgpum_thresholds_t t = th ? *th : drgpum_thresholds_t{2, 80, 80};
   cudaStream_t st = as_stream(stream);
   FinalParams p;
@@ -934,6 +970,7 @@ DRGPUM_API drgpum_status drgpum_object_stats(drgpum_ctx* ctx, drgpum_object_stat
                                              drgpum_counters_t* h_ctr, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "object_stats before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   cudaStream_t st = as_stream(stream);
   if (ctx->owned && !(ctx->final_valid && ctx->gathered))
     return fail(ctx, DRGPUM_ESTATE, "object_stats after merge_peers_owned needs finalize + gather_peers");
@@ -961,6 +998,7 @@ DRGPUM_API drgpum_status drgpum_patterns(drgpum_ctx* ctx, const drgpum_threshold
                                          drgpum_pattern_report_t* h_out, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "patterns before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   drgpum_thresholds_t t = th ? *th : drgpum_thresholds_t{2, 80, 80};
   cudaStream_t st = as_stream(stream);
   if (ctx->owned && !(ctx->final_valid && ctx->gathered && same_th(t, ctx->final_th)))
@@ -979,17 +1017,26 @@ DRGPUM_API drgpum_status drgpum_patterns(drgpum_ctx* ctx, const drgpum_threshold
 DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx* ctx, uint64_t* h_errors, void* stream) {
   if (!ctx || !h_errors) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return DRGPUM_ESTATE;
+  if (drgpum_status _d = set_device(ctx)) return _d;
   cudaStream_t st = as_stream(stream);
-  unsigned long long c[C_SLOTS];
+  unsigned long long c[C_SLOTS], per_rank[kMaxPeers];
   CK(cudaMemcpyAsync(c, ctx->ws + ctx->L.ctr, sizeof c, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(per_rank, ctx->ws + ctx->L.cons, sizeof per_rank, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
-  *h_errors = ctx->owned && ctx->gathered ? c[C_CONSISTENCY_ALL] : c[C_CONSISTENCY];
+  if (ctx->owned && ctx->gathered) {   // every rank's count of its own objects
+    uint64_t sum = 0;
+    for (uint32_t r = 0; r < ctx->own_P; ++r) sum += per_rank[r];
+    *h_errors = sum;
+  } else {
+    *h_errors = c[C_CONSISTENCY];
+  }
   return DRGPUM_OK;
 }
 
 DRGPUM_API drgpum_status drgpum_path_stats(drgpum_ctx* ctx, uint64_t out[4], void* stream) {
   if (!ctx || !out) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return DRGPUM_ESTATE;
+  if (drgpum_status _d = set_device(ctx)) return _d;
   cudaStream_t st = as_stream(stream);
   unsigned long long c[C_SLOTS];
   CK(cudaMemcpyAsync(c, ctx->ws + ctx->L.ctr, sizeof c, cudaMemcpyDeviceToHost, st));
@@ -1006,6 +1053,7 @@ DRGPUM_API drgpum_status drgpum_redundant_alloc(drgpum_ctx* ctx, uint32_t pct, u
                                                 void* stream) {
   if (!ctx || !n_pairs || (cap && (!reuser || !donor))) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "redundant_alloc before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
   std::vector<drgpum_object_stats_t> st(ctx->n_obj);
   drgpum_status s = drgpum_object_stats(ctx, st.data(), nullptr, stream);
   if (s != DRGPUM_OK) return s;
@@ -1066,6 +1114,10 @@ DRGPUM_API drgpum_status drgpum_dependency_graph(drgpum_ctx* ctx, const uint32_t
   if (!ctx || !n_edges || (ctx->n_api && !h_stream) || (cap && !h_src && !h_dst && !h_label))
     return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "dependency_graph before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
+  if (ctx->owned)   // hit rows are merged for this rank's objects only
+    return fail(ctx, DRGPUM_ESTATE, "dependency_graph after merge_peers_owned: the hit rows of the other ranks' "
+                "objects are not merged here (use merge_peers or merge_or)");
   std::vector<uint64_t> off;
   std::vector<uint32_t> api;
   std::vector<uint8_t> rw;
@@ -1096,6 +1148,10 @@ DRGPUM_API drgpum_status drgpum_patterns_topo(drgpum_ctx* ctx, const uint32_t* h
                                               drgpum_pattern_report_t* h_out, void* stream) {
   if (!ctx || !h_out || (ctx->n_api && !h_T)) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "patterns_topo before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
+  if (ctx->owned)   // hit rows are merged for this rank's objects only
+    return fail(ctx, DRGPUM_ESTATE, "patterns_topo after merge_peers_owned: the hit rows of the other ranks' "
+                "objects are not merged here (use merge_peers or merge_or)");
   const uint32_t n_api = ctx->n_api;
   for (uint32_t v = 0; v < n_api; ++v)
     if (h_T[v] >= n_api) return fail(ctx, DRGPUM_EINVAL, "T[%u] = %u >= n_api", v, h_T[v]);

@@ -61,7 +61,7 @@ enum : int { C_RECORDS = 0, C_ATTRIBUTED, C_UNATTRIBUTED, C_CLIPPED, C_INVALID,
              C_TILES_AFFINE_UNION, C_TILES_AFFINE_WORDS, C_TILES_FAST, C_TILES_SLOW,
              C_WORK,   // attribution work cursor (chunk tickets handed out)
              C_RQ_COUNT_ALT,   // range-queue count of odd-numbered attribute calls
-             C_CONSISTENCY_ALL,   // sum of every rank's C_CONSISTENCY after gather_peers
+             C_RESERVED14,
              C_SLOTS = 16 };
 
 struct AttrParams {
@@ -192,18 +192,23 @@ struct MergeOwnedParams {
 };
 
 // Gather (B7''): rank r stores bytes [lo, hi) of the stats and of the
-// reports sections (its objects) into every peer, and adds its consistency
-// count into every peer's C_CONSISTENCY_ALL.
+// reports sections (its objects) into every peer, and its consistency count
+// into slot r of every peer's per-rank consistency array (a plain store, so
+// a re-finalize + re-gather replaces the count instead of adding it again).
 struct GatherParams {
   uint8_t* peer[kMaxPeers];
   uint32_t n_peers, rank;
-  uint64_t stats_off, s_lo, s_hi, reports_off, r_lo, r_hi, ctr_off;
+  uint64_t stats_off, s_lo, s_hi, reports_off, r_lo, r_hi, ctr_off, cons_off;
 };
 
 // Launchers (return the number of kernels enqueued).
-int launch_attribute(const AttrParams& p, int num_sms, cudaStream_t s);   // p.rq_slot alternates per call
+// Set the kernels' attributes on the CURRENT device and return their
+// resident blocks per SM (called by workspace_bind; cached in the context).
+int attribute_occupancy();
+int frequency_occupancy();
+int launch_attribute(const AttrParams& p, int num_sms, int occ, cudaStream_t s);   // p.rq_slot alternates per call
 int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
-int launch_frequency(const FreqParams& p, uint64_t n_slots, int num_sms, cudaStream_t s);
+int launch_frequency(const FreqParams& p, uint64_t n_slots, int num_sms, int occ, cudaStream_t s);
 int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t s);
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);

@@ -38,7 +38,8 @@ class Session:
     kinds:   uint8 array, the GPU-API kind of every timestamp.
     """
 
-    def __init__(self, objects, kinds, device=None, structured=False, frequency=False, workspace_alloc=None):
+    def __init__(self, objects, kinds, device=None, structured=False, frequency=False, workspace_alloc=None,
+                 queue_capacity=None):
         if not torch.cuda.is_available():
             raise RuntimeError("drgpum Session needs a CUDA device (there is no CPU fallback)")
         self.L = _lib.load()
@@ -59,6 +60,8 @@ class Session:
         feats = (_lib.FEATURE_STRUCTURED if structured else 0) | (_lib.FEATURE_FREQUENCY if frequency else 0)
         if feats:
             check(self._h, self.L.drgpum_set_features(self._h, feats))
+        if queue_capacity is not None:   # (range entries, aux entries); tests drive the overflow paths
+            check(self._h, self.L.drgpum_set_queue_capacity(self._h, *queue_capacity))
         nbytes = ctypes.c_uint64()
         check(self._h, self.L.drgpum_workspace_size(self._h, ctypes.byref(nbytes)))
         # workspace_alloc(nbytes, device) -> uint8 CUDA tensor (e.g. torch
@@ -235,6 +238,12 @@ class Session:
     def counters_tensor(self):
         v = self.view
         return self.workspace[v.counters_off: v.counters_off + 8 * 5].view(torch.int64)
+
+    def raw_counters(self):
+        """All 16 u64 counter slots of the workspace (diagnostics: [5] is the
+        range-queue overflow count, [6] the consistency count)."""
+        v = self.view
+        return self.workspace[v.counters_off: v.counters_off + 8 * 16].view(torch.int64)
 
     def merge_or(self, src, n_src, src_stride_words, word_lo, word_hi, stream=None):
         check(self._h, self.L.drgpum_merge_or(self._h, ctypes.c_void_p(src.data_ptr()), n_src,

@@ -12,10 +12,10 @@ import pytest
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-@pytest.mark.parametrize("config", ["C2", "C3"])
+@pytest.mark.parametrize("config", ["C2", "C3", "C5"])
 def test_reference_arm_json_line(config):
     out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference",
-                          "--config", config, "--steps", "1", "--warmup", "0", "--ref-sample", "20000"],
+                          "--config", config, "--steps", "1", "--warmup", "0", "--ref-sample", "200000"],
                          capture_output=True, text=True, timeout=600, cwd=ROOT)
     assert out.returncode == 0, out.stderr[-2000:]
     lines = [l for l in out.stdout.splitlines() if l.strip()]
@@ -29,6 +29,8 @@ def test_reference_arm_json_line(config):
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0
     assert config in d["config"]["workload"]
+    assert d["same_config"] is True and d["config"]["sample_records"] > 0
+    assert "index %" in d["cpu_baseline"]["sample"]
 
 
 def test_reference_arm_other_ranks_are_silent():
@@ -37,3 +39,23 @@ def test_reference_arm_other_ranks_are_silent():
                           "--steps", "1", "--warmup", "0", "--ref-sample", "1000"],
                          capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
     assert out.returncode == 0 and out.stdout.strip() == ""
+
+
+def test_gpus_2_launches_two_ranks():
+    """bench.py --gpus N without torchrun re-launches itself with N ranks
+    (torch.distributed.run); --dry-run checks the rank plumbing over gloo."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--dry-run"],
+                         capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.strip().startswith("{")]
+    assert len(lines) == 1, out.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["ranks_reporting"] == 2 and d["rank_sum"] == 1
+
+
+def test_world_size_must_match_gpus():
+    env = dict(os.environ, RANK="0", WORLD_SIZE="1", LOCAL_RANK="0")
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--dry-run"],
+                         capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
+    assert out.returncode != 0 and "WORLD_SIZE=1" in (out.stderr + out.stdout)

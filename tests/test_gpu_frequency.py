@@ -13,9 +13,9 @@ def _sorted(recs):
     return recs[np.argsort(recs["meta"] & 0x7FFFFFFF, kind="stable")]
 
 
-def _check(objs, kinds, recs, chunks=1, pct=20):
+def _check(objs, kinds, recs, chunks=1, pct=20, queue_capacity=None):
     from paper_conf_asplos_linzs23_b200 import Session
-    s = Session(objs, kinds, frequency=True)
+    s = Session(objs, kinds, frequency=True, queue_capacity=queue_capacity)
     d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
     b = np.linspace(0, len(recs), chunks + 1).astype(np.int64)
     for x, y in zip(b, b[1:]):
@@ -104,3 +104,13 @@ def _chain_program(seed, n_apis=400, n_elem=2048):
 def test_dependency_chain(seed, chunks):
     objs, kinds, r = _chain_program(seed)
     _check(objs, kinds, r, chunks=chunks)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_wide_record_queue_overflow(seed):
+    """Wide records that do not fit the chunk queue (capacity 1) are counted
+    in place by the warp that found them (frequency.cu queue_range)."""
+    p = build_tiny(seed)
+    _check(p.objects, p.kinds, _sorted(gen_all_records(p)), queue_capacity=(0, 1))
+    c = build_config("C1")
+    _check(c.objects, c.kinds, _sorted(gen_all_records(c)), queue_capacity=(0, 1))

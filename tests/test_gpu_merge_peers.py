@@ -234,6 +234,26 @@ def test_owned_state_rules():
     a.object_stats()
     with pytest.raises(DrgpumError):
         a.patterns((3, 80, 80))
+    # NEXT-4 reads every object's hit row: refused after an owned merge
+    streams = np.zeros(p.n_api, np.uint32)
+    with pytest.raises(DrgpumError):
+        a.dependency_graph(streams)
+    with pytest.raises(DrgpumError):
+        a.patterns_topo(np.arange(p.n_api, dtype=np.uint32))
+    # re-finalize + re-gather (the flow the header prescribes for new
+    # thresholds) replaces each rank's consistency count instead of adding it
+    assert a.consistency_errors() == 0 and b.consistency_errors() == 0
+    a.first_last()[0].fill_(0)     # corrupt rank 0's first-use words: its objects now disagree
+    counts = []
+    for _ in range(2):
+        a.finalize((3, 80, 80)); b.finalize((3, 80, 80))
+        torch.cuda.synchronize()
+        a.gather_peers(ptrs, 0); b.gather_peers(ptrs, 1)
+        torch.cuda.synchronize()
+        counts.append((a.consistency_errors(), b.consistency_errors()))
+    a.patterns((3, 80, 80))
+    assert counts[0][0] > 0 and counts[0][0] == counts[0][1] and counts[1] == counts[0], counts
     a.reset()                                       # a new trace: ordinary rules again
     a.attribute(d)
     a.patterns((3, 80, 80))
+    a.dependency_graph(streams)

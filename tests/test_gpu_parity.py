@@ -18,9 +18,9 @@ from tracegen import (build_config, build_tiny, gen_all_records, gen_records, OB
 from tests.golden_util import golden_names, load, to_arrays  # noqa: E402
 
 
-def _session(objs, kinds):
+def _session(objs, kinds, **kw):
     from paper_conf_asplos_linzs23_b200 import Session
-    return Session(objs, kinds)
+    return Session(objs, kinds, **kw)
 
 
 def _acc_rank(kinds):
@@ -56,8 +56,8 @@ def expected_or_words(s, orc, objs, kinds):
     return exp
 
 
-def run_gpu(objs, kinds, recs, chunks=1, host=False, th=None, shuffle_seed=None):
-    s = _session(objs, kinds)
+def run_gpu(objs, kinds, recs, chunks=1, host=False, th=None, shuffle_seed=None, session_kw=None):
+    s = _session(objs, kinds, **(session_kw or {}))
     r = recs
     if shuffle_seed is not None:
         r = recs[np.random.default_rng(shuffle_seed).permutation(len(recs))]
@@ -229,3 +229,86 @@ def test_redundant_allocation_end_to_end(name):
     want = redundant_allocations(p.objects["size"], ost["t_first"], ost["t_last"],
                                  ost["n_access_apis"] > 0, 10)
     assert got == want and len(want) > 0
+
+
+# ---------------------------------------------------------------- queue overflow
+@pytest.mark.parametrize("cap", [1, 3])
+def test_range_queue_overflow(cap):
+    """A3b: with a range queue of `cap` entries, every range record that does
+    not fit is expanded in place by the warp that found it (attribute.cu
+    enqueue_range's fallback).  Results must still equal the oracle's, and
+    the overflow counter must show that the fallback ran."""
+    kinds = np.array([0, 0, 3, 2, 3, 4, 2, 1], dtype=np.uint8)
+    objs = np.zeros(2, dtype=OBJ_DTYPE)
+    objs[0] = (1 << 40, 1 << 26, 4, 0, 7, 0)        # 2^24 elements: 128 range chunks
+    objs[1] = ((1 << 40) + (1 << 27), 3 << 20, 1, 1, NEVER, 1)
+    recs = np.zeros(8, dtype=REC_DTYPE)
+    recs[0] = ((1 << 40) + 4, (1 << 26) - 9, 2 | (1 << 31))        # memset, ragged
+    recs[1] = ((1 << 40) + (1 << 27) + 1, (3 << 20) - 2, 2 | (1 << 31))
+    recs[2] = ((1 << 40) + 1000, 1 << 20, 3)                        # memcpy read
+    recs[3] = ((1 << 40) + (1 << 27) + 5, 777777, 3 | (1 << 31))
+    recs[4] = ((1 << 40) + 12345 * 4, 99999, 4 | (1 << 31))         # memset
+    recs[5] = ((1 << 40) + 8, 4, 5)                                 # kernel, inline
+    recs[6] = ((1 << 40) + (1 << 27), 3 << 20, 6)                   # whole object
+    recs[7] = ((1 << 40) + (1 << 26) - 64, 0xFFFF, 6 | (1 << 31))   # clipped
+    s = check_parity(objs, kinds, recs, session_kw={"queue_capacity": (cap, 0)})
+    assert int(s.raw_counters()[5].item()) > 0, "the overflow path did not run"
+
+
+def test_range_queue_overflow_c1_and_tiny():
+    """The same fallback on generated traces (C1's memcpy/memset ranges and
+    tiny programs with ranges running past object ends), queue of one entry."""
+    p = build_config("C1")
+    check_parity(p.objects, p.kinds, gen_all_records(p), session_kw={"queue_capacity": (1, 0)})
+    for seed in range(6):
+        t = build_tiny(seed)
+        check_parity(t.objects, t.kinds, gen_all_records(t), session_kw={"queue_capacity": (1, 0)})
+
+
+# ---------------------------------------------------------------- CUDA graphs
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_cuda_graph_replay(name):
+    """bench.py times the step (reset, attribute, finalize) as a CUDA-graph
+    replay.  Capture it once and replay it three times: every replay must give
+    the oracle's results (the host-side call parity that selects the
+    range-queue counter slot is frozen into the graph, so consecutive replays
+    exercise both slots' reset logic)."""
+    p = build_config(name, **({"n_records": 1 << 24} if name == "C2" else {}))
+    r = gen_records(p, 0, p.n_records)
+    orc = Oracle(p.objects, p.kinds)
+    orc.attribute(r)
+    ost, octr = orc.stats()
+    orep = orc.patterns()
+    s = _session(p.objects, p.kinds)
+    d = torch.from_numpy(r.view(np.uint8)).cuda()
+    # C1: one attribute call per step (as bench.py); C2: two (both slots)
+    cuts = [0, p.n_records] if name == "C1" else [0, p.n_records // 2, p.n_records]
+
+    def step():
+        s.reset()
+        for a, b in zip(cuts, cuts[1:]):
+            s.attribute(d[16 * a: 16 * b])
+        s.finalize()
+
+    step()                      # warm-up outside the capture
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        step()
+    exp = None
+    for rep in range(3):
+        g.replay()
+        torch.cuda.synchronize()
+        st, ctr = s.object_stats()
+        rp = s.patterns()
+        for k in octr.dtype.names:
+            assert int(ctr[k]) == int(octr[k]), (rep, k)
+        for k in ost.dtype.names:
+            assert np.array_equal(st[k], ost[k]), (rep, k)
+        for k in orep.dtype.names:
+            assert np.array_equal(rp[k], orep[k]), (rep, k)
+        assert s.consistency_errors() == 0
+        orw = s.or_words().cpu().numpy().view(np.uint32).copy()
+        if exp is None:
+            exp = expected_or_words(s, orc, p.objects, p.kinds)
+        assert np.array_equal(orw, exp), rep

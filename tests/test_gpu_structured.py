@@ -11,9 +11,9 @@ from tracegen import build_config, build_tiny, gen_all_records  # noqa: E402
 from tests.golden_util import load, to_arrays  # noqa: E402
 
 
-def _gpu(objs, kinds, recs, chunks=1):
+def _gpu(objs, kinds, recs, chunks=1, queue_capacity=None):
     from paper_conf_asplos_linzs23_b200 import Session
-    s = Session(objs, kinds, structured=True)
+    s = Session(objs, kinds, structured=True, queue_capacity=queue_capacity)
     d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
     b = np.linspace(0, len(recs), chunks + 1).astype(np.int64)
     for x, y in zip(b, b[1:]):
@@ -27,8 +27,8 @@ def _oracle(objs, kinds, recs):
     return o.structured()
 
 
-def _check(objs, kinds, recs, chunks=1):
-    s, (sa, ov) = _gpu(objs, kinds, recs, chunks)
+def _check(objs, kinds, recs, chunks=1, queue_capacity=None):
+    s, (sa, ov) = _gpu(objs, kinds, recs, chunks, queue_capacity)
     osa, oov = _oracle(objs, kinds, recs)
     assert np.array_equal(sa, osa) and np.array_equal(ov, oov)
     return s, sa, ov
@@ -65,3 +65,13 @@ def test_reset_and_main_results_unchanged():
     assert np.array_equal(a.object_stats()[0], b.object_stats()[0])
     a.reset(); a.attribute(d)
     assert np.array_equal(a.structured()[0], _oracle(p.objects, p.kinds, r)[0])
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_wide_record_queue_overflow(seed):
+    """Wide records that do not fit the SA range queue (capacity 1) claim
+    their elements in place (attribute.cu structured_kernel's fallback)."""
+    p = build_tiny(seed)
+    _check(p.objects, p.kinds, gen_all_records(p), queue_capacity=(0, 1))
+    c = build_config("C1")
+    _check(c.objects, c.kinds, gen_all_records(c), queue_capacity=(0, 1))

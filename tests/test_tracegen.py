@@ -55,3 +55,33 @@ def test_generation_is_deterministic(seed):
     a, b = build_tiny(seed), build_tiny(seed)
     assert np.array_equal(a.objects, b.objects) and np.array_equal(a.kinds, b.kinds)
     assert np.array_equal(gen_all_records(a), gen_all_records(b))
+
+
+def test_object_sample_keeps_record_values():
+    """object_sample (the bounded CPU-oracle sample of bench.py) emits, for
+    the kept bursts, exactly the records the full program emits for them."""
+    from tracegen import object_sample
+    for name, kw in (("C1", {}), ("C5", {"n_records": 1 << 21})):
+        p = build_config(name, **kw)
+        full = gen_records(p, 0, p.n_records)
+        sub = object_sample(p, 7, 3)
+        got = gen_records(sub, 0, sub.n_records)
+        owner = np.repeat(np.arange(len(p.bursts)), p.bursts["count"].astype(np.int64))
+        keep = np.zeros(len(p.bursts), bool)
+        keep[sub.burst_id.astype(np.int64)] = True
+        assert np.array_equal(got, full[keep[owner]])
+        assert sub.n_obj == len(range(3, p.n_obj, 7))
+        assert np.array_equal(sub.objects, p.objects[3::7])
+
+
+def test_object_sample_oracle_results_equal_full_run():
+    """Dropping objects never changes which object a record belongs to (no two
+    objects overlap in address and lifetime, reading R5), so the oracle's
+    results for a kept object are the same in the sample and the full run."""
+    from oracle import run_oracle
+    from tracegen import object_sample
+    p = build_config("C1")
+    _, st, _, rep = run_oracle(p.objects, p.kinds, gen_records(p, 0, p.n_records))
+    sub = object_sample(p, 4, 1)
+    _, st2, _, rep2 = run_oracle(sub.objects, sub.kinds, gen_records(sub, 0, sub.n_records))
+    assert np.array_equal(st2, st[1::4]) and np.array_equal(rep2, rep[1::4])

@@ -14,12 +14,12 @@ recipe of each config is written out in DESIGN.md §"Input recipe".
 from .layout import (OBJ_DTYPE, REC_DTYPE, BURST_DTYPE, API_ALLOC, API_FREE,
                      API_MEMCPY, API_MEMSET, API_KERNEL, NEVER,
                      PAT_AFFINE, PAT_RANDOM, PAT_RANGE, PAT_RAW)
-from .program import Program, ProgramBuilder, build_config, build_tiny, CONFIGS
+from .program import Program, ProgramBuilder, build_config, build_tiny, object_sample, CONFIGS
 from .records import gen_records, gen_all_records
 
 __all__ = [
     "OBJ_DTYPE", "REC_DTYPE", "BURST_DTYPE", "API_ALLOC", "API_FREE",
     "API_MEMCPY", "API_MEMSET", "API_KERNEL", "NEVER", "PAT_AFFINE",
     "PAT_RANDOM", "PAT_RANGE", "PAT_RAW", "Program", "ProgramBuilder",
-    "build_config", "build_tiny", "CONFIGS", "gen_records", "gen_all_records",
+    "build_config", "build_tiny", "object_sample", "CONFIGS", "gen_records", "gen_all_records",
 ]

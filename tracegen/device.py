@@ -31,6 +31,8 @@ class DeviceProgram:
 
     def __init__(self, prog, device="cuda"):
         import torch
+        if prog.burst_id is not None:
+            raise ValueError("device generation needs a program's own bursts (not an object_sample)")
         self.prog = prog
         self.device = torch.device(device)
         self.bursts = torch.from_numpy(np.ascontiguousarray(prog.bursts).view(np.uint8)).to(self.device)

@@ -34,6 +34,9 @@ class Program:
     bursts: np.ndarray           # BURST_DTYPE[n_burst]
     prefix: np.ndarray           # u64[n_burst+1], record prefix counts
     meta: dict = field(default_factory=dict)
+    # burst ids for record(i)'s hash when the bursts are a subset of another
+    # program's (object_sample); None = the bursts' own indices
+    burst_id: np.ndarray = None
 
     @property
     def n_records(self):
@@ -559,6 +562,35 @@ def build_tiny(seed, n_obj_max=48, n_api_max=200, n_rec_max=4000, reuse=True):
 
 
 CONFIGS = {"C1": build_c1, "C2": build_c2}
+
+
+def object_sample(prog, k, offset=0):
+    """The sub-program of objects o with o % k == offset and every burst that
+    targets them (plus every k-th injected odd-record burst), over the SAME
+    timeline: a proportional 1/k slice of the workload, used to time the CPU
+    oracle on a bounded sample whose per-object fixed costs (bitmaps, scans)
+    scale with the records like the full trace's.  Records keep the values
+    they have in the full program (bursts keep their burst ids for the RANDOM
+    hash).  Host generation only (tracegen/gen.cu has no burst ids)."""
+    k = max(1, int(k))
+    n = prog.n_obj
+    keep_obj = (np.arange(n) % k) == offset
+    new_idx = np.full(n + 1, 0xFFFFFFFF, np.uint64)
+    new_idx[:n][keep_obj] = np.arange(int(keep_obj.sum()), dtype=np.uint64)
+    bo = prog.bursts["obj"].astype(np.int64)
+    is_obj = bo < n
+    bid_all = np.arange(len(prog.bursts), dtype=np.uint64) if prog.burst_id is None else prog.burst_id
+    keep_b = np.where(is_obj, keep_obj[np.minimum(bo, n - 1)], (bid_all % np.uint64(k)) == np.uint64(offset))
+    bursts = prog.bursts[keep_b].copy()
+    ob = bursts["obj"].astype(np.int64)
+    bursts["obj"] = np.where(ob < n, new_idx[np.minimum(ob, n)], bursts["obj"]).astype(np.uint32)
+    counts = bursts["count"].astype(np.uint64)
+    prefix = np.zeros(len(bursts) + 1, np.uint64)
+    np.cumsum(counts, out=prefix[1:])
+    objs = prog.objects[keep_obj].copy()
+    return Program(f"{prog.name}/objects%{k}=={offset}", prog.seed, objs, prog.kinds, bursts, prefix,
+                   dict(prog.meta, sample_of=prog.name, sample_k=k, sample_offset=offset),
+                   burst_id=bid_all[keep_b])
 
 
 def build_config(name, **kw):

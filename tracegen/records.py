@@ -48,7 +48,8 @@ def gen_records(prog, i0, i1, out=None):
         elem = start + (j * F["stride"][b]) % span
         rnd = pat == PAT_RANDOM
         if rnd.any():
-            h = splitmix64(np.uint64(prog.seed) ^ (b[rnd].astype(np.uint64) << np.uint64(32)) ^ j[rnd])
+            bid = b[rnd].astype(np.uint64) if prog.burst_id is None else prog.burst_id[b[rnd]]
+            h = splitmix64(np.uint64(prog.seed) ^ (bid << np.uint64(32)) ^ j[rnd])
             elem[rnd] = start[rnd] + h % span[rnd]
         base = F["base"][b]
         addr = base + elem * F["elem"][b].astype(np.uint64)
