@@ -84,7 +84,7 @@ def args_():
     ap.add_argument("--no-parity", action="store_true", help="skip the golden-digest check")
     ap.add_argument("--extra-configs", default="C4,C2",
                     help="comma list of configs measured after the main one at N=1 (key other_configs); '' = none")
-    ap.add_argument("--cpu-sample", type=int, default=30_000_000,
+    ap.add_argument("--cpu-sample", type=int, default=250_000_000,
                     help="target records of the oracle's timed sample (an object_sample of the workload)")
     ap.add_argument("--e2e-sample", type=int, default=1 << 28,
                     help="records per step of the host-buffer (e2e) leg")

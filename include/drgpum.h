@@ -350,6 +350,18 @@ DRGPUM_API drgpum_status drgpum_consistency_errors(drgpum_ctx *ctx,
 DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx *ctx, uint8_t *h_sa, uint8_t *h_overlap,
                                            void *stream);
 
+/* API group of the NEXT-2 / NEXT-3 analyses [R22b, R23]: h_in_group[t] != 0
+ * puts the GPU API at timestamp t in the group (NULL = every API, the
+ * default after workspace_bind).  The paper reports structured access "at GPU
+ * kernel gramschmidt_kernel3" (l.400): the group is then the invocations of
+ * that kernel.  The structured-access pass of the following trace_attribute
+ * calls only considers records of APIs in the group (set it before
+ * attributing a trace); drgpum_structured counts the group's accessing APIs;
+ * drgpum_slice_frequency uses the group at query time.  Synchronous (the
+ * host array is consumed).  ESTATE before workspace_bind or without one of
+ * the two features. */
+DRGPUM_API drgpum_status drgpum_set_api_group(drgpum_ctx *ctx, const uint8_t *h_in_group, void *stream);
+
 /* NEXT-2 results (synchronous; ESTATE unless DRGPUM_FEATURE_FREQUENCY, EINVAL
  * if the records were not in timestamp order).  For every (object O, access
  * API A in O's lifetime): n = elements A touched, S1 = sum of their access
@@ -364,6 +376,19 @@ DRGPUM_API drgpum_status drgpum_frequency(drgpum_ctx *ctx, uint32_t pct, uint32_
                                           uint32_t *h_first, void *stream);
 DRGPUM_API drgpum_status drgpum_frequency_slots(drgpum_ctx *ctx, uint64_t *h_acc,
                                                 uint64_t *n_slots, void *stream);
+
+/* Slice-level non-uniform access frequency [R22b] (Def 3.9 l.196 at the
+ * granularity of §7.3 l.400, "the variance of access frequencies of
+ * individual slices in R_gpu is 58%"): for object O, each API A of the group
+ * (drgpum_set_api_group) that accesses O touches a slice of O whose access
+ * frequency is F_A = S1 of slot (O, A) (the sum of its elements' counts).  O
+ * matches iff the population coefficient of variation of {F_A} exceeds pct%,
+ * exactly (n*S2 - S1^2) * 100^2 > pct^2 * S1^2 with n = number of such APIs,
+ * S1 = sum F_A, S2 = sum F_A^2.  h_match u8[n_obj]; h_moments u64[4*n_obj] =
+ * {n, S1, S2 low 64 bits, S2 high 64 bits} per object.  Either may be NULL.
+ * Synchronous; errors as drgpum_frequency. */
+DRGPUM_API drgpum_status drgpum_slice_frequency(drgpum_ctx *ctx, uint32_t pct, uint8_t *h_match,
+                                                uint64_t *h_moments, void *stream);
 
 /* Diagnostics (not part of the method): how many 32-record tiles took each
  * attribution path since the last reset -- out[0] affine run with one union

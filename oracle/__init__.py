@@ -57,6 +57,8 @@ def _load():
         L.oracle_get_accesses.restype = U64
         L.oracle_track_structured.argtypes = [P]
         L.oracle_structured.argtypes = [P, P, P]
+        L.oracle_structured_group.argtypes = [P, P, P, P]
+        L.oracle_slice_frequency.argtypes = [P, P, P]
         L.oracle_track_frequency.argtypes = [P]
         L.oracle_frequency.argtypes = [P, P, P, P, P, P, U64]
         L.oracle_frequency.restype = U64
@@ -119,13 +121,26 @@ class Oracle:
         _load().oracle_patterns(self._h, _ptr(th), _ptr(out))
         return out
 
-    def structured(self):
-        """NEXT-3: (sa u8[n_obj], overlap u8[n_obj]); needs structured=True."""
+    def structured(self, group=None):
+        """NEXT-3: (sa u8[n_obj], overlap u8[n_obj]) over the APIs t with
+        group[t] != 0 (None = all APIs) [R23]; needs structured=True."""
         n = self.objects.shape[0]
         sa = np.zeros(n, np.uint8)
         ov = np.zeros(n, np.uint8)
-        _load().oracle_structured(self._h, _ptr(sa), _ptr(ov))
+        g = None if group is None else np.ascontiguousarray(group, dtype=np.uint8)
+        _load().oracle_structured_group(self._h, None if g is None else _ptr(g), _ptr(sa), _ptr(ov))
         return sa, ov
+
+    def slice_frequency(self, group=None):
+        """Slice-level NUAF moments [R22b] over the APIs t with group[t] != 0:
+        per object (n, sum F, sum F^2) as Python ints, F = total access
+        frequency of one API's slice; needs frequency=True."""
+        n = self.objects.shape[0]
+        out = np.zeros(4 * n, np.uint64)
+        g = None if group is None else np.ascontiguousarray(group, dtype=np.uint8)
+        _load().oracle_slice_frequency(self._h, None if g is None else _ptr(g), _ptr(out))
+        q = out.reshape(n, 4)
+        return [(int(a), int(b), int(c) | (int(d) << 64)) for a, b, c, d in q]
 
     def frequency(self):
         """NEXT-2 rows (obj, ts, n, s1, s2) in (object, ts) order; needs frequency=True."""

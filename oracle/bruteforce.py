@@ -140,11 +140,12 @@ def validate(objects, kinds):
     return 0
 
 
-def bruteforce_structured(objects, kinds, records):
+def bruteforce_structured(objects, kinds, records, group=None):
     """NEXT-3 structured access by definition (Def 3.10, l.200): per object,
     the set of elements each accessing GPU API touches; SA iff at least two
-    APIs access O and their slices are pairwise disjoint.  Returns (sa, overlap)
-    lists of 0/1."""
+    APIs access O and their slices are pairwise disjoint.  Only the APIs t
+    with group[t] count (None = all) [R23].  Returns (sa, overlap) lists of
+    0/1."""
     n_api = len(kinds)
     objs = [dict(base=int(o["base"]), size=int(o["size"]), E=int(o["elem_size"]),
                  ta=int(o["t_alloc"]), tf=int(o["t_free"])) for o in objects]
@@ -164,7 +165,7 @@ def bruteforce_structured(objects, kinds, records):
                 break
     sa, ov = [], []
     for sl in slices:
-        sets = list(sl.values())
+        sets = [v for t, v in sl.items() if group is None or group[t]]
         overlap = any(sets[a] & sets[b] for a in range(len(sets)) for b in range(a + 1, len(sets)))
         ov.append(int(overlap))
         sa.append(int(len(sets) >= 2 and not overlap))
@@ -198,3 +199,18 @@ def bruteforce_frequency(objects, kinds, records):
         f = list(hm[(i, ts)].values())
         rows.append((i, ts, len(f), sum(f), sum(c * c for c in f)))
     return rows
+
+
+def bruteforce_slice_frequency(objects, kinds, records, group=None):
+    """Slice-level NUAF [R22b] by definition: for every object, over the APIs
+    t with group[t] (None = all) that access it, F_t = number of (record,
+    element) touches of t on the object (byte-wise expansion, an element
+    counted once per record); returns per object (n, sum F, sum F^2)."""
+    rows = bruteforce_frequency(objects, kinds, records)
+    out = [[0, 0, 0] for _ in objects]
+    for (i, ts, n, s1, s2) in rows:
+        if group is None or group[ts]:
+            out[i][0] += 1
+            out[i][1] += s1
+            out[i][2] += s1 * s1
+    return [tuple(x) for x in out]

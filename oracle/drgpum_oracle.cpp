@@ -33,6 +33,7 @@
 #include <cstdint>
 #include <cstring>
 #include <map>
+#include <set>
 #include <vector>
 #include <algorithm>
 
@@ -68,10 +69,10 @@ struct State {
   std::vector<std::map<uint32_t, Flags>> accesses;  // APIs that access O, by T
   Counters ctr;
   std::vector<std::vector<uint32_t>> alloc_at, free_at;   // per timestamp
-  // NEXT-3 structured access (Def 3.10): per object, element -> the GPU API
-  // that touched it, and whether any element was touched by two APIs
-  std::vector<std::map<uint64_t, uint32_t>> elem_api;
-  std::vector<uint8_t> overlap;
+  // NEXT-3 structured access (Def 3.10; §5.2 l.270 "multiple bitmaps for a
+  // data object, where each bitmap represents memory accesses of a GPU API"):
+  // per (object, API) the set of elements that API touched
+  std::map<std::pair<uint32_t, uint32_t>, std::set<uint64_t>> api_elems;
   bool track_sa = false;
   // NEXT-2 non-uniform access frequency (Def 3.9, l.271): per (object, API)
   // the "hashmap" of element -> access frequency of that API
@@ -158,8 +159,7 @@ void oracle_free(void* p) { delete static_cast<State*>(p); }
 void oracle_track_structured(void* p) {
   State& s = *static_cast<State*>(p);
   s.track_sa = true;
-  s.elem_api.assign(s.objs.size(), {});
-  s.overlap.assign(s.objs.size(), 0);
+  s.api_elems.clear();
 }
 
 // NEXT-2: keep, per (object, GPU API), the access frequency of every element
@@ -194,13 +194,58 @@ uint64_t oracle_frequency(void* p, uint32_t* obj, uint32_t* ts, uint64_t* n, uin
 
 // NEXT-3 structured access (Def 3.10, l.200; §5.2 l.270): object O matches if
 // each GPU API that accesses it touches a slice of O and the slices do not
-// overlap -- at least two accessing APIs and no element touched by two of
-// them.  out[o] = 1 if O matches; overlap[o] = 1 if two APIs share an element.
-void oracle_structured(void* p, uint8_t* out, uint8_t* overlap) {
+// overlap -- the per-API bitmaps of O are pairwise disjoint, and at least two
+// APIs access O.  [R23] The APIs considered are those with in_group[t] != 0
+// (NULL = every API): the paper reports the pattern "at GPU kernel
+// gramschmidt_kernel3" (l.400), i.e. over the invocations of one kernel.
+// out[o] = 1 if O matches; overlap[o] = 1 if two of those APIs share an element.
+void oracle_structured_group(void* p, const uint8_t* in_group, uint8_t* out, uint8_t* overlap) {
   State& s = *static_cast<State*>(p);
-  for (size_t o = 0; o < s.objs.size(); ++o) {
-    overlap[o] = s.overlap[o];
-    out[o] = (s.accesses[o].size() >= 2 && !s.overlap[o]) ? 1 : 0;
+  const size_t n = s.objs.size();
+  std::vector<uint64_t> n_api(n, 0), sum(n, 0);
+  std::vector<std::set<uint64_t>> uni(n);
+  for (const auto& kv : s.api_elems) {
+    const uint32_t o = kv.first.first, t = kv.first.second;
+    if (in_group && !in_group[t]) continue;
+    n_api[o]++;
+    sum[o] += kv.second.size();
+    uni[o].insert(kv.second.begin(), kv.second.end());
+  }
+  for (size_t o = 0; o < n; ++o) {
+    const bool ov = uni[o].size() < sum[o];      // some element is in two APIs' bitmaps
+    overlap[o] = ov ? 1 : 0;
+    out[o] = (n_api[o] >= 2 && !ov) ? 1 : 0;
+  }
+}
+
+void oracle_structured(void* p, uint8_t* out, uint8_t* overlap) {
+  oracle_structured_group(p, nullptr, out, overlap);
+}
+
+// Slice-level access frequency (Def 3.9 l.196 read at the granularity of
+// l.400: "the variance of access frequencies of individual slices in R_gpu is
+// 58%") [R22b]: for object O and the APIs with in_group[t] != 0, the access
+// frequency of API A's slice is F_A = the sum of the element frequencies of
+// A's hashmap for O (l.271).  out[4o..4o+3] = { n = number of such APIs that
+// access O, sum F_A, and sum F_A^2 as (low 64 bits, high 64 bits) }.  Needs
+// oracle_track_frequency.
+void oracle_slice_frequency(void* p, const uint8_t* in_group, uint64_t* out) {
+  State& s = *static_cast<State*>(p);
+  const size_t n = s.objs.size();
+  std::vector<unsigned __int128> s2(n, 0);
+  for (size_t o = 0; o < n; ++o) out[4 * o] = out[4 * o + 1] = 0;
+  for (const auto& kv : s.freq) {
+    const uint32_t o = kv.first.first, t = kv.first.second;
+    if (in_group && !in_group[t]) continue;
+    uint64_t F = 0;
+    for (const auto& ec : kv.second) F += ec.second;
+    out[4 * o] += 1;
+    out[4 * o + 1] += F;
+    s2[o] += (unsigned __int128)F * F;
+  }
+  for (size_t o = 0; o < n; ++o) {
+    out[4 * o + 2] = (uint64_t)s2[o];
+    out[4 * o + 3] = (uint64_t)(s2[o] >> 64);
   }
 }
 
@@ -261,11 +306,9 @@ void oracle_attribute(void* p, const Rec* recs, uint64_t n) {
         auto& hm = s.freq[{o, t}];
         for (uint64_t e = e0; e <= e1; ++e) hm[e] += 1;
       }
-      if (s.track_sa) {                                               // Def 3.10
-        for (uint64_t e = e0; e <= e1; ++e) {
-          auto ins = s.elem_api[o].emplace(e, t);
-          if (!ins.second && ins.first->second != t) s.overlap[o] = 1;
-        }
+      if (s.track_sa) {                                               // l.270
+        auto& bm = s.api_elems[{o, t}];
+        for (uint64_t e = e0; e <= e1; ++e) bm.insert(e);
       }
       if (t < s.first[o]) s.first[o] = t;
       if (t > s.last[o]) s.last[o] = t;

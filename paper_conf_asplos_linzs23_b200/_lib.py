@@ -60,7 +60,7 @@ class DrgpumError(RuntimeError):
         self.status = status
 
 
-EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_set_features", "drgpum_set_queue_capacity", "drgpum_structured",
+EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_set_features", "drgpum_set_queue_capacity", "drgpum_set_api_group", "drgpum_slice_frequency", "drgpum_structured",
            "drgpum_frequency", "drgpum_frequency_slots",
            "drgpum_workspace_size",
            "drgpum_workspace_bind", "drgpum_reset", "drgpum_trace_attribute",
@@ -106,6 +106,8 @@ def load():
         "drgpum_path_stats": ([P, P, P], I),
         "drgpum_set_features": ([P, U32], I),
         "drgpum_set_queue_capacity": ([P, U32, U32], I),
+        "drgpum_set_api_group": ([P, P, P], I),
+        "drgpum_slice_frequency": ([P, U32, P, P, P], I),
         "drgpum_structured": ([P, P, P, P], I),
         "drgpum_frequency": ([P, U32, P, P, P], I),
         "drgpum_frequency_slots": ([P, P, ctypes.POINTER(U64), P], I),

@@ -1113,7 +1113,7 @@ __global__ void __launch_bounds__(256) structured_kernel(const __grid_constant__
     const uint32_t size = r.z, ts = r.w & 0x7FFFFFFFu;
     if (size == 0 || ts >= p.n_api || addr > ~0ull - size) continue;
     const uint32_t rank = __ldg(p.acc_rank + ts);
-    if (rank == kNone) continue;
+    if (rank == kNone || !__ldg(q.in_group + ts)) continue;
     if (!(addr - c_base < c_size && ts > c_ta && ts < c_tf)) {
       const uint32_t o = find_object(p, p.l1, addr, ts);   // level-1 keys from global here
       if (o == kNone) continue;

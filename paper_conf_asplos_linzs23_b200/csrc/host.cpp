@@ -38,7 +38,7 @@ struct Layout {
   uint64_t rfull;                 // per object: a whole-object range was queued in this trace
   uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage;
   // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
-  uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end;
+  uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end, sa_group;
   // NEXT-2 frequency (feature): cells[sum n_elem], acc[n_slots][3], state, queue, outputs
   uint64_t fq_cells, fq_acc, fq_state, fq_q, fq_end, fq_slot_base, fq_out_count, fq_out_first;
   uint64_t fq_ctl, fq_run_start, fq_segs, fq_seg_of_ts, fq_seg_touch, fq_seg_off, fq_seg_logcap, fq_solo;
@@ -84,6 +84,7 @@ struct drgpum_ctx {
   std::vector<uint64_t> elem_base, slot_base;
   uint64_t n_elem_total = 0, n_slots = 0;
   uint32_t sa_q_cap = 1u << 20;
+  std::vector<uint8_t> api_group;   // NEXT-2/3 API group [R22b, R23] (1 = in), mirrored in the workspace
   Layout L{};
   uint8_t* ws = nullptr;
   uint64_t ws_bytes = 0;
@@ -138,6 +139,8 @@ drgpum_status set_device(drgpum_ctx* ctx) {
 uint32_t ilog2(uint32_t e) { uint32_t s = 0; while ((1u << s) < e) ++s; return s; }
 
 drgpum_status compute_layout(drgpum_ctx* c);
+drgpum_status gather_accesses(drgpum_ctx* ctx, cudaStream_t st, std::vector<uint64_t>& off,
+                              std::vector<uint32_t>& api, std::vector<uint8_t>& rw);
 
 // NEXT-2 per-API hash tables: entries per batch (power of two).  Small
 // enough that a batch's tables stay resident in L2 (random atomics on
@@ -338,9 +341,11 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   L.reports = put(sizeof(drgpum_pattern_report_t) * n);
   L.rq = put(sizeof(RangeEntry) * c->rq_cap);
   L.stage = put(2 * kStageRecords * sizeof(drgpum_record_t));
-  L.sa_owner = L.sa_overlap = L.sa_elem_base = L.sa_q = L.sa_qcount = L.sa_end = off;
-  if (c->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY))
+  L.sa_owner = L.sa_overlap = L.sa_elem_base = L.sa_q = L.sa_qcount = L.sa_end = L.sa_group = off;
+  if (c->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY)) {
     L.sa_elem_base = put(8 * n);              // shared by both features
+    L.sa_group = put(n_api);                  // API group of the SA pass [R23] (1 = in)
+  }
   if (c->features & DRGPUM_FEATURE_STRUCTURED) {
     L.sa_owner = put(4 * c->n_elem_total);
     L.sa_overlap = put(4 * n);
@@ -482,6 +487,7 @@ SaParams sa_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   q.q = at<SaRange>(c, c->L.sa_q);
   q.q_cap = c->sa_q_cap;
   q.q_count = at<unsigned long long>(c, c->L.sa_qcount);
+  q.in_group = at<uint8_t>(c, c->L.sa_group);
   return q;
 }
 
@@ -562,18 +568,48 @@ DRGPUM_API drgpum_status drgpum_structured(drgpum_ctx* ctx, uint8_t* h_sa, uint8
   if (drgpum_status _d = set_device(ctx)) return _d;
   if (!(ctx->features & DRGPUM_FEATURE_STRUCTURED))
     return fail(ctx, DRGPUM_ESTATE, "DRGPUM_FEATURE_STRUCTURED was not enabled");
-  std::vector<drgpum_object_stats_t> st(ctx->n_obj);
-  drgpum_status s = drgpum_object_stats(ctx, st.data(), nullptr, stream);
-  if (s != DRGPUM_OK) return s;
-  std::vector<uint32_t> ov(ctx->n_obj);
   cudaStream_t strm = as_stream(stream);
+  // accessing APIs of the group per object [R23]: the finalized n_access_apis
+  // when the group is every API, else counted on the hit rows
+  std::vector<uint64_t> n_in(ctx->n_obj, 0);
+  const bool all = std::all_of(ctx->api_group.begin(), ctx->api_group.end(), [](uint8_t g) { return g != 0; });
+  if (all) {
+    std::vector<drgpum_object_stats_t> st(ctx->n_obj);
+    drgpum_status s = drgpum_object_stats(ctx, st.data(), nullptr, stream);
+    if (s != DRGPUM_OK) return s;
+    for (uint64_t o = 0; o < ctx->n_obj; ++o) n_in[o] = st[o].n_access_apis;
+  } else {
+    std::vector<uint64_t> off;
+    std::vector<uint32_t> api;
+    std::vector<uint8_t> rw;
+    drgpum_status s = gather_accesses(ctx, strm, off, api, rw);
+    if (s != DRGPUM_OK) return s;
+    for (uint64_t o = 0; o < ctx->n_obj; ++o)
+      for (uint64_t k = off[o]; k < off[o + 1]; ++k) n_in[o] += ctx->api_group[api[k]] ? 1 : 0;
+  }
+  std::vector<uint32_t> ov(ctx->n_obj);
   if (ctx->n_obj) {
     CK(cudaMemcpyAsync(ov.data(), ctx->ws + ctx->L.sa_overlap, 4 * ctx->n_obj, cudaMemcpyDeviceToHost, strm));
     CK(cudaStreamSynchronize(strm));
   }
   for (uint64_t o = 0; o < ctx->n_obj; ++o) {
     if (h_overlap) h_overlap[o] = ov[o] ? 1 : 0;
-    if (h_sa) h_sa[o] = (st[o].n_access_apis >= 2 && !ov[o]) ? 1 : 0;
+    if (h_sa) h_sa[o] = (n_in[o] >= 2 && !ov[o]) ? 1 : 0;
+  }
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_set_api_group(drgpum_ctx* ctx, const uint8_t* h_in_group, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "set_api_group before workspace_bind");
+  if (drgpum_status _d = set_device(ctx)) return _d;
+  if (!(ctx->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY)))
+    return fail(ctx, DRGPUM_ESTATE, "set_api_group needs DRGPUM_FEATURE_STRUCTURED or _FREQUENCY");
+  for (uint32_t t = 0; t < ctx->n_api; ++t) ctx->api_group[t] = h_in_group ? (h_in_group[t] ? 1 : 0) : 1;
+  cudaStream_t st = as_stream(stream);
+  if (ctx->n_api) {
+    CK(cudaMemcpyAsync(ctx->ws + ctx->L.sa_group, ctx->api_group.data(), ctx->n_api, cudaMemcpyHostToDevice, st));
+    CK(cudaStreamSynchronize(st));   // the host copy may change with the next call
   }
   return DRGPUM_OK;
 }
@@ -631,6 +667,43 @@ DRGPUM_API drgpum_status drgpum_frequency_slots(drgpum_ctx* ctx, uint64_t* h_acc
   return DRGPUM_OK;
 }
 
+DRGPUM_API drgpum_status drgpum_slice_frequency(drgpum_ctx* ctx, uint32_t pct, uint8_t* h_match,
+                                                uint64_t* h_moments, void* stream) {
+  if (!ctx) return DRGPUM_EINVAL;
+  cudaStream_t st = as_stream(stream);
+  drgpum_status r = frequency_ready(ctx, st);
+  if (r != DRGPUM_OK) return r;
+  std::vector<uint64_t> acc(3 * ctx->n_slots);
+  if (ctx->n_slots) {
+    CK(cudaMemcpyAsync(acc.data(), ctx->ws + ctx->L.fq_acc, 24 * ctx->n_slots, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  // [R22b] per object: over the group's accessing APIs A, F_A = S1 of slot
+  // (O, A); CV of {F_A} > pct% iff (n*S2 - S1^2) * 100^2 > pct^2 * S1^2
+  uint64_t slot = 0;
+  for (uint64_t o = 0; o < ctx->n_obj; ++o) {
+    const auto& l = ctx->layout[o];
+    uint64_t n = 0, s1 = 0;
+    unsigned __int128 s2 = 0;
+    for (uint32_t k = 0; k < l.n_hit_apis; ++k, ++slot) {
+      const uint64_t F = acc[3 * slot + 1];
+      if (!acc[3 * slot] || !ctx->api_group[ctx->acc_ts[l.r_lo + k]]) continue;
+      ++n;
+      s1 += F;
+      s2 += (unsigned __int128)F * F;
+    }
+    const unsigned __int128 S1 = s1, var = (unsigned __int128)n * s2 - S1 * S1;
+    if (h_match) h_match[o] = (s1 > 0 && var * 10000 > (unsigned __int128)pct * pct * S1 * S1) ? 1 : 0;
+    if (h_moments) {
+      h_moments[4 * o] = n;
+      h_moments[4 * o + 1] = s1;
+      h_moments[4 * o + 2] = (uint64_t)s2;
+      h_moments[4 * o + 3] = (uint64_t)(s2 >> 64);
+    }
+  }
+  return DRGPUM_OK;
+}
+
 DRGPUM_API drgpum_status drgpum_workspace_size(const drgpum_ctx* ctx, uint64_t* bytes) {
   if (!ctx || !bytes) return DRGPUM_EINVAL;
   if (ctx->state < S_LOADED) return DRGPUM_ESTATE;
@@ -676,8 +749,11 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
   if ((r = up(L.tiles, ctx->tiles.data(), sizeof(Tile) * ctx->tiles.size()))) return r;
   if ((r = up(L.groups, ctx->groups.data(), sizeof(Group) * ctx->groups.size()))) return r;
   if ((r = up(L.group_off, ctx->group_off.data(), 4 * ctx->group_off.size()))) return r;
-  if (ctx->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY))
+  if (ctx->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY)) {
     if ((r = up(L.sa_elem_base, ctx->elem_base.data(), 8 * n))) return r;
+    ctx->api_group.assign(ctx->n_api, 1);
+    if ((r = up(L.sa_group, ctx->api_group.data(), ctx->n_api))) return r;
+  }
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
     if ((r = up(L.fq_slot_base, ctx->slot_base.data(), 8 * n))) return r;
   if ((r = enqueue_reset(ctx, st))) return r;

@@ -95,6 +95,7 @@ struct SaParams {
   SaRange* q;                // large-range queue
   uint32_t q_cap;
   unsigned long long* q_count;
+  const uint8_t* in_group;   // [n_api] 1 = the API takes part in the pass [R23]
 };
 
 // NEXT-2 non-uniform access frequency pass (optional feature).

@@ -178,8 +178,29 @@ class Session:
         check(self._h, self.L.drgpum_path_stats(self._h, _np_ptr(out), _stream_handle(stream)))
         return dict(zip(("affine_union", "affine_words", "tile_fast", "slow"), (int(x) for x in out)))
 
+    def set_api_group(self, in_group=None, stream=None):
+        """drgpum_set_api_group: u8[n_api] mask of the APIs the NEXT-2/3
+        analyses consider (None = all) [R22b, R23]; set before attributing
+        for the structured-access pass."""
+        g = None if in_group is None else np.ascontiguousarray(in_group, dtype=np.uint8)
+        if g is not None and g.shape[0] != self.n_api:
+            raise ValueError("in_group needs one entry per API")
+        check(self._h, self.L.drgpum_set_api_group(self._h, None if g is None else _np_ptr(g),
+                                                   _stream_handle(stream)))
+
+    def slice_frequency(self, pct=20, stream=None):
+        """Slice-level NUAF [R22b]: (match u8[n_obj], moments list of
+        (n, S1, S2) Python ints) over the API group; needs frequency=True."""
+        m = np.zeros(self.n_obj, np.uint8)
+        mo = np.zeros(4 * self.n_obj, np.uint64)
+        check(self._h, self.L.drgpum_slice_frequency(self._h, pct, _np_ptr(m), _np_ptr(mo),
+                                                     _stream_handle(stream)))
+        q = mo.reshape(self.n_obj, 4)
+        return m, [(int(a), int(b), int(c) | (int(d) << 64)) for a, b, c, d in q]
+
     def structured(self, stream=None):
-        """NEXT-3: (sa u8[n_obj], overlap u8[n_obj]); needs structured=True."""
+        """NEXT-3: (sa u8[n_obj], overlap u8[n_obj]) over the API group
+        (set_api_group); needs structured=True."""
         sa = np.zeros(self.n_obj, np.uint8)
         ov = np.zeros(self.n_obj, np.uint8)
         check(self._h, self.L.drgpum_structured(self._h, _np_ptr(sa), _np_ptr(ov), _stream_handle(stream)))

@@ -75,3 +75,51 @@ def test_wide_record_queue_overflow(seed):
     _check(p.objects, p.kinds, gen_all_records(p), queue_capacity=(0, 1))
     c = build_config("C1")
     _check(c.objects, c.kinds, gen_all_records(c), queue_capacity=(0, 1))
+
+
+def _grouped(objs, kinds, recs, group):
+    """GPU (structured + frequency, API group set before attributing) vs O1."""
+    from paper_conf_asplos_linzs23_b200 import Session
+    recs = recs[np.argsort(recs["meta"] & 0x7FFFFFFF, kind="stable")]     # NUAF needs API order
+    s = Session(objs, kinds, structured=True, frequency=True)
+    s.set_api_group(group)
+    s.attribute(torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda())
+    sa, ov = s.structured()
+    m, mom = s.slice_frequency(20)
+    o = Oracle(objs, kinds, structured=True, frequency=True)
+    o.attribute(recs)
+    osa, oov = o.structured(group)
+    assert np.array_equal(sa, osa) and np.array_equal(ov, oov)
+    omom = o.slice_frequency(group)
+    assert mom == omom
+    from oracle import nuaf_cv_exceeds
+    assert m.tolist() == [int(nuaf_cv_exceeds(a, b, c, 20)) for a, b, c in omom]
+    return sa, mom
+
+
+def test_gramschmidt_polybench_grouped():
+    """§7.3 l.400: R_gpu is structured AT gramschmidt_kernel3 and its slices'
+    access-frequency CV prints as 58% -- on the GPU, equal to the oracle."""
+    from fractions import Fraction
+    from tests.golden_util import gramschmidt_polybench
+    fx = load("gramschmidt_polybench")
+    objs, kinds, recs, k3, _ = gramschmidt_polybench(fx)
+    sa, ((n, s1, s2),) = _grouped(objs, kinds, recs, k3)
+    assert sa[0] == 1
+    cv2 = Fraction(n * s2 - s1 * s1, s1 * s1)
+    assert Fraction(575, 1000) ** 2 <= cv2 < Fraction(585, 1000) ** 2
+    sa_all, _ = _grouped(objs, kinds, recs, None)
+    assert sa_all[0] == 0
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_groups_tiny(seed):
+    p = build_tiny(7800 + seed)
+    g = (np.random.default_rng(seed).random(p.n_api) < 0.5).astype(np.uint8)
+    _grouped(p.objects, p.kinds, gen_all_records(p), g)
+
+
+def test_random_groups_c1():
+    p = build_config("C1")
+    g = (np.random.default_rng(5).random(p.n_api) < 0.3).astype(np.uint8)
+    _grouped(p.objects, p.kinds, gen_all_records(p), g)
