@@ -12,6 +12,9 @@ SEL="tests/test_gpu_parity.py::test_golden_fixtures tests/test_gpu_parity.py::te
  tests/test_gpu_parity.py::test_c1_full tests/test_gpu_parity.py::test_c1_host_ingest \
  tests/test_gpu_parity.py::test_empty_and_degenerate tests/test_gpu_parity.py::test_max_range_record \
  tests/test_gpu_parity.py::test_uint32_size_boundary tests/test_gpu_parity.py::test_range_queue_overflow \
+ tests/test_gpu_parity.py::test_range_queue_overflow_c1_and_tiny tests/test_gpu_parity.py::test_cuda_graph_replay \
+ tests/test_gpu_merge_peers.py::test_owned_state_rules tests/test_gpu_structured.py::test_random_groups_tiny \
+ tests/test_gpu_structured.py::test_gramschmidt_polybench_grouped tests/test_gpu_frequency.py::test_wide_record_queue_overflow \
  tests/test_gpu_merge_peers.py::test_virtual_peers_c1 tests/test_gpu_merge_peers.py::test_virtual_peers_owned_c1 \
  tests/test_gpu_merge_peers.py::test_virtual_peers_owned_tiny_reuse \
  tests/test_gpu_frequency.py::test_tiny tests/test_gpu_frequency.py::test_dependency_chain \
@@ -20,7 +23,7 @@ SEL="tests/test_gpu_parity.py::test_golden_fixtures tests/test_gpu_parity.py::te
 for tool in memcheck racecheck synccheck; do
   extra=""
   [ $tool = memcheck ] && extra="--leak-check no"
-  timeout 2400 $CS --tool $tool $extra --print-limit 200 --target-processes all \
+  timeout 1500 $CS --tool $tool $extra --print-limit 200 --target-processes all \
       --kernel-name-exclude regex:"^(at::|void at::|cub|void cub|elementwise|vectorized|reduce_kernel|unrolled)" \
       python -m pytest $SEL -q -p no:cacheprovider > $OUT/$tool.log 2>&1
   echo "$tool rc=$?" | tee -a $OUT/summary.txt
