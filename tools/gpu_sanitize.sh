@@ -24,7 +24,7 @@ for tool in memcheck racecheck synccheck; do
   extra=""
   [ $tool = memcheck ] && extra="--leak-check no"
   timeout 1500 $CS --tool $tool $extra --print-limit 200 --target-processes all \
-      --kernel-name-exclude regex:"^(at::|void at::|cub|void cub|elementwise|vectorized|reduce_kernel|unrolled)" \
+      --kernel-name regex=drgpum \
       python -m pytest $SEL -q -p no:cacheprovider > $OUT/$tool.log 2>&1
   echo "$tool rc=$?" | tee -a $OUT/summary.txt
   grep -E "ERROR SUMMARY|RACECHECK SUMMARY|passed|failed" $OUT/$tool.log | tail -4 | tee -a $OUT/summary.txt
