@@ -731,7 +731,7 @@ def main():
     w.close()
     if world == 1 and a.extra_configs:
         line["other_configs"] = {}
-        for cfg in [c for c in a.extra_configs.split(",") if c and c != a.config]:
+        for cfg in [c for c in a.extra_configs.split(",") if c in WORKLOADS and c != a.config]:
             try:
                 line["other_configs"][cfg] = other_config(cfg, a, hbm, hbm_src)
             except Exception as e:   # noqa: BLE001 -- an extra must not lose the main line

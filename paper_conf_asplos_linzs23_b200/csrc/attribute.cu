@@ -291,6 +291,11 @@ constexpr uint32_t kScratchWords = DRGPUM_SCRATCH;
 #ifndef DRGPUM_WINDOW
 #define DRGPUM_WINDOW 1
 #endif
+// Small objects' contiguous unions (affine tier) and chained tiles also go
+// through the scratch (A/B macro).
+#ifndef DRGPUM_UNION_SCRATCH
+#define DRGPUM_UNION_SCRATCH 1
+#endif
 constexpr uint64_t kNoScratch = ~0ull;
 
 struct alignas(16) WarpSmem {
@@ -595,6 +600,7 @@ __device__ __forceinline__ void scratch_bind(uint32_t wsm, uint32_t* orw, uint64
   const uint64_t cur = lds64(wsm + kOffScBase);
   if (cur == bm_word) return;   // warp-uniform
   if (cur != kNoScratch) scratch_flush(wsm, orw, cur, lane);
+  else __syncwarp();            // every lane has read cur before lane 0 overwrites it
   if (lane == 0) sts64(wsm + kOffScBase, bm_word);
   __syncwarp();
 }
@@ -634,6 +640,11 @@ __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_
 __device__ __forceinline__ void fast_or_c(uint32_t wsm, uint32_t* orw, const FastCache& c, uint32_t e0,
                                           uint32_t e1, int lane) {
   if (scratch_ok(c)) {
+#if DRGPUM_UNION_SCRATCH
+    scratch_bind(wsm, orw, c.bm_word, lane);   // chained or not: the scratch
+    scratch_record(wsm, e0, e1);
+    return;
+#else
     const uint32_t pe0 = __shfl_up_sync(FULL_MASK, e0, 1);
     const uint32_t pe1 = __shfl_up_sync(FULL_MASK, e1, 1);
     const bool chain = lane == 0 || (e0 >= pe0 && e0 <= pe1 + 1 && e1 >= pe1);
@@ -642,6 +653,7 @@ __device__ __forceinline__ void fast_or_c(uint32_t wsm, uint32_t* orw, const Fas
       scratch_record(wsm, e0, e1);
       return;
     }
+#endif
   }
 #if DRGPUM_WINDOW
   else {   // a large object's irregular tile within < 64 words: scratch window
@@ -705,6 +717,21 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
   if (st32 <= sz || st32 <= (1u << c.shift)) {
     const uint32_t lo = o0 >> c.shift, hi = uint32_t(off_end - 1) >> c.shift;
     const uint32_t wlo = lo >> 5, nw = (hi >> 5) - wlo;
+#if DRGPUM_UNION_SCRATCH
+    // a small object's union goes to the scratch: a sweep that wraps around
+    // the object (C5's 8 KiB objects, C3's activations) re-ORs the same
+    // words every pass, in shared memory instead of as global RED sectors
+    if (scratch_ok(c)) {
+      scratch_bind(wsm, orw, c.bm_word, lane);
+      for (uint32_t w = lane; w <= nw; w += 32) {
+        uint32_t m = 0xFFFFFFFFu;
+        if (w == 0) m &= 0xFFFFFFFFu << (lo & 31);
+        if (w == nw) m &= 0xFFFFFFFFu >> (31 - (hi & 31));
+        red_shared_or(wsm + kOffScratch + 4 * (wlo + w), m);
+      }
+      return 1;
+    }
+#endif
     uint32_t* base = orw + c.bm_word + wlo;
     for (uint32_t w = lane; w <= nw; w += 32) {
       uint32_t m = 0xFFFFFFFFu;

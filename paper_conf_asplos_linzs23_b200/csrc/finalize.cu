@@ -491,40 +491,71 @@ __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const Fina
   drgpum_object_stats_t* stats = static_cast<drgpum_object_stats_t*>(p.stats);
   drgpum_pattern_report_t* reps = static_cast<drgpum_pattern_report_t*>(p.reports);
   for (uint64_t o = p.o_lo + gwarp; o < p.o_hi; o += nwarps) {
-    // ---- bitmap groups of o, in order
+    // ---- bitmap groups of o, in order (one load for a single-group object)
     const uint32_t t0 = p.group_off[o], t1 = p.group_off[o + 1];
     BitMonoid bm = bm_identity();
-    for (uint32_t tb = t0; tb < t1; tb += 32) {
-      BitMonoid m = (tb + lane < t1) ? p.group_part[tb + lane] : bm_identity();
+    if (t1 - t0 == 1) {
+      bm = p.group_part[t0];
+    } else {
+      for (uint32_t tb = t0; tb < t1; tb += 32) {
+        BitMonoid m = (tb + lane < t1) ? p.group_part[tb + lane] : bm_identity();
 #pragma unroll
-      for (int d = 1; d < 32; d <<= 1) m = bm_cat(m, bm_shfl_down(m, d));
-      if (lane == 0) bm = bm_cat(bm, m);
+        for (int d = 1; d < 32; d <<= 1) m = bm_cat(m, bm_shfl_down(m, d));
+        if (lane == 0) bm = bm_cat(bm, m);
+      }
     }
-    // ---- hit row of o: 2 bits per access API inside its lifetime
+    // ---- hit row of o: 2 bits per access API inside its lifetime.  Each
+    // lane folds a contiguous run of hit words in order (count, first / last
+    // accessing API with its write / copy-set flags, TI gaps and DW pairs
+    // inside the run); the lanes are then joined at their boundaries: the
+    // gap / pair between a lane's first API and the previous non-empty
+    // lane's last one (one indexed shuffle), and warp sums / maxima.
     const DevObj ob = p.objs[o];
     const uint32_t nh = p.n_hit[o];
     const uint32_t nwords = (2 * nh + 31) / 32;
-    // each lane folds a contiguous run of hit words, then one ordered tree
     const uint32_t per = (nwords + 31) / 32;
     const uint32_t wlo = min(nwords, lane * per), whi = min(nwords, wlo + per);
-    HitM hm = hit_identity();
+    uint32_t cnt = 0, f_ts = 0, f_fl = 0, l_ts = 0, l_fl = 0, ti_cnt = 0, ti_max = 0, ti_sum = 0, dw = 0;
     for (uint32_t wi = wlo; wi < whi; ++wi) {
       uint32_t w = p.orw[ob.hit_word + wi];
       while (w) {
-        const uint32_t b = __ffs(w) - 1;
-        const uint32_t j = b >> 1;                  // API slot inside this word
-        const uint32_t pair = (w >> (2 * j)) & 3u;  // bit0 read, bit1 write
+        const uint32_t j = uint32_t(__ffs(w) - 1) >> 1;    // API slot inside this word
+        const uint32_t pair = (w >> (2 * j)) & 3u;         // bit0 read, bit1 write
         w &= ~(3u << (2 * j));
         const uint32_t rank = ob.r_lo + wi * 16 + j;
         const uint32_t ts = acc_ts[rank];
-        const uint32_t cs = acc_cs[rank];
-        const uint32_t wr = (pair >> 1) & 1u;
-        const HitM one{1, ts, ts, wr | (cs << 1) | (wr << 2) | (cs << 3), 0, 0, 0, 0};
-        hm = hit_cat(hm, one, p.ti_min_idle);
+        const uint32_t fl = (pair >> 1) | (uint32_t(acc_cs[rank]) << 1);   // bit0 write, bit1 copy/set
+        if (cnt == 0) {
+          f_ts = ts; f_fl = fl;
+        } else {
+          const uint32_t gap = ts - l_ts - 1;               // APIs strictly between (R6)
+          if (gap >= p.ti_min_idle) { ++ti_cnt; ti_max = max(ti_max, gap); ti_sum += gap; }
+          if (l_fl == 3u && fl == 3u) ++dw;                 // Def 3.7, R12
+        }
+        l_ts = ts; l_fl = fl; ++cnt;
       }
     }
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) hm = hit_cat(hm, hit_shfl_down(hm, d), p.ti_min_idle);
+    const uint32_t nz = __ballot_sync(FULL_MASK, cnt != 0);
+    HitM hm = hit_identity();
+    if (nz) {
+      const uint32_t below = nz & ((1u << lane) - 1u);
+      const int pl = below ? 31 - __clz(below) : lane;
+      const uint32_t p_ts = __shfl_sync(FULL_MASK, l_ts, pl);
+      const uint32_t p_fl = __shfl_sync(FULL_MASK, l_fl, pl);
+      if (cnt && below) {
+        const uint32_t gap = f_ts - p_ts - 1;
+        if (gap >= p.ti_min_idle) { ++ti_cnt; ti_max = max(ti_max, gap); ti_sum += gap; }
+        if (p_fl == 3u && f_fl == 3u) ++dw;
+      }
+      const int fl0 = __ffs(nz) - 1, fl1 = 31 - __clz(nz);
+      hm.cnt = __reduce_add_sync(FULL_MASK, cnt);
+      hm.first_ts = __shfl_sync(FULL_MASK, f_ts, fl0);
+      hm.last_ts = __shfl_sync(FULL_MASK, l_ts, fl1);
+      hm.ti_cnt = __reduce_add_sync(FULL_MASK, ti_cnt);
+      hm.ti_max = __reduce_max_sync(FULL_MASK, ti_max);
+      hm.ti_sum = __reduce_add_sync(FULL_MASK, ti_sum);   // sum of disjoint gaps < n_api < 2^31
+      hm.dw = __reduce_add_sync(FULL_MASK, dw);
+    }
     if (lane != 0) continue;
     // ---- stats (A6)
     const uint64_t n = (ob.end - ob.base) >> ob.shift;
@@ -637,6 +668,42 @@ int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_by
   return 1;
 }
 
+// Sparse reset (drgpum_reset after the first bind): one warp per tile, then
+// one warp per object for the hit rows; only objects with first[o] != NEVER
+// hold nonzero words.  Tiles start 4-word aligned inside 4-word padded
+// bitmaps, so whole 16-B stores cover them.
+__global__ void __launch_bounds__(256) reset_touched_kernel(uint32_t* __restrict__ orw,
+    const Tile* __restrict__ tiles, uint64_t n_tiles, const DevObj* __restrict__ objs,
+    const uint32_t* __restrict__ n_hit, const uint32_t* __restrict__ first, uint64_t n_obj) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
+    const Tile tl = tiles[t];
+    if (__ldg(first + tl.obj) == kNever) continue;   // warp-uniform
+    uint4* v = reinterpret_cast<uint4*>(orw + tl.word_lo);
+    const uint32_t nv = (tl.n_words + 3) / 4;
+    for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
+  }
+  for (uint64_t o = gwarp; o < n_obj; o += nwarps) {
+    if (__ldg(first + o) == kNever) continue;
+    const uint64_t hw = objs[o].hit_word;
+    const uint32_t nw = (2 * n_hit[o] + 31) / 32;
+    for (uint32_t i = lane; i < nw; i += 32) orw[hw + i] = 0;
+  }
+}
+
+int launch_reset_touched(uint32_t* orw, const Tile* tiles, uint64_t n_tiles, const DevObj* objs,
+                         const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, int num_sms,
+                         cudaStream_t s) {
+  const uint64_t work = n_tiles > n_obj ? n_tiles : n_obj;
+  if (!work) return 0;
+  uint64_t b = (work + 7) / 8;
+  if (b > uint64_t(num_sms) * 16) b = uint64_t(num_sms) * 16;
+  reset_touched_kernel<<<(unsigned)b, 256, 0, s>>>(orw, tiles, n_tiles, objs, n_hit, first, n_obj);
+  return 1;
+}
+
 // B7: OR n_src received slices into the owned words (after an all-to-all).
 __global__ void __launch_bounds__(256) merge_or_kernel(uint32_t* __restrict__ dst,
     const uint32_t* __restrict__ src, uint32_t n_src, uint64_t stride, uint64_t n_words) {
@@ -746,6 +813,93 @@ int launch_merge_owned(const MergeOwnedParams& q, int num_sms, cudaStream_t s) {
   if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
   merge_owned_kernel<<<(unsigned)b, 256, 0, s>>>(q);
   return 1;
+}
+
+// B7'' sparse: the owned merge reading only what a peer wrote.  A peer's
+// words of object o are nonzero only if its first[o] is set (every bit is
+// attributed or merged together with a first-use fold), so kernel 1 (one
+// warp per owned object) reads every peer's first/last, folds MIN / MAX,
+// records the mask of peers that touched o, and ORs those peers' hit rows;
+// kernel 2 (one warp per owned tile) ORs the bitmap tiles of the peers in the
+// mask.  Objects touched only here keep their local words (no traffic);
+// objects no rank touched cost two u32 reads per peer.  With record-range
+// shards most objects live inside one shard's time window, so the NVLink
+// traffic drops from (P-1)/P of the shadow to about the touched part of it.
+__global__ void __launch_bounds__(256) merge_owned_objects_kernel(const MergeOwnedParams q) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  uint8_t* const own = q.peer[q.rank];
+  for (uint64_t o = q.o_lo + gwarp; o < q.o_hi; o += nwarps) {
+    uint32_t f = 0xFFFFFFFFu, l = 0;
+    unsigned long long mask = 0;
+    for (uint32_t p0 = 0; p0 < q.n_peers; p0 += 32) {
+      const uint32_t p = p0 + lane;
+      uint32_t fp = 0xFFFFFFFFu, lp = 0;
+      if (p < q.n_peers) {
+        fp = __ldcg(reinterpret_cast<const uint32_t*>(q.peer[p] + q.first_off) + o);
+        lp = __ldcg(reinterpret_cast<const uint32_t*>(q.peer[p] + q.last_off) + o);
+      }
+      f = min(f, __reduce_min_sync(FULL_MASK, fp));
+      l = max(l, __reduce_max_sync(FULL_MASK, lp));
+      mask |= (unsigned long long)__ballot_sync(FULL_MASK, fp != 0xFFFFFFFFu) << p0;
+    }
+    if (lane == 0) {
+      reinterpret_cast<uint32_t*>(own + q.first_off)[o] = f;
+      reinterpret_cast<uint32_t*>(own + q.last_off)[o] = l;
+      q.pmask[o] = mask;
+    }
+    if ((mask & ~(1ull << q.rank)) == 0) continue;   // nobody else touched o
+    const uint64_t hw = q.objs[o].hit_word;
+    const uint32_t nw = (2 * q.n_hit[o] + 31) / 32;
+    for (uint32_t i = lane; i < nw; i += 32) {
+      uint32_t v = 0;
+      for (unsigned long long m = mask; m; m &= m - 1)
+        v |= __ldcg(reinterpret_cast<const uint32_t*>(q.peer[__ffsll(m) - 1] + q.or_off) + hw + i);
+      reinterpret_cast<uint32_t*>(own + q.or_off)[hw + i] = v;
+    }
+  }
+  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  if (q.rank == 0 && tid < 5) {   // records, attributed, unattributed, clipped, invalid
+    unsigned long long sum = 0;
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      sum += __ldcg(reinterpret_cast<const unsigned long long*>(q.peer[r] + q.ctr_off) + tid);
+    for (uint32_t r = 0; r < q.n_peers; ++r)
+      __stcg(reinterpret_cast<unsigned long long*>(q.peer[r] + q.ctr_off) + tid, sum);
+  }
+}
+
+__global__ void __launch_bounds__(256) merge_owned_tiles_kernel(const MergeOwnedParams q) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  uint8_t* const own = q.peer[q.rank];
+  for (uint64_t t = q.t_lo + gwarp; t < q.t_hi; t += nwarps) {
+    const Tile tl = q.tiles[t];
+    const unsigned long long mask = q.pmask[tl.obj];
+    if ((mask & ~(1ull << q.rank)) == 0) continue;   // warp-uniform: local words are final
+    const uint32_t nv = (tl.n_words + 3) / 4;
+    for (uint32_t i = lane; i < nv; i += 32) {
+      uint4 v = make_uint4(0, 0, 0, 0);
+      for (unsigned long long m = mask; m; m &= m - 1) {
+        const uint4 x = __ldcg(reinterpret_cast<const uint4*>(q.peer[__ffsll(m) - 1] + q.or_off + 4 * tl.word_lo) + i);
+        v.x |= x.x; v.y |= x.y; v.z |= x.z; v.w |= x.w;
+      }
+      reinterpret_cast<uint4*>(own + q.or_off + 4 * tl.word_lo)[i] = v;
+    }
+  }
+}
+
+int launch_merge_owned_sparse(const MergeOwnedParams& q, int num_sms, cudaStream_t s) {
+  const uint64_t no = q.o_hi - q.o_lo, nt = q.t_hi - q.t_lo;
+  uint64_t b1 = (max(no, uint64_t(1)) + 7) / 8;
+  if (b1 > uint64_t(num_sms) * 16) b1 = uint64_t(num_sms) * 16;
+  merge_owned_objects_kernel<<<(unsigned)b1, 256, 0, s>>>(q);
+  if (!nt) return 1;
+  uint64_t b2 = (nt + 7) / 8;
+  if (b2 > uint64_t(num_sms) * 16) b2 = uint64_t(num_sms) * 16;
+  merge_owned_tiles_kernel<<<(unsigned)b2, 256, 0, s>>>(q);
+  return 2;
 }
 
 // B7'': gather of the finalized stats / reports of rank r's objects into

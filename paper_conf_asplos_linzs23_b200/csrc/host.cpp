@@ -33,6 +33,7 @@ enum State { S_CREATED = 0, S_LOADED = 1, S_BOUND = 2 };
 
 struct Layout {
   uint64_t orw, first, last, ctr, cons;     // dynamic (reset per trace)
+  uint64_t pmask;
   uint64_t dyn_end;
   uint64_t objs, seg_start, seg_cand_off, seg, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
   uint64_t rfull;                 // per object: a whole-object range was queued in this trace
@@ -333,6 +334,7 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   L.acc_cs = put(c->n_acc);
   L.n_hit = put(4 * n);
   L.tiles = put(sizeof(Tile) * c->tiles.size());
+  L.pmask = put(8 * n);                      // owned merge: peers that touched each object
   L.tile_part = put(sizeof(BitMonoid) * c->tiles.size());
   L.groups = put(sizeof(Group) * c->groups.size());
   L.group_off = put(4 * (n + 1));
@@ -411,9 +413,28 @@ drgpum_status validate(drgpum_ctx* c, const drgpum_object_t* objs, uint64_t n_ob
   return DRGPUM_OK;
 }
 
-drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s) {
-  // dynamic state: shadow words, last, counters = 0; first = NEVER (one kernel)
-  ctx->launches += launch_reset(ctx->ws, ctx->L.dyn_end, ctx->L.first, 4 * ctx->n_obj, ctx->num_sms, s);
+#ifndef DRGPUM_SPARSE_RESET
+#define DRGPUM_SPARSE_RESET 1
+#endif
+#ifndef DRGPUM_SPARSE_MERGE
+#define DRGPUM_SPARSE_MERGE 1   // owned merge reads only the peers that touched an object
+#endif
+drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s, bool dense) {
+  // dynamic state: shadow words, last, counters = 0; first = NEVER.  Dense
+  // (bind: the memory is fresh): one pass over all of it.  Sparse (every
+  // later reset): only the touched objects' bitmap tiles and hit rows -- the
+  // OR words of an object are nonzero only if its first[] is not NEVER --,
+  // then the small sections from first[] on.
+  if (dense || !DRGPUM_SPARSE_RESET) {
+    ctx->launches += launch_reset(ctx->ws, ctx->L.dyn_end, ctx->L.first, 4 * ctx->n_obj, ctx->num_sms, s);
+  } else {
+    ctx->launches += launch_reset_touched(at<uint32_t>(ctx, ctx->L.orw), at<Tile>(ctx, ctx->L.tiles),
+                                          ctx->tiles.size(), at<DevObj>(ctx, ctx->L.objs),
+                                          at<uint32_t>(ctx, ctx->L.n_hit), at<uint32_t>(ctx, ctx->L.first),
+                                          ctx->n_obj, ctx->num_sms, s);
+    ctx->launches += launch_reset(ctx->ws + ctx->L.first, ctx->L.dyn_end - ctx->L.first, 0, 4 * ctx->n_obj,
+                                  ctx->num_sms, s);
+  }
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     CK(cudaMemsetAsync(ctx->ws + ctx->L.sa_owner, 0, ctx->L.sa_end - ctx->L.sa_owner, s));
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
@@ -756,7 +777,7 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
   }
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
     if ((r = up(L.fq_slot_base, ctx->slot_base.data(), 8 * n))) return r;
-  if ((r = enqueue_reset(ctx, st))) return r;
+  if ((r = enqueue_reset(ctx, st, true))) return r;
   // host vectors stay alive in ctx, so the async uploads are safe; make the
   // bind synchronous anyway so callers may immediately reuse their stream
   CK(cudaStreamSynchronize(st));
@@ -768,7 +789,7 @@ DRGPUM_API drgpum_status drgpum_reset(drgpum_ctx* ctx, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "reset before workspace_bind");
   if (drgpum_status _d = set_device(ctx)) return _d;
-  return enqueue_reset(ctx, as_stream(stream));
+  return enqueue_reset(ctx, as_stream(stream), false);
 }
 
 DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_record_t* d_recs,
@@ -956,7 +977,17 @@ DRGPUM_API drgpum_status drgpum_merge_peers_owned(drgpum_ctx* ctx, void* const* 
   q.b_lo = bw(lo); q.b_hi = bw(hi);   // multiples of 4 (every bitmap is padded to 4 words)
   q.h_lo = hw(lo); q.h_hi = hw(hi);
   q.o_lo = lo; q.o_hi = hi;
+  q.tiles = at<Tile>(ctx, ctx->L.tiles);
+  q.t_lo = ctx->tile_off[lo];
+  q.t_hi = ctx->tile_off[hi];
+  q.objs = at<DevObj>(ctx, ctx->L.objs);
+  q.n_hit = at<uint32_t>(ctx, ctx->L.n_hit);
+  q.pmask = at<unsigned long long>(ctx, ctx->L.pmask);
+#if DRGPUM_SPARSE_MERGE
+  ctx->launches += launch_merge_owned_sparse(q, ctx->num_sms, as_stream(stream));
+#else
   ctx->launches += launch_merge_owned(q, ctx->num_sms, as_stream(stream));
+#endif
   CK(cudaGetLastError());
   ctx->final_valid = false;
   ctx->owned = true;

@@ -190,6 +190,13 @@ struct MergeOwnedParams {
   uint32_t n_peers, rank;
   uint64_t or_off, first_off, last_off, ctr_off;
   uint64_t b_lo, b_hi, h_lo, h_hi, o_lo, o_hi;
+  // sparse form: the owned objects' tiles [t_lo, t_hi) and per-object masks
+  // of the peers whose first[] is set (only those hold nonzero words)
+  const Tile* tiles;
+  uint64_t t_lo, t_hi;
+  const DevObj* objs;
+  const uint32_t* n_hit;
+  unsigned long long* pmask;   // [n_obj] (this workspace)
 };
 
 // Gather (B7''): rank r stores bytes [lo, hi) of the stats and of the
@@ -214,8 +221,15 @@ int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);
 int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_bytes, int num_sms, cudaStream_t s);
+// Sparse reset of the OR words: zero the bitmap tiles and hit rows of the
+// objects whose first[] is not NEVER (every attributed or merged bit of an
+// object comes with a first-use fold, so the others are still all zero).
+int launch_reset_touched(uint32_t* orw, const Tile* tiles, uint64_t n_tiles, const DevObj* objs,
+                         const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, int num_sms,
+                         cudaStream_t s);
 int launch_merge_peers(const MergePeersParams& q, int num_sms, cudaStream_t s);
 int launch_merge_owned(const MergeOwnedParams& q, int num_sms, cudaStream_t s);
+int launch_merge_owned_sparse(const MergeOwnedParams& q, int num_sms, cudaStream_t s);
 int launch_gather_peers(const GatherParams& q, int num_sms, cudaStream_t s);
 int launch_merge_or(uint32_t* dst, const uint32_t* src, uint32_t n_src,
                     uint64_t src_stride, uint64_t n_words, int num_sms, cudaStream_t s);

@@ -312,3 +312,55 @@ def test_cuda_graph_replay(name):
         if exp is None:
             exp = expected_or_words(s, orc, p.objects, p.kinds)
         assert np.array_equal(orw, exp), rep
+
+
+def test_sparse_reset_between_traces():
+    """drgpum_reset zeroes only the objects whose first-use word is set (the
+    bitmap tiles and hit rows of the touched objects).  Trace A touches one
+    half of the objects, trace B the other half plus some of A's: after
+    reset, the shadow must be exactly B's (objects only A touched come back
+    all zero), including after a reset that follows a merge of a second
+    session's shadow (merged bits carry merged first-use words)."""
+    p = build_config("C1")
+    r = gen_all_records(p)
+    orc_any = Oracle(p.objects, p.kinds)
+    # which object each record belongs to (oracle-independent: by address range)
+    base = p.objects["base"].astype(np.uint64)
+    end = base + p.objects["size"].astype(np.uint64)
+    order = np.argsort(base)
+    k = np.searchsorted(base[order], r["addr"], side="right") - 1
+    obj = np.where(k >= 0, order[np.maximum(k, 0)], -1)
+    inside = (k >= 0) & (r["addr"] < end[np.maximum(obj, 0)])
+    even = inside & (obj % 2 == 0)
+    recs_a, recs_b = r[even], r[~even | (np.arange(len(r)) % 7 == 0)]
+    s = _session(p.objects, p.kinds)
+    dev = lambda x: torch.from_numpy(np.ascontiguousarray(x).view(np.uint8)).cuda()
+    for first_trace in (recs_a, recs_b, r):
+        s.reset()
+        s.attribute(dev(first_trace))
+        s.finalize()
+        s.reset()
+        s.attribute(dev(recs_b))
+        orc = Oracle(p.objects, p.kinds)
+        orc.attribute(recs_b)
+        ost, octr = orc.stats()
+        st, ctr = s.object_stats()
+        for name in ost.dtype.names:
+            assert np.array_equal(st[name], ost[name]), name
+        assert np.array_equal(s.or_words().cpu().numpy().view(np.uint32),
+                              expected_or_words(s, orc, p.objects, p.kinds))
+    # after a merge: OR a second session's shadow (trace A) into s, reset, B
+    t = _session(p.objects, p.kinds)
+    t.attribute(dev(recs_a))
+    s.reset()
+    s.attribute(dev(recs_b))
+    s.merge_peers([s.workspace.data_ptr(), t.workspace.data_ptr()], 0)
+    t.merge_peers([s.workspace.data_ptr(), t.workspace.data_ptr()], 1)
+    torch.cuda.synchronize()
+    s.reset()
+    s.attribute(dev(recs_b))
+    orc = Oracle(p.objects, p.kinds)
+    orc.attribute(recs_b)
+    assert np.array_equal(s.or_words().cpu().numpy().view(np.uint32),
+                          expected_or_words(s, orc, p.objects, p.kinds))
+    del orc_any
