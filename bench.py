@@ -510,11 +510,13 @@ def roofline(w, m, touched, hbm, hbm_src):
     if os.path.exists(tfile):
         try:
             t = json.load(open(tfile)).get(w.cfg)
-            traffic = None if t is None else int(t["bytes_per_launch"])
+            traffic = None if t is None else int(t["bytes_per_launch"])   # one launch of w.chunks
         except Exception:
             traffic = None
     return {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
             "frac": achieved / hbm, "traffic": traffic,
+            "algorithmic_bytes_per_launch": alg_bytes / len(w.chunks),
+            "launches_per_step": len(w.chunks),
             "kernel": "drgpum_trace_attribute (attribute_kernel + range_expand_kernel)",
             "algorithmic_bytes": alg_bytes, "records_per_rank": w.n_local,
             "bytes_rule": "16 B per record + 4 B per touched shadow word",
