@@ -150,26 +150,23 @@ __device__ __noinline__ uint32_t interior_zero_run(uint32_t u) {
 #ifndef DRGPUM_TR_UNIFORM
 #define DRGPUM_TR_UNIFORM 2
 #endif
+#ifndef DRGPUM_TR_SMALL
+#define DRGPUM_TR_SMALL 1   // tiles of <= 128 words: 4 words per lane, no transpose
+#endif
 #ifndef DRGPUM_TR_GRID_PER_SM
 #define DRGPUM_TR_GRID_PER_SM 16
 #endif
-__global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(const uint32_t* __restrict__ orw,
-    const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr) {
-  const int lane = threadIdx.x & 31;
-  if (blockIdx.x == 0 && threadIdx.x == 0) ctr[C_CONSISTENCY] = 0;   // counted by object_finalize_kernel
-  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  constexpr uint32_t kLaneWords = kTileWords / 32;          // 32 words = 1024 bits per lane
+// One tile of kLaneWords words per lane: 32 (full 1024-word tiles, lane l
+// folds words [32l, 32l+32) after a transpose through buf) or 4 (tiles of at
+// most 128 words -- small objects and objects' last tiles: the coalesced 16-B
+// load already gives lane l words [4l, 4l+4), no transpose, 4-step folds).
+// The run-view length of a 4-word-lane tile is 4096 bits; such tiles are
+// always an object's last, so the length only has to cover its real bits.
+template <uint32_t kLaneWords>
+__device__ __forceinline__ void reduce_one_tile(const uint32_t* __restrict__ orw, const Tile& tl, uint64_t t,
+                                                BitMonoid* __restrict__ out, uint4* buf, int lane) {
   constexpr uint32_t kLaneBits = kLaneWords * 32;
-  static_assert(kLaneWords == 32, "transpose below assumes 8 x 16-B chunks per lane");
-  // per-warp 4-KB transpose buffer: the tile is read coalesced (lane l: words
-  // 128b + 4l .. +3) and each 16-B chunk stored where its owning lane reads
-  // it back; slot = owner * 8 + (chunk ^ (owner & 7)) keeps both sides free
-  // of bank conflicts
-  __shared__ uint4 s_tile[8][kTileWords / 4];
-  uint4* buf = s_tile[threadIdx.x >> 5];
-  for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
-    const Tile tl = tiles[t];
+  static_assert(kLaneWords == 32 || kLaneWords == 4, "lane widths");
     const uint32_t nbits = uint32_t(tl.n_bits);
     const uint32_t w0 = kLaneWords * uint32_t(lane);
     uint4 v[kLaneWords / 4];
@@ -197,7 +194,7 @@ __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(cons
           const uint64_t L = 32u * kLaneBits;
           out[t] = all1 ? BitMonoid{L, L, 0, L - 1, 0, 0, 0} : BitMonoid{L, 0, kNoPos, kNoPos, L, L, L};
         }
-        continue;
+        return;
       }
     }
 #if DRGPUM_TR_UNIFORM > 1
@@ -231,20 +228,22 @@ __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(cons
           out[t] = all1 ? BitMonoid{L, nbits, 0, nbits - 1u, 0, 0, 0}
                         : BitMonoid{L, 0, kNoPos, kNoPos, nbits, 0, nbits};
         }
-        continue;
+        return;
       }
     }
 #endif
 #endif
-    __syncwarp();   // the previous tile's reads of buf are done
+    if constexpr (kLaneWords == 32) {   // lane l <- words [32l, 32l+32) through the buffer
+      __syncwarp();   // the previous tile's reads of buf are done
 #pragma unroll
-    for (int b = 0; b < int(kLaneWords / 4); ++b) {
-      const uint32_t owner = 4 * b + (lane >> 3), chunk = lane & 7;
-      buf[owner * 8 + (chunk ^ (owner & 7))] = v[b];
-    }
-    __syncwarp();
+      for (int b = 0; b < int(kLaneWords / 4); ++b) {
+        const uint32_t owner = 4 * b + (lane >> 3), chunk = lane & 7;
+        buf[owner * 8 + (chunk ^ (owner & 7))] = v[b];
+      }
+      __syncwarp();
 #pragma unroll
-    for (int k = 0; k < int(kLaneWords / 4); ++k) v[k] = buf[lane * 8 + (k ^ (lane & 7))];
+      for (int k = 0; k < int(kLaneWords / 4); ++k) v[k] = buf[lane * 8 + (k ^ (lane & 7))];
+    }   // kLaneWords == 4: the coalesced load already gave lane l words [4l, 4l+4)
     // lane fold, branch-free per word: real popcount and the nonzero real
     // words (lowest / highest accessed bit at the end); run view: z = zeros
     // since the last 1, so a word with a 1 closes a zero run of z + ctz(u)
@@ -306,10 +305,17 @@ __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(cons
     // real word (read back from the transpose buffer, masked like above)
     uint32_t lo = kNoPos32, hi = kNoPos32;
     if (nzr) {
-      const uint32_t* wl = reinterpret_cast<const uint32_t*>(buf + lane * 8);
       const int jl = __ffs(nzr) - 1, jh = 31 - __clz(nzr);
-      const uint32_t xl = wl[4 * ((jl >> 2) ^ (lane & 7)) + (jl & 3)];
-      const uint32_t xh = wl[4 * ((jh >> 2) ^ (lane & 7)) + (jh & 3)];
+      uint32_t xl, xh;
+      if constexpr (kLaneWords == 32) {
+        const uint32_t* wl = reinterpret_cast<const uint32_t*>(buf + lane * 8);
+        xl = wl[4 * ((jl >> 2) ^ (lane & 7)) + (jl & 3)];
+        xh = wl[4 * ((jh >> 2) ^ (lane & 7)) + (jh & 3)];
+      } else {
+        const uint32_t xs[4] = {v[0].x, v[0].y, v[0].z, v[0].w};
+        xl = xs[jl & 3];
+        xh = xs[jh & 3];
+      }
       const uint32_t bl = (w0 + jl) * 32, bh = (w0 + jh) * 32;
       const uint32_t nl = min(32u, nbits - bl), nh = min(32u, nbits - bh);   // both words hold real bits
       const uint32_t ml = nl == 32 ? xl : xl & ((1u << nl) - 1u);
@@ -380,6 +386,27 @@ __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(cons
       r.pre = acc.pre; r.suf = acc.suf; r.best = acc.best;
       out[t] = r;
     }
+}
+
+__global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(const uint32_t* __restrict__ orw,
+    const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr) {
+  const int lane = threadIdx.x & 31;
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctr[C_CONSISTENCY] = 0;   // counted by object_finalize_kernel
+  const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  static_assert(kTileWords == 1024, "transpose assumes 8 x 16-B chunks per lane");
+  // per-warp 4-KB transpose buffer: the tile is read coalesced (lane l: words
+  // 128b + 4l .. +3) and each 16-B chunk stored where its owning lane reads
+  // it back; slot = owner * 8 + (chunk ^ (owner & 7)) keeps both sides free
+  // of bank conflicts
+  __shared__ uint4 s_tile[8][kTileWords / 4];
+  uint4* buf = s_tile[threadIdx.x >> 5];
+  for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
+    const Tile tl = tiles[t];
+#if DRGPUM_TR_SMALL
+    if (tl.n_words <= 128) { reduce_one_tile<4>(orw, tl, t, out, buf, lane); continue; }
+#endif
+    reduce_one_tile<32>(orw, tl, t, out, buf, lane);
   }
 }
 
@@ -678,27 +705,52 @@ __global__ void __launch_bounds__(256) reset_touched_kernel(uint32_t* __restrict
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
-    const Tile tl = tiles[t];
-    if (__ldg(first + tl.obj) == kNever) continue;   // warp-uniform
-    uint4* v = reinterpret_cast<uint4*>(orw + tl.word_lo);
-    const uint32_t nv = (tl.n_words + 3) / 4;
-    for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
+  // 32 tiles per warp step: each lane checks one tile's object (independent
+  // loads), then the warp zeroes the touched ones
+  for (uint64_t t0 = gwarp * 32; t0 < n_tiles; t0 += nwarps * 32) {
+    const uint64_t t = t0 + lane;
+    Tile tl{0, 0, 0, 0, 0};
+    bool touched = false;
+    if (t < n_tiles) {
+      tl = tiles[t];
+      touched = __ldg(first + tl.obj) != kNever;
+    }
+    uint32_t m = __ballot_sync(FULL_MASK, touched);
+    while (m) {
+      const int j = __ffs(m) - 1;
+      m &= m - 1;
+      const uint64_t wlo = __shfl_sync(FULL_MASK, tl.word_lo, j);
+      const uint32_t nv = (__shfl_sync(FULL_MASK, tl.n_words, j) + 3) / 4;
+      uint4* v = reinterpret_cast<uint4*>(orw + wlo);
+      for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
+    }
   }
-  for (uint64_t o = gwarp; o < n_obj; o += nwarps) {
-    if (__ldg(first + o) == kNever) continue;
-    const uint64_t hw = objs[o].hit_word;
-    const uint32_t nw = (2 * n_hit[o] + 31) / 32;
-    for (uint32_t i = lane; i < nw; i += 32) orw[hw + i] = 0;
+  for (uint64_t o0 = gwarp * 32; o0 < n_obj; o0 += nwarps * 32) {   // hit rows, 32 objects per step
+    const uint64_t o = o0 + lane;
+    const bool touched = o < n_obj && __ldg(first + o) != kNever;
+    uint64_t hw = 0;
+    uint32_t nw = 0;
+    if (touched) {
+      hw = objs[o].hit_word;
+      nw = (2 * n_hit[o] + 31) / 32;
+    }
+    uint32_t m = __ballot_sync(FULL_MASK, touched);
+    while (m) {
+      const int j = __ffs(m) - 1;
+      m &= m - 1;
+      const uint64_t h = __shfl_sync(FULL_MASK, hw, j);
+      const uint32_t n = __shfl_sync(FULL_MASK, nw, j);
+      for (uint32_t i = lane; i < n; i += 32) orw[h + i] = 0;
+    }
   }
 }
 
 int launch_reset_touched(uint32_t* orw, const Tile* tiles, uint64_t n_tiles, const DevObj* objs,
                          const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, int num_sms,
                          cudaStream_t s) {
-  const uint64_t work = n_tiles > n_obj ? n_tiles : n_obj;
-  if (!work) return 0;
-  uint64_t b = (work + 7) / 8;
+  const uint64_t work = (n_tiles > n_obj ? n_tiles : n_obj) / 32;
+  if (!work && !n_tiles) return 0;
+  uint64_t b = (work + 7) / 8 + 1;
   if (b > uint64_t(num_sms) * 16) b = uint64_t(num_sms) * 16;
   reset_touched_kernel<<<(unsigned)b, 256, 0, s>>>(orw, tiles, n_tiles, objs, n_hit, first, n_obj);
   return 1;
