@@ -282,7 +282,7 @@ __device__ __forceinline__ void reduce_one_tile(const uint32_t* __restrict__ orw
       run = masked ? real | ~vm : x;
     };
     if (full) {
-      pop = kLaneBits; nzr = 0xFFFFFFFFu; z = 0; pre = 0; seen = true;
+      pop = kLaneBits; nzr = kLaneWords == 32 ? 0xFFFFFFFFu : (1u << kLaneWords) - 1u; z = 0; pre = 0; seen = true;
     } else if (empty) {
       z = kLaneBits;
     } else if (!masked) {
