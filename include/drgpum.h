@@ -224,6 +224,16 @@ DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx *ctx, uint32_t features)
 DRGPUM_API drgpum_status drgpum_set_queue_capacity(drgpum_ctx *ctx, uint32_t range_entries,
                                                    uint32_t aux_entries);
 
+/* NEXT-2 (DRGPUM_FEATURE_FREQUENCY) processes every attribute call in
+ * sub-calls of at most records_per_call records (default 2^24); the
+ * workspace holds 3 x records_per_call 8-byte event keys twice, plus the
+ * digit histograms (~100 B per record of capacity).  The events of one API
+ * that continues across calls are carried and must fit the capacity too
+ * (ENOMEM at the query otherwise).  Set after objects_load, before
+ * workspace_size / workspace_bind (ESTATE otherwise); EINVAL outside
+ * [1024, 2^31]. */
+DRGPUM_API drgpum_status drgpum_set_frequency_capacity(drgpum_ctx *ctx, uint64_t records_per_call);
+
 /* Bytes of device workspace the loaded program needs (ESTATE before load). */
 DRGPUM_API drgpum_status drgpum_workspace_size(const drgpum_ctx *ctx, uint64_t *bytes);
 

@@ -5,164 +5,44 @@
 // zeroes it when a GPU API that will access the object starts, counts every
 // instrumented access of that API, and when the API finishes tests the
 // variance of the frequencies.  Reading R22: the statistics run
-// over the elements the API touched (the hashmap's cells); CV is the
-// population coefficient of variation; NUAF at API A iff CV > X (20%),
-// exactly: (n*S2 - S1^2) * 100^2 > X^2 * S1^2.
+// over the elements the API touched; CV is the population coefficient of
+// variation; NUAF at API A iff CV > X (20%), exactly
+// (n*S2 - S1^2) * 100^2 > X^2 * S1^2, with n = elements A touched, S1 = sum
+// of their frequencies, S2 = sum of their squares -- per (object, API) slot.
 //
-// B200 version: the paper's hashmap, one per API, all APIs at once.  The
-// records of one API form a contiguous "segment" of the timestamp-sorted
-// trace.  Every increment of an element's count returns the previous count
-// c, so the (object, API) sums follow without a second pass: n += (c == 0),
-// S1 += 1, S2 += 2c + 1.
-//   1. freq_scan_kernel / freq_plan_kernel: run starts per timestamp, ordered
-//      compaction into segments.
-//   2. freq_count_kernel: records and element touches per (object, API)
-//      slot (warp-aggregated).  A slot with ONE record needs no counting at
-//      all -- each of its elements is touched exactly once (n = S1 = S2 =
-//      its element count): every memcpy / memset.  The other slots' touches
-//      size their segment's open-addressing table (capacity 2^k >= 2x
-//      touches).
-//   3. freq_table_plan_kernel: tables laid out by a prefix sum, cut into
-//      batches of `budget` entries.
-//   4. freq_apply_kernel (cooperative): per batch, zero the tables, insert
-//      every record's elements (CAS on the key, add on the count), expand
-//      wide records (> 64 elements) grid-wide; the segments of a batch are
-//      independent, so they all run concurrently.  Segments that may continue
-//      across an attribute call (the first and the last of a call) or whose
-//      table would not fit keep their counts in per-element cells {API tag,
-//      count} instead and run alone, in trace order, after the batches.
-// Lanes accumulate locally while they stay in one slot, then in a small
-// per-block shared-memory table, flushed to the global sums at the end.
-#include <cooperative_groups.h>
-
+// B200 version, sort-based (no hash tables, no dependent atomics):
+//   1. freq_events_kernel: every attributed record is the interval
+//      [g0, g1] of global element indices it touches; consecutive records of
+//      a warp that touch adjacent, disjoint intervals of one object in one
+//      API (sequential sweeps) are merged into one interval first.  Each
+//      interval becomes two 64-bit keys (rank << pos_bits) | 2*g0 (start)
+//      and (rank << pos_bits) | 2*g1 + 1 (end); rank = access-API rank.
+//   2. An LSD radix sort (8-bit digits, stable: tile histograms, a
+//      digit-major exclusive scan, a tile-local stable ranking through shared
+//      memory and coalesced stores) orders the keys by (API, element).
+//      Passes whose digit is the same for every key are skipped.
+//   3. The sweep: a scan of +1 (start) / -1 (end) gives, after key i, the
+//      number c of intervals covering the elements between key i and key
+//      i+1 -- [ceil(p_i/2), ceil(p_{i+1}/2)) -- i.e. the access frequency of
+//      each of those len elements within that API.  Each such run adds
+//      (len, c*len, c*c*len) to (n, S1, S2) of its (object, API) slot
+//      (intervals never span objects or APIs, so runs with c > 0 do not
+//      either; every API's intervals are balanced, so no segmented scan is
+//      needed).
+//   4. The call's last API may continue in the next call (records are in
+//      timestamp order across calls): its sorted keys are carried to the
+//      front of the other key buffer and sorted together with the next
+//      call's; a query sweeps the carried keys into a copy of the sums.
 #include "internal.cuh"
-
-namespace cg = cooperative_groups;
 
 namespace drgpum {
 
-constexpr uint64_t kFreqInline = 64;         // wider records are expanded grid-wide
-constexpr uint64_t kFreqChunk = 1024;        // elements per queue chunk (32 per lane)
-constexpr int kU = 8;                        // elements in flight per lane
-constexpr int kFreqThreads = 256;
-constexpr uint64_t kNone64 = ~0ull;
+#define FULL_MASK 0xFFFFFFFFu
+constexpr int kFT = 256;                       // threads per block, every kernel here
+constexpr uint32_t kSweepItems = 8;            // keys per thread in the sweep
+constexpr uint32_t kSweepChunk = kFT * kSweepItems;
 
-// kU elements x0 + st*j at once (valid bits in v): first probes and the adds
-// are issued back to back, so a lane waits for two round trips per kU elements
-__device__ __forceinline__ void tbl_incr_many(FreqEntry* t, uint32_t logc, uint64_t x0, uint64_t st, uint32_t v,
-                                              uint32_t (&prev)[kU]) {
-  const uint32_t mask = (1u << logc) - 1;
-  unsigned long long k[kU];
-  uint32_t h[kU];
-#pragma unroll
-  for (int j = 0; j < kU; ++j)
-    if (v >> j & 1) {
-      const unsigned long long key = x0 + st * j + 1;
-      h[j] = uint32_t((key * 0x9E3779B97F4A7C15ull) >> (64 - logc));
-      k[j] = atomicCAS(&t[h[j]].key, 0ull, key);
-    }
-#pragma unroll
-  for (int j = 0; j < kU; ++j)
-    if (v >> j & 1) {
-      const unsigned long long key = x0 + st * j + 1;
-      while (k[j] != 0 && k[j] != key) {
-        h[j] = (h[j] + 1) & mask;
-        k[j] = atomicCAS(&t[h[j]].key, 0ull, key);
-      }
-    }
-#pragma unroll
-  for (int j = 0; j < kU; ++j)
-    if (v >> j & 1) prev[j] = uint32_t(atomicAdd(&t[h[j]].cnt, 1ull));
-}
-
-// one key, `add` more touches; returns the count before them
-__device__ __forceinline__ uint32_t tbl_add(FreqEntry* t, uint32_t logc, unsigned long long key, uint32_t add) {
-  const uint32_t mask = (1u << logc) - 1;
-  uint32_t h = uint32_t((key * 0x9E3779B97F4A7C15ull) >> (64 - logc));
-  unsigned long long k = atomicCAS(&t[h].key, 0ull, key);
-  while (k != 0 && k != key) {
-    h = (h + 1) & mask;
-    k = atomicCAS(&t[h].key, 0ull, key);
-  }
-  return uint32_t(atomicAdd(&t[h].cnt, (unsigned long long)add));
-}
-
-__device__ __forceinline__ void cell_incr_many(unsigned long long* cells, uint32_t tag, uint64_t x0, uint64_t st,
-                                               uint32_t v, uint32_t (&prev)[kU]) {
-#pragma unroll
-  for (int j = 0; j < kU; ++j)
-    if (v >> j & 1)
-      asm volatile("red.relaxed.gpu.global.max.u64 [%0], %1;" ::"l"(cells + x0 + st * j),
-                   "l"((unsigned long long)tag << 32) : "memory");
-#pragma unroll
-  for (int j = 0; j < kU; ++j)
-    if (v >> j & 1) prev[j] = uint32_t(atomicAdd(cells + x0 + st * j, 1ull));
-}
-
-// Per-block (object, API) accumulators in shared memory.
-constexpr int kBlkSlots = 16;
-struct BlkAcc {
-  unsigned long long slot[kBlkSlots], n[kBlkSlots], s1[kBlkSlots], s2[kBlkSlots];
-};
-
-__device__ __forceinline__ void blk_add(BlkAcc& b, unsigned long long* acc, uint64_t slot, uint64_t n,
-                                        uint64_t s1, uint64_t s2) {
-  const unsigned h = unsigned(slot) & (kBlkSlots - 1);
-  for (int k = 0; k < kBlkSlots; ++k) {
-    const unsigned j = (h + k) & (kBlkSlots - 1);
-    unsigned long long cur = b.slot[j];
-    if (cur == ~0ull) cur = atomicCAS(&b.slot[j], ~0ull, (unsigned long long)slot);
-    if (cur == ~0ull || cur == slot) {
-      atomicAdd(&b.n[j], (unsigned long long)n);
-      atomicAdd(&b.s1[j], (unsigned long long)s1);
-      atomicAdd(&b.s2[j], (unsigned long long)s2);
-      return;
-    }
-  }
-  atomicAdd(acc + 3 * slot, (unsigned long long)n);            // table full: straight to global
-  atomicAdd(acc + 3 * slot + 1, (unsigned long long)s1);
-  atomicAdd(acc + 3 * slot + 2, (unsigned long long)s2);
-}
-
-// flush the block table to the global accumulators and clear it (block-wide)
-__device__ __forceinline__ void blk_flush(BlkAcc& b, unsigned long long* acc) {
-  __syncthreads();
-  if (threadIdx.x < kBlkSlots) {
-    const unsigned j = threadIdx.x;
-    const unsigned long long sl = b.slot[j];
-    if (sl != ~0ull && b.s1[j]) {
-      atomicAdd(acc + 3 * sl, b.n[j]);
-      atomicAdd(acc + 3 * sl + 1, b.s1[j]);
-      atomicAdd(acc + 3 * sl + 2, b.s2[j]);
-    }
-    b.slot[j] = ~0ull;
-    b.n[j] = b.s1[j] = b.s2[j] = 0;
-  }
-  __syncthreads();
-}
-
-struct SlotAcc {
-  uint64_t slot = ~0ull, n = 0, s1 = 0, s2 = 0;
-  __device__ void flush(BlkAcc& b, unsigned long long* acc) {
-    if (slot != ~0ull && s1) blk_add(b, acc, slot, n, s1, s2);
-    n = s1 = s2 = 0;
-  }
-  __device__ void to(BlkAcc& b, unsigned long long* acc, uint64_t sl) {
-    if (sl != slot) { flush(b, acc); slot = sl; }
-  }
-  __device__ void add(BlkAcc& b, unsigned long long* acc, uint64_t sl, uint32_t prev) {
-    to(b, acc, sl);
-    n += prev == 0;
-    s1 += 1;
-    s2 += 2ull * prev + 1;
-  }
-  __device__ void add_once(BlkAcc& b, unsigned long long* acc, uint64_t sl, uint64_t len) {
-    to(b, acc, sl);            // len distinct elements, each touched once
-    n += len;
-    s1 += len;
-    s2 += len;
-  }
-};
+__device__ __forceinline__ uint32_t ts_of(const AttrParams& p, uint64_t i) { return __ldcs(&p.recs[i].w) & 0x7FFFFFFFu; }
 
 // object lookup (same index and rules as the attribution kernel)
 __device__ __forceinline__ uint32_t freq_find(const AttrParams& p, const uint64_t* l1, uint64_t addr,
@@ -179,20 +59,18 @@ __device__ __forceinline__ uint32_t freq_find(const AttrParams& p, const uint64_
   return l == c0 ? kNone : p.cand[l - 1].obj;
 }
 
-__device__ __forceinline__ uint32_t ts_of(const AttrParams& p, uint64_t i) { return __ldcs(&p.recs[i].w) & 0x7FFFFFFFu; }
-
-// A lane's cached object, and the element range / slot of one record.
+// A lane's cached object.
 struct LaneObj {
-  uint64_t base = 0, size = 0, eb = 0, sb = 0;
-  uint32_t ta = 0, tf = 0, rlo = 0, shift = 0;
+  uint64_t base = 0, size = 0, eb = 0;
+  uint32_t ta = 0, tf = 0, shift = 0, obj = kNone;
 };
-struct Touch { uint64_t g0, g1, slot; };   // global elements [g0, g1]
 
-// false if the record touches no live object (or is malformed)
+// the global element interval [g0, g1] record i touches, false if it touches
+// no live object (or is malformed); c caches the object between records
 __device__ __forceinline__ bool resolve(const FreqParams& q, const uint64_t* l1, LaneObj& c, uint64_t i,
-                                        uint32_t t, uint32_t rank, Touch& out) {
+                                        uint32_t t, uint64_t& g0, uint64_t& g1) {
   const AttrParams& p = q.a;
-  const uint4 r = __ldcs(p.recs + i);                 // streamed: keep L2 for the tables
+  const uint4 r = __ldcs(p.recs + i);                 // streamed once
   const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
   const uint32_t size = r.z;
   if (size == 0 || addr > ~0ull - size) return false;
@@ -202,356 +80,428 @@ __device__ __forceinline__ bool resolve(const FreqParams& q, const uint64_t* l1,
     const DevObj d = p.objs[o];
     if (t >= d.t_free) return false;
     c.base = d.base; c.size = d.end - d.base; c.ta = d.t_alloc; c.tf = d.t_free;
-    c.rlo = d.r_lo; c.shift = d.shift;
-    c.eb = q.elem_base[o]; c.sb = q.slot_base[o];
+    c.shift = d.shift; c.obj = o; c.eb = q.elem_base[o];
   }
   const uint64_t off = addr - c.base, end = min(off + size, c.size);
-  out.g0 = c.eb + (off >> c.shift);
-  out.g1 = c.eb + ((end - 1) >> c.shift);
-  out.slot = c.sb + (rank - c.rlo);
+  g0 = c.eb + (off >> c.shift);
+  g1 = c.eb + ((end - 1) >> c.shift);
   return true;
 }
 
-// every element of [g0, g1] (stride st, for lanes of a warp) touched once more
-// in the table tb (lc) or, if tag != 0, in the element cells
-struct Counter {
-  FreqEntry* tb;
-  unsigned long long* cells;
-  uint32_t lc, tag;
-  template <typename Acc>
-  __device__ __forceinline__ void range(Acc& add, uint64_t g0, uint64_t g1, uint64_t st) const {
-    for (uint64_t x0 = g0; x0 <= g1; x0 += st * kU) {
-      uint32_t v = 0, prev[kU];
-#pragma unroll
-      for (int j = 0; j < kU; ++j)
-        if (x0 + st * j <= g1) v |= 1u << j;
-      if (tag) cell_incr_many(cells, tag, x0, st, v, prev);
-      else tbl_incr_many(tb, lc, x0, st, v, prev);
-#pragma unroll
-      for (int j = 0; j < kU; ++j)
-        if (v >> j & 1) add(prev[j]);
-    }
-  }
-};
+__device__ __forceinline__ uint64_t* keys_buf(const FreqParams& q, uint32_t which) {
+  return which ? q.keys1 : q.keys0;
+}
+// buffer holding the keys before radix pass d (skipped passes do not flip)
+__device__ __forceinline__ uint32_t buf_before(const FreqParams& q, uint32_t d) {
+  uint32_t b = uint32_t(q.ctl[1]);
+  for (uint32_t k = 0; k < d; ++k) b ^= q.ctl[8 + k] ? 0u : 1u;
+  return b;
+}
+__device__ __forceinline__ uint64_t n_keys(const FreqParams& q) {
+  const unsigned long long n = q.ctl[0];
+  return n < q.cap ? n : q.cap;
+}
 
-// 1. order check, run start per timestamp, start of the invalid-timestamp tail
-__global__ void __launch_bounds__(256) freq_scan_kernel(const __grid_constant__ FreqParams q) {
+// ---------------------------------------------------------------- 1. events
+__global__ void __launch_bounds__(kFT) freq_order_kernel(const __grid_constant__ FreqParams q) {
   const AttrParams& p = q.a;
   const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
   for (uint64_t i = tid; i < p.n; i += nth) {
     const uint32_t t = ts_of(p, i);
-    const uint32_t tp = i ? ts_of(p, i - 1) : 0u;
-    if (i && t < tp) atomicOr(q.state, 1u);
-    if (i == 0 || t != tp) {
-      if (t < p.n_api) q.run_start[t] = i;
-      else atomicMin(reinterpret_cast<unsigned long long*>(q.run_start + p.n_api), (unsigned long long)i);
-    }
-  }
-  if (tid == 0 && p.n && ts_of(p, 0) < q.state[1]) atomicOr(q.state, 1u);
-}
-
-// 1b. one block: ordered compaction of the run starts into segments
-__global__ void __launch_bounds__(1024) freq_plan_kernel(const __grid_constant__ FreqParams q) {
-  __shared__ uint32_t s_w[32];
-  const AttrParams& p = q.a;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  if (*reinterpret_cast<volatile uint32_t*>(q.state)) return;     // unsorted: ctl stays zero
-  const uint32_t n_api = p.n_api;
-  uint64_t base = 0;
-  for (uint64_t c0 = 0; c0 < n_api; c0 += blockDim.x) {
-    const uint64_t t = c0 + threadIdx.x;
-    const uint64_t v = t < n_api ? q.run_start[t] : kNone64;
-    const bool has = v != kNone64;
-    const unsigned bal = __ballot_sync(0xffffffffu, has);
-    if (lane == 0) s_w[warp] = __popc(bal);
-    __syncthreads();
-    uint32_t before = 0, round = 0;
-    for (int w = 0; w < nw; ++w) { if (w < warp) before += s_w[w]; round += s_w[w]; }
-    before += __popc(bal & ((1u << lane) - 1));
-    if (has) {
-      q.segs[base + before] = v;
-      q.seg_of_ts[t] = uint32_t(base + before);
-    }
-    base += round;
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    const uint64_t tail = q.run_start[n_api];
-    const uint64_t end_valid = tail == kNone64 ? p.n : tail;
-    q.segs[base] = end_valid;
-    q.ctl->n_segs = base;
-    q.ctl->end_valid = end_valid;
-    q.state[1] = ts_of(p, p.n - 1);
+    if (i ? t < ts_of(p, i - 1) : (q.state[1] && uint64_t(t) + 1 < q.state[1])) atomicOr(q.state, 1u);
   }
 }
 
-__device__ __forceinline__ bool is_boundary(uint64_t k, uint64_t n_segs) { return k == 0 || k + 1 == n_segs; }
-
-// 2. records and element touches per slot (interior segments only)
-__global__ void __launch_bounds__(256) freq_count_kernel(const __grid_constant__ FreqParams q) {
+__global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant__ FreqParams q) {
   __shared__ uint64_t s_l1[kL1MaxKeys];
   const AttrParams& p = q.a;
   for (uint32_t j = threadIdx.x; j < p.n_l1; j += blockDim.x) s_l1[j] = p.l1[j];
   __syncthreads();
-  const uint64_t n_segs = q.ctl->n_segs, end = q.ctl->end_valid;
+  const int lane = threadIdx.x & 31;
+  uint64_t* out = keys_buf(q, uint32_t(q.ctl[1]));
   // each warp walks one contiguous chunk (lane caches stay on one object)
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
   const uint64_t gw = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
-  const uint64_t chunk = ((end + nwarps - 1) / nwarps + 31) / 32 * 32;
-  const uint64_t w_lo = min(end, gw * chunk), w_hi = min(end, w_lo + chunk);
+  const uint64_t chunk = ((p.n + nwarps - 1) / nwarps + 31) / 32 * 32;
+  const uint64_t w_lo = min(p.n, gw * chunk), w_hi = min(p.n, w_lo + chunk);
   LaneObj c;
-  for (uint64_t i = w_lo + (threadIdx.x & 31); i < w_lo + (w_hi - w_lo + 31) / 32 * 32; i += 32) {
-    const uint64_t end_ = w_hi;
-    unsigned long long slot = kNone64;
-    uint64_t touches = 0;
-    uint32_t k = 0;
-    if (i < end_) {
+  for (uint64_t i0 = w_lo; i0 < w_hi; i0 += 32) {     // warp-uniform trip count
+    const uint64_t i = i0 + lane;
+    bool valid = false;
+    uint64_t g0 = 0, g1 = 0;
+    uint32_t rank = kNone;
+    if (i < w_hi) {
       const uint32_t t = ts_of(p, i);
-      const uint32_t rank = p.acc_rank[t];
-      Touch tc;
-      if (rank != kNone) {
-        k = q.seg_of_ts[t];
-        if (!is_boundary(k, n_segs) && resolve(q, s_l1, c, i, t, rank, tc)) {
-          slot = tc.slot;
-          touches = tc.g1 - tc.g0 + 1;
-        }
+      if (t < p.n_api) {
+        rank = __ldg(p.acc_rank + t);
+        valid = rank != kNone && resolve(q, s_l1, c, i, t, g0, g1);
       }
     }
-    const unsigned grp = __match_any_sync(0xffffffffu, slot);
-    const uint32_t lo16 = __reduce_add_sync(grp, uint32_t(touches & 0xFFFF));
-    const uint32_t hi16 = __reduce_add_sync(grp, uint32_t(touches >> 16));
-    if (slot != kNone64 && int(threadIdx.x & 31) == __ffs(grp) - 1) {
-      const uint32_t old = atomicAdd(q.slot_recs + slot, uint32_t(__popc(grp)));
-      atomicAdd(q.slot_touch + slot, (unsigned long long)hi16 * 65536ull + lo16);
-      if (old == 0) {
-        const unsigned long long at = atomicAdd(&q.ctl->n_list, 1ull);
-        q.slot_list[at] = FreqSlotSeg{slot, k, 0};
-      }
+    // merge chains of adjacent, disjoint intervals of one object and API
+    const uint32_t obj = valid ? c.obj : kNone;
+    const uint64_t pg1 = __shfl_up_sync(FULL_MASK, g1, 1);
+    const uint32_t prk = __shfl_up_sync(FULL_MASK, rank, 1);
+    const uint32_t pob = __shfl_up_sync(FULL_MASK, obj, 1);
+    const uint32_t vb = __ballot_sync(FULL_MASK, valid);
+    const bool pv = lane > 0 && ((vb >> (lane - 1)) & 1u);
+    const bool chain = valid && pv && prk == rank && pob == obj && g0 == pg1 + 1;
+    const uint32_t cb = __ballot_sync(FULL_MASK, chain);
+    const bool head = valid && !chain;
+    const bool tail = valid && (lane == 31 || !((cb >> (lane + 1)) & 1u));
+    const uint32_t hb = __ballot_sync(FULL_MASK, head), tb = __ballot_sync(FULL_MASK, tail);
+    const uint32_t cnt = __popc(hb) + __popc(tb);
+    if (!cnt) continue;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(&q.ctl[0], (unsigned long long)cnt);
+    base = __shfl_sync(FULL_MASK, base, 0);
+    if (base + cnt > q.cap) {                        // capacity exceeded: flagged, results invalid
+      if (lane == 0) atomicOr(q.state, 2u);
+      continue;
     }
+    const uint32_t lt = (1u << lane) - 1u;
+    const uint64_t hi = uint64_t(rank) << q.pos_bits;
+    if (head) out[base + __popc(hb & lt)] = hi | (2 * g0);
+    if (tail) out[base + __popc(hb) + __popc(tb & lt)] = hi | (2 * g1 + 1);
   }
 }
 
-// 2b. touches that need a table, per segment (slots with more than one record)
-__global__ void __launch_bounds__(256) freq_slotseg_kernel(const __grid_constant__ FreqParams q) {
-  const uint64_t n = q.ctl->n_list;
-  for (uint64_t j = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; j < n; j += uint64_t(gridDim.x) * blockDim.x) {
-    const FreqSlotSeg e = q.slot_list[j];
-    if (q.slot_recs[e.slot] > 1) atomicAdd(q.seg_touch + e.seg, q.slot_touch[e.slot]);
-  }
-}
-
-// 3. one block: table capacities, prefix sum, batches, the ordered list of solo segments
-__global__ void __launch_bounds__(1024) freq_table_plan_kernel(const __grid_constant__ FreqParams q) {
-  __shared__ unsigned long long s_w[32];
-  __shared__ uint32_t s_c[32];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const uint64_t n_segs = q.ctl->n_segs;
-  const uint64_t B = q.budget;
-  unsigned long long base = 0;
-  uint64_t n_solo = 0;
-  for (uint64_t c0 = 0; c0 < n_segs; c0 += blockDim.x) {
-    const uint64_t k = c0 + threadIdx.x;
-    bool solo = false;
-    unsigned long long cap = 0;
-    uint32_t logc = 0;
-    if (k < n_segs) {
-      solo = is_boundary(k, n_segs);
-      const unsigned long long touch = q.seg_touch[k];
-      if (!solo && touch) {
-        const unsigned long long want = max(2ull * touch, 64ull);
-        logc = 64 - __clzll(want - 1);
-        cap = 1ull << logc;
-        if (cap > B) { solo = true; cap = 0; logc = 0; }
-      }
-    }
-    unsigned long long v = cap;                       // inclusive warp scan
-    for (int d = 1; d < 32; d <<= 1) {
-      const unsigned long long u = __shfl_up_sync(0xffffffffu, v, d);
-      if (lane >= d) v += u;
-    }
-    if (lane == 31) s_w[warp] = v;
-    const unsigned sb = __ballot_sync(0xffffffffu, solo);
-    if (lane == 0) s_c[warp] = __popc(sb);
+// ---------------------------------------------------------------- 2. radix sort
+// (a) tile histograms of digit d, digit-major: hist[digit * ntiles + tile];
+// totals per digit for the skip test
+__global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
+  __shared__ uint32_t s_h[256];
+  const uint64_t n = n_keys(q);
+  const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
+  const uint64_t* src = keys_buf(q, buf_before(q, d));
+  const uint32_t shift = 8 * d;
+  for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    s_h[threadIdx.x] = 0;
     __syncthreads();
-    unsigned long long before = 0, round = 0;
-    uint32_t sbefore = 0, sround = 0;
-    for (int w = 0; w < nw; ++w) {
-      if (w < warp) { before += s_w[w]; sbefore += s_c[w]; }
-      round += s_w[w];
-      sround += s_c[w];
-    }
-    if (k < n_segs) {
-      if (solo) {
-        q.solo[n_solo + sbefore + __popc(sb & ((1u << lane) - 1))] = uint32_t(k);
-        q.seg_logcap[k] = kFreqSolo;
-      } else {
-        const unsigned long long my_base = base + before + v - cap;
-        const uint64_t batch = my_base / B;
-        const uint64_t off = my_base - batch * B;
-        q.seg_logcap[k] = uint8_t(logc);
-        q.seg_off[k] = off;
-        if (batch < q.max_batches) {
-          atomicMax(q.batch_extent + batch, (unsigned long long)(off + cap));
-          atomicMin(q.batch_first + batch, uint32_t(k));
-          atomicMax(&q.ctl->n_batches, (unsigned long long)(batch + 1));
-        } else {
-          atomicOr(q.state, 2u);                       // table plan overflow
-        }
-      }
+    const uint64_t t0 = tile * kFreqTileKeys;
+#pragma unroll 4
+    for (uint32_t k = 0; k < kFreqTileKeys / kFT; ++k) {
+      const uint64_t idx = t0 + k * kFT + threadIdx.x;
+      if (idx < n) atomicAdd(&s_h[(src[idx] >> shift) & 255u], 1u);
     }
     __syncthreads();
-    base += round;
-    n_solo += sround;
+    const uint32_t v = s_h[threadIdx.x];
+    q.hist[uint64_t(threadIdx.x) * ntiles + tile] = v;
+    if (v) atomicAdd(&q.ctl[16 + threadIdx.x], (unsigned long long)v);
+    __syncthreads();
   }
-  if (threadIdx.x == 0) q.ctl->n_solo = n_solo;
 }
 
-struct ApplyShared {
-  BlkAcc blk;
-  uint64_t l1[kL1MaxKeys];
+// block-wide exclusive scan of one value per thread (kFT threads)
+__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* s_w, uint32_t& total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL_MASK, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_w[w] = x;
+  __syncthreads();
+  uint32_t before = 0;
+  total = 0;
+#pragma unroll
+  for (int k = 0; k < kFT / 32; ++k) {
+    const uint32_t s = s_w[k];
+    before += k < w ? s : 0u;
+    total += s;
+  }
+  __syncthreads();
+  return before + x - v;
+}
+
+// (b) exclusive scan of hist (digit-major) in blocks of kFreqScanItems -> offs,
+// block sums -> part; block 0 also decides whether pass d can be skipped
+__global__ void __launch_bounds__(kFT) freq_scan_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
+  __shared__ uint32_t s_w[kFT / 32];
+  const uint64_t n = n_keys(q);
+  const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
+  const uint64_t E = 256 * ntiles;
+  const uint64_t nb = (E + kFreqScanItems - 1) / kFreqScanItems;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    bool skip = n == 0;
+    for (int k = 0; k < 256 && !skip; ++k) skip = q.ctl[16 + k] == n;
+    q.ctl[8 + d] = skip ? 1ull : 0ull;
+  }
+  constexpr uint32_t kI = kFreqScanItems / kFT;
+  for (uint64_t b = blockIdx.x; b < nb; b += gridDim.x) {
+    const uint64_t e0 = b * kFreqScanItems + uint64_t(threadIdx.x) * kI;
+    uint32_t v[kI], sum = 0;
+#pragma unroll
+    for (uint32_t k = 0; k < kI; ++k) { v[k] = e0 + k < E ? q.hist[e0 + k] : 0u; sum += v[k]; }
+    uint32_t total;
+    uint32_t run = block_excl_scan(sum, s_w, total);
+#pragma unroll
+    for (uint32_t k = 0; k < kI; ++k) {
+      if (e0 + k < E) q.offs[e0 + k] = run;
+      run += v[k];
+    }
+    if (threadIdx.x == 0) q.part[b] = total;
+  }
+}
+
+// (c) one block: exclusive scan of part[0, nb) in place (mode 0: the radix
+// digit-offset blocks of pass d; mode 1: the sweep chunks of [0, split),
+// signed sums)
+__global__ void __launch_bounds__(1024) freq_part_scan_kernel(const __grid_constant__ FreqParams q, uint32_t mode,
+                                                              uint32_t d) {
+  __shared__ long long s_w[32];
+  uint64_t nb;
+  if (mode == 0) {
+    if (q.ctl[8 + d]) return;
+    const uint64_t n = n_keys(q);
+    const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
+    nb = (256 * ntiles + kFreqScanItems - 1) / kFreqScanItems;
+  } else {
+    nb = (q.ctl[2] + kSweepChunk - 1) / kSweepChunk;
+  }
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  long long carry = 0;
+  for (uint64_t c0 = 0; c0 < nb; c0 += blockDim.x) {
+    const uint64_t i = c0 + threadIdx.x;
+    long long v = 0;
+    if (i < nb) v = mode == 0 ? (long long)q.part[i] : (long long)(int32_t)q.part[i];
+    long long x = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const long long y = __shfl_up_sync(FULL_MASK, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) s_w[w] = x;
+    __syncthreads();
+    long long before = 0, total = 0;
+    for (int k = 0; k < int(blockDim.x / 32); ++k) { before += k < w ? s_w[k] : 0; total += s_w[k]; }
+    __syncthreads();
+    if (i < nb) q.part[i] = uint32_t(carry + before + x - v);
+    carry += total;
+  }
+}
+
+// (d) stable scatter of pass d: each tile's keys are ranked by digit in
+// shared memory (warp match + per-warp digit counts in warp order, 16
+// sub-chunks of 256 keys in key order), then stored digit run by digit run
+__global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
+  __shared__ uint64_t s_keys[kFreqTileKeys];
+  __shared__ uint32_t s_wc[kFT / 32][256];
+  __shared__ uint32_t s_start[256], s_run[256], s_goff[256], s_w[kFT / 32];
+  if (q.ctl[8 + d]) return;                          // every key has the same digit: pass skipped
+  const uint64_t n = n_keys(q);
+  const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
+  const uint32_t src_b = buf_before(q, d);
+  const uint64_t* src = keys_buf(q, src_b);
+  uint64_t* dst = keys_buf(q, src_b ^ 1u);
+  const uint32_t shift = 8 * d;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const uint64_t e = uint64_t(threadIdx.x) * ntiles + tile;
+    const uint32_t cnt = q.hist[e];
+    s_goff[threadIdx.x] = q.offs[e] + q.part[e / kFreqScanItems];
+    uint32_t tot;
+    s_start[threadIdx.x] = block_excl_scan(cnt, s_w, tot);
+    s_run[threadIdx.x] = 0;
+    const uint64_t t0 = tile * kFreqTileKeys;
+    for (uint32_t sub = 0; sub < kFreqTileKeys / kFT; ++sub) {
+#pragma unroll
+      for (int w = 0; w < kFT / 32; ++w) s_wc[w][threadIdx.x] = 0;
+      __syncthreads();
+      const uint64_t idx = t0 + sub * kFT + threadIdx.x;
+      const bool valid = idx < n;
+      const uint64_t key = valid ? src[idx] : 0ull;
+      const uint32_t dg = uint32_t(key >> shift) & 255u;
+      const uint32_t peers = __match_any_sync(FULL_MASK, valid ? dg : 256u + uint32_t(lane));
+      const uint32_t rk = __popc(peers & lt);
+      if (valid && rk == 0) s_wc[warp][dg] = __popc(peers);
+      __syncthreads();
+      uint32_t run = s_run[threadIdx.x];
+#pragma unroll
+      for (int w = 0; w < kFT / 32; ++w) {
+        const uint32_t v = s_wc[w][threadIdx.x];
+        s_wc[w][threadIdx.x] = run;
+        run += v;
+      }
+      s_run[threadIdx.x] = run;
+      __syncthreads();
+      if (valid) s_keys[s_start[dg] + s_wc[warp][dg] + rk] = key;
+      __syncthreads();
+    }
+    const uint32_t tn = uint32_t(min(uint64_t(kFreqTileKeys), n - t0));
+    for (uint32_t j = threadIdx.x; j < tn; j += kFT) {
+      const uint64_t key = s_keys[j];
+      const uint32_t dg = uint32_t(key >> shift) & 255u;
+      dst[s_goff[dg] + (j - s_start[dg])] = key;
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------- 3. sweep
+// split = first key of the call's last API (carried to the next call);
+// queries (mode 1) sweep every key
+__global__ void freq_split_kernel(const __grid_constant__ FreqParams q, uint32_t mode) {
+  const uint64_t n = n_keys(q);
+  if (q.state[0] & 2u) { q.ctl[2] = 0; return; }     // capacity exceeded: nothing is valid
+  if (mode == 1 || n == 0) { q.ctl[2] = n; return; }
+  const uint64_t* k = keys_buf(q, buf_before(q, q.n_digits));
+  const uint64_t target = (k[n - 1] >> q.pos_bits) << q.pos_bits;
+  uint64_t lo = 0, hi = n;
+  while (lo < hi) { const uint64_t m = (lo + hi) / 2; if (k[m] < target) lo = m + 1; else hi = m; }
+  q.ctl[2] = lo;
+}
+
+__device__ __forceinline__ int ev_sign(uint64_t key) { return (key & 1ull) ? -1 : 1; }
+
+// per chunk of kSweepChunk keys of [0, split): sum of the +1 / -1 events
+__global__ void __launch_bounds__(kFT) freq_sweep_sum_kernel(const __grid_constant__ FreqParams q) {
+  __shared__ uint32_t s_w[kFT / 32];
+  const uint64_t split = q.ctl[2];
+  const uint64_t* k = keys_buf(q, buf_before(q, q.n_digits));
+  const uint64_t nb = (split + kSweepChunk - 1) / kSweepChunk;
+  for (uint64_t b = blockIdx.x; b < nb; b += gridDim.x) {
+    const uint64_t i0 = b * kSweepChunk + uint64_t(threadIdx.x) * kSweepItems;
+    int s = 0;
+#pragma unroll
+    for (uint32_t j = 0; j < kSweepItems; ++j) if (i0 + j < split) s += ev_sign(k[i0 + j]);
+    uint32_t total;
+    block_excl_scan(uint32_t(s), s_w, total);
+    if (threadIdx.x == 0) q.part[b] = total;
+  }
+}
+
+struct SlotSum {
+  uint64_t slot = ~0ull, n = 0, s1 = 0, s2 = 0;
+  __device__ void flush(unsigned long long* acc) {
+    if (slot != ~0ull && n) {
+      atomicAdd(acc + 3 * slot, (unsigned long long)n);
+      atomicAdd(acc + 3 * slot + 1, (unsigned long long)s1);
+      atomicAdd(acc + 3 * slot + 2, (unsigned long long)s2);
+    }
+    n = s1 = s2 = 0;
+  }
 };
 
-__global__ void __launch_bounds__(kFreqThreads, 2) freq_apply_kernel(const __grid_constant__ FreqParams q) {
-  cg::grid_group g = cg::this_grid();
-  __shared__ ApplyShared sh;
-  const AttrParams& p = q.a;
-  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
-  const int lane = threadIdx.x & 31;
-  const uint64_t gwarp = tid >> 5, nwarps = nth >> 5;
-  if (threadIdx.x < kBlkSlots) {
-    sh.blk.slot[threadIdx.x] = ~0ull;
-    sh.blk.n[threadIdx.x] = sh.blk.s1[threadIdx.x] = sh.blk.s2[threadIdx.x] = 0;
-  }
-  for (uint32_t j = threadIdx.x; j < p.n_l1; j += blockDim.x) sh.l1[j] = p.l1[j];
-  __syncthreads();
-  if (*reinterpret_cast<volatile uint32_t*>(q.state)) return;     // uniform across the grid
-  const uint64_t n_segs = q.ctl->n_segs, n_batches = q.ctl->n_batches, n_solo = q.ctl->n_solo;
-  LaneObj c;
-  SlotAcc sa;
-  uint64_t q_done = 0;
-  // a record wider than kFreqInline elements: queued in 4096-element chunks
-  // (tag != 0: cells of a solo segment, else the table of segment `seg`)
-  auto counter = [&](uint32_t tag, uint32_t seg) {
-    Counter ct;
-    ct.cells = q.cells;
-    ct.tag = tag;
-    ct.lc = tag ? 0u : q.seg_logcap[seg];
-    ct.tb = tag ? q.table : q.table + q.seg_off[seg];
-    return ct;
-  };
-  // a record wider than kFreqInline elements: queued in kFreqChunk-element
-  // chunks (tag != 0: cells of a solo segment, else the table of segment `seg`)
-  auto queue_range = [&](const Touch& tc, uint32_t tag, uint32_t seg) {
-    const uint64_t nch = (tc.g1 - tc.g0) / kFreqChunk + 1;
-    const unsigned long long s0 = atomicAdd(&q.ctl->q_count, (unsigned long long)nch);
-    for (uint64_t j = 0; j < nch; ++j) {
-      const uint64_t l0 = tc.g0 + j * kFreqChunk, h0 = min(tc.g1, l0 + kFreqChunk - 1);
-      if (s0 + j < q.q_cap) {
-        q.q[s0 + j] = FreqChunk{l0, h0, tc.slot, tag, seg};
-      } else {
-        const uint64_t sl = tc.slot;
-        auto add = [&](uint32_t pv) { sa.add(sh.blk, q.acc, sl, pv); };
-        counter(tag, seg).range(add, l0, h0, 1);
+// the runs: from key i (count c after it) to key i+1, len = ceil(p_{i+1}/2)
+// - ceil(p_i/2) elements with frequency c in the API of key i
+__global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__ FreqParams q,
+                                                         unsigned long long* acc) {
+  __shared__ uint32_t s_w[kFT / 32];
+  const uint64_t split = q.ctl[2];
+  const uint64_t* k = keys_buf(q, buf_before(q, q.n_digits));
+  const uint64_t nb = (split + kSweepChunk - 1) / kSweepChunk;
+  const uint64_t pmask = (1ull << q.pos_bits) - 1;
+  uint64_t c_lo = 1, c_hi = 0, c_sb = 0;          // cached object's element range, slot base, r_lo
+  uint32_t c_rlo = 0;
+  SlotSum ss;
+  for (uint64_t b = blockIdx.x; b < nb; b += gridDim.x) {
+    const uint64_t i0 = b * kSweepChunk + uint64_t(threadIdx.x) * kSweepItems;
+    uint64_t kk[kSweepItems + 1];
+    int s = 0;
+#pragma unroll
+    for (uint32_t j = 0; j <= kSweepItems; ++j) kk[j] = i0 + j < split ? k[i0 + j] : ~0ull;
+#pragma unroll
+    for (uint32_t j = 0; j < kSweepItems; ++j) if (kk[j] != ~0ull) s += ev_sign(kk[j]);
+    uint32_t total;
+    int c = int(q.part[b]) + int(block_excl_scan(uint32_t(s), s_w, total));
+#pragma unroll
+    for (uint32_t j = 0; j < kSweepItems; ++j) {
+      if (kk[j] == ~0ull) break;
+      c += ev_sign(kk[j]);
+      if (c <= 0 || kk[j + 1] == ~0ull) continue;   // c > 0: the next key belongs to the same API
+      const uint64_t p0 = kk[j] & pmask, p1 = kk[j + 1] & pmask;
+      const uint64_t x0 = (p0 + 1) >> 1, x1 = (p1 + 1) >> 1;
+      if (x1 <= x0) continue;
+      const uint64_t len = x1 - x0;
+      if (!(x0 >= c_lo && x0 < c_hi)) {             // object of element x0: binary search
+        uint32_t lo = 0, hi = uint32_t(q.n_obj);
+        while (hi - lo > 1) { const uint32_t m = (lo + hi) >> 1; if (q.elem_base[m] <= x0) lo = m; else hi = m; }
+        const DevObj dv = q.a.objs[lo];
+        c_lo = q.elem_base[lo];
+        c_hi = c_lo + ((dv.end - dv.base) >> dv.shift);
+        c_sb = q.slot_base[lo];
+        c_rlo = dv.r_lo;
       }
+      const uint64_t slot = c_sb + ((kk[j] >> q.pos_bits) - c_rlo);
+      if (slot != ss.slot) { ss.flush(acc); ss.slot = slot; }
+      const uint64_t cu = uint64_t(c);
+      ss.n += len;
+      ss.s1 += cu * len;
+      ss.s2 += cu * cu * len;
     }
-  };
-  // this phase's queued chunks, grid-wide, one warp per chunk
-  auto drain = [&]() {
-    g.sync();
-    const unsigned long long raw = *reinterpret_cast<volatile unsigned long long*>(&q.ctl->q_count);
-    const uint64_t qc = raw < q.q_cap ? raw : q.q_cap;
-    for (uint64_t e = q_done + gwarp; e < qc; e += nwarps) {
-      const FreqChunk fr = q.q[e];
-      const uint64_t sl = fr.slot;
-      auto add = [&](uint32_t pv) { sa.add(sh.blk, q.acc, sl, pv); };
-      if (fr.g_lo + lane <= fr.g_hi) counter(fr.tag, fr.seg).range(add, fr.g_lo + lane, fr.g_hi, 32);
-    }
-    q_done = raw;
-    g.sync();
-  };
+  }
+  ss.flush(acc);
+}
 
-  // 4a. batches of interior segments with per-API tables, all segments of a batch at once
-  for (uint64_t b = 0; b < n_batches; ++b) {
-    const uint32_t f = q.batch_first[b];
-    if (f == kNone) continue;
-    uint64_t nxt = n_segs;
-    for (uint64_t b2 = b + 1; b2 < n_batches; ++b2)
-      if (q.batch_first[b2] != kNone) { nxt = q.batch_first[b2]; break; }
-    const uint64_t rec_lo = q.segs[f], rec_hi = q.segs[nxt];
-    const uint64_t ext = q.batch_extent[b];
-    uint4* tz = reinterpret_cast<uint4*>(q.table);
-    for (uint64_t e = tid; e < ext; e += nth) tz[e] = make_uint4(0, 0, 0, 0);
-    g.sync();
-    uint32_t c_t = kNever, c_rank = kNone, c_k = 0;
-    uint8_t c_lc = 0;
-    FreqEntry* c_tb = q.table;
-    const uint64_t chunk = ((rec_hi - rec_lo + nwarps - 1) / nwarps + 31) / 32 * 32;
-    const uint64_t w_lo = min(rec_hi, rec_lo + gwarp * chunk), w_hi = min(rec_hi, w_lo + chunk);
-    for (uint64_t i0 = w_lo; i0 < w_hi; i0 += 32) {         // contiguous per warp, warp-uniform
-      const uint64_t i = i0 + lane;
-      Touch tc;
-      bool tbl = false;
-      if (i < w_hi) {
-        const uint32_t t = ts_of(p, i);
-        if (t != c_t) {
-          c_t = t;
-          c_rank = p.acc_rank[t];
-          c_k = q.seg_of_ts[t];
-          c_lc = q.seg_logcap[c_k];
-          c_tb = q.table + q.seg_off[c_k];
-        }
-        if (c_rank != kNone && c_lc != kFreqSolo && resolve(q, sh.l1, c, i, t, c_rank, tc)) {
-          if (q.slot_recs[tc.slot] == 1)                   // the slot's only record
-            sa.add_once(sh.blk, q.acc, tc.slot, tc.g1 - tc.g0 + 1);
-          else if (tc.g1 - tc.g0 < kFreqInline)
-            tbl = true;
-          else
-            queue_range(tc, 0u, c_k);
-        }
-      }
-      // table touches, element by element, lanes hitting the same (table,
-      // element) merged into one add (hot elements of random bursts)
-      const uint64_t len = tbl ? tc.g1 - tc.g0 + 1 : 0;
-      const uint32_t max_len = __reduce_max_sync(0xffffffffu, uint32_t(len));
-      for (uint32_t j = 0; j < max_len; ++j) {
-        const unsigned long long key = j < len ? tc.g0 + j + 1 : 0ull;
-        const unsigned grp = __match_any_sync(0xffffffffu, key) & __match_any_sync(0xffffffffu, c_k);
-        const int leader = __ffs(grp) - 1;
-        uint32_t base = 0;
-        if (key && lane == leader) base = tbl_add(c_tb, c_lc, key, __popc(grp));
-        base = __shfl_sync(0xffffffffu, base, leader);
-        if (key) sa.add(sh.blk, q.acc, tc.slot, base + __popc(grp & ((1u << lane) - 1)));
-      }
-    }
-    drain();
+// ---------------------------------------------------------------- 4. carry
+__global__ void __launch_bounds__(kFT) freq_carry_kernel(const __grid_constant__ FreqParams q) {
+  const uint64_t n = n_keys(q), split = q.ctl[2];
+  const uint32_t b = buf_before(q, q.n_digits);
+  const uint64_t* src = keys_buf(q, b);
+  uint64_t* dst = keys_buf(q, b ^ 1u);
+  for (uint64_t i = split + uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n;
+       i += uint64_t(gridDim.x) * blockDim.x)
+    dst[i - split] = src[i];
+}
+
+__global__ void freq_carry_ctl_kernel(const __grid_constant__ FreqParams q) {
+  const uint64_t n = n_keys(q), split = q.ctl[2];
+  const uint32_t b = buf_before(q, q.n_digits);
+  q.ctl[0] = n - split;
+  q.ctl[1] = b ^ 1u;
+  for (int d = 0; d < 8; ++d) q.ctl[8 + d] = 0;
+  if (q.a.n) q.state[1] = ts_of(q.a, q.a.n - 1) + 1u;
+}
+
+// ---------------------------------------------------------------- launchers
+static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& launches) {
+  const unsigned g = unsigned(num_sms) * 4;
+  for (uint32_t d = 0; d < q.n_digits; ++d) {
+    cudaMemsetAsync(q.ctl + 16, 0, 8 * 256, s);
+    freq_hist_kernel<<<g, kFT, 0, s>>>(q, d);
+    freq_scan_kernel<<<g, kFT, 0, s>>>(q, d);
+    freq_part_scan_kernel<<<1, 1024, 0, s>>>(q, 0, d);
+    freq_scatter_kernel<<<g, kFT, 0, s>>>(q, d);
+    launches += 4;
   }
-  // 4b. solo segments (call boundaries, oversized tables), one at a time, in trace order
-  for (uint64_t s = 0; s < n_solo; ++s) {
-    const uint32_t k = q.solo[s];
-    const uint64_t rec_lo = q.segs[k], rec_hi = q.segs[k + 1];
-    const uint32_t t = ts_of(p, rec_lo);
-    const uint32_t rank = p.acc_rank[t];
-    if (rank == kNone) continue;
-    const uint32_t tag = rank + 1;
-    const uint64_t chunk = ((rec_hi - rec_lo + nwarps - 1) / nwarps + 31) / 32 * 32;
-    const uint64_t w_lo = min(rec_hi, rec_lo + gwarp * chunk), w_hi = min(rec_hi, w_lo + chunk);
-    for (uint64_t i = w_lo + lane; i < w_hi; i += 32) {
-      Touch tc;
-      if (!resolve(q, sh.l1, c, i, t, rank, tc)) continue;
-      if (tc.g1 - tc.g0 < kFreqInline) {
-        const uint64_t sl = tc.slot;
-        auto add = [&](uint32_t pv) { sa.add(sh.blk, q.acc, sl, pv); };
-        counter(tag, k).range(add, tc.g0, tc.g1, 1);
-      } else {
-        queue_range(tc, tag, k);
-      }
-    }
-    drain();
-  }
-  sa.flush(sh.blk, q.acc);
-  blk_flush(sh.blk, q.acc);
+}
+
+static void sweep(const FreqParams& q, unsigned long long* acc, uint32_t mode, int num_sms, cudaStream_t s,
+                  int& launches) {
+  const unsigned g = unsigned(num_sms) * 4;
+  freq_split_kernel<<<1, 1, 0, s>>>(q, mode);
+  freq_sweep_sum_kernel<<<g, kFT, 0, s>>>(q);
+  freq_part_scan_kernel<<<1, 1024, 0, s>>>(q, 1, 0);
+  freq_sweep_kernel<<<g, kFT, 0, s>>>(q, acc);
+  launches += 4;
+}
+
+int launch_frequency(const FreqParams& q, int num_sms, cudaStream_t s) {
+  if (q.a.n == 0) return 0;
+  int launches = 0;
+  uint64_t b = (q.a.n + 255) / 256;
+  if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
+  freq_order_kernel<<<(unsigned)b, kFT, 0, s>>>(q);
+  freq_events_kernel<<<unsigned(num_sms) * 8, kFT, 0, s>>>(q);
+  launches += 2;
+  radix_sort(q, num_sms, s, launches);
+  sweep(q, q.acc, 0, num_sms, s, launches);
+  freq_carry_kernel<<<unsigned(num_sms) * 4, kFT, 0, s>>>(q);
+  freq_carry_ctl_kernel<<<1, 1, 0, s>>>(q);
+  return launches + 2;
+}
+
+int launch_frequency_query(const FreqParams& q, uint64_t n_slots, int num_sms, cudaStream_t s) {
+  int launches = 0;
+  if (n_slots) cudaMemcpyAsync(q.acc_q, q.acc, 24 * n_slots, cudaMemcpyDeviceToDevice, s);
+  // the carried keys are the sorted tail of the last call: swept as they
+  // are, with no radix pass (n_digits = 0 selects the current buffer)
+  FreqParams z = q;
+  z.n_digits = 0;
+  sweep(z, q.acc_q, 1, num_sms, s, launches);
+  return launches;
 }
 
 // per object: the APIs at which it matches NUAF, and the first of them
@@ -575,37 +525,6 @@ __global__ void __launch_bounds__(256) frequency_reduce_kernel(const FreqReduceP
     q.out_count[o] = cnt;
     q.out_first[o] = first;
   }
-}
-
-int frequency_occupancy() {
-  int occ = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, freq_apply_kernel, kFreqThreads, 0);
-  if (occ < 1) occ = 1;
-  return occ > 2 ? 2 : occ;
-}
-
-int launch_frequency(const FreqParams& q, uint64_t n_slots, int num_sms, int occ, cudaStream_t s) {
-  if (q.a.n == 0) return 0;
-  const uint64_t n_api = q.a.n_api;
-  cudaMemsetAsync(q.ctl, 0, sizeof(FreqCtl), s);
-  cudaMemsetAsync(q.run_start, 0xFF, 8 * (n_api + 1), s);
-  cudaMemsetAsync(q.seg_touch, 0, 8 * (n_api + 1), s);
-  cudaMemsetAsync(q.batch_first, 0xFF, 4 * (uint64_t(q.max_batches) + 1), s);
-  cudaMemsetAsync(q.batch_extent, 0, 8 * uint64_t(q.max_batches), s);
-  if (n_slots) {
-    cudaMemsetAsync(q.slot_recs, 0, 4 * n_slots, s);
-    cudaMemsetAsync(q.slot_touch, 0, 8 * n_slots, s);
-  }
-  uint64_t b = (q.a.n + 255) / 256;
-  if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
-  freq_scan_kernel<<<(unsigned)b, 256, 0, s>>>(q);
-  freq_plan_kernel<<<1, 1024, 0, s>>>(q);
-  freq_count_kernel<<<(unsigned)b, 256, 0, s>>>(q);
-  freq_slotseg_kernel<<<num_sms, 256, 0, s>>>(q);
-  freq_table_plan_kernel<<<1, 1024, 0, s>>>(q);
-  void* args[] = {const_cast<FreqParams*>(&q)};
-  cudaLaunchCooperativeKernel((void*)freq_apply_kernel, dim3(num_sms * occ), dim3(kFreqThreads), args, 0, s);
-  return 6;
 }
 
 int launch_frequency_reduce(const FreqReduceParams& q, int num_sms, cudaStream_t s) {

@@ -41,9 +41,8 @@ struct Layout {
   // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end, sa_group;
   // NEXT-2 frequency (feature): cells[sum n_elem], acc[n_slots][3], state, queue, outputs
-  uint64_t fq_cells, fq_acc, fq_state, fq_q, fq_end, fq_slot_base, fq_out_count, fq_out_first;
-  uint64_t fq_ctl, fq_run_start, fq_segs, fq_seg_of_ts, fq_seg_touch, fq_seg_off, fq_seg_logcap, fq_solo;
-  uint64_t fq_batch_first, fq_batch_extent, fq_slot_recs, fq_slot_touch, fq_slot_list, fq_table;
+  uint64_t fq_acc, fq_state, fq_ctl, fq_end, fq_acc_q, fq_slot_base, fq_out_count, fq_out_first;
+  uint64_t fq_keys0, fq_keys1, fq_hist, fq_offs, fq_part;
   uint64_t total;
 };
 
@@ -54,7 +53,7 @@ inline uint64_t align_up(uint64_t x, uint64_t a = kAlign) { return (x + a - 1) /
 struct drgpum_ctx {
   int device = 0;
   int num_sms = 148;
-  int attr_occ = 1, freq_occ = 1;   // blocks per SM of the persistent kernels, on this device
+  int attr_occ = 1;   // blocks per SM of the persistent attribution kernel, on this device
   State state = S_CREATED;
   std::string err;
   uint64_t launches = 0;
@@ -85,6 +84,8 @@ struct drgpum_ctx {
   std::vector<uint64_t> elem_base, slot_base;
   uint64_t n_elem_total = 0, n_slots = 0;
   uint32_t sa_q_cap = 1u << 20;
+  uint64_t fq_recs = 1ull << 24;   // NEXT-2: records per frequency sub-call
+  uint32_t fq_pos_bits = 1, fq_digits = 1;
   std::vector<uint8_t> api_group;   // NEXT-2/3 API group [R22b, R23] (1 = in), mirrored in the workspace
   Layout L{};
   uint8_t* ws = nullptr;
@@ -143,15 +144,12 @@ drgpum_status compute_layout(drgpum_ctx* c);
 drgpum_status gather_accesses(drgpum_ctx* ctx, cudaStream_t st, std::vector<uint64_t>& off,
                               std::vector<uint32_t>& api, std::vector<uint8_t>& rw);
 
-// NEXT-2 per-API hash tables: entries per batch (power of two).  Small
-// enough that a batch's tables stay resident in L2 (random atomics on
-// DRAM-resident lines run at a few G/s), 2^12 .. 2^21 entries (32 MiB; the
-// table region is twice that)
-uint64_t freq_budget(const drgpum_ctx* c) {
-  uint64_t want = std::max<uint64_t>(2 * c->n_elem_total, 1ull << 12), b = 1;
-  while (b < want && b < (1ull << 21)) b <<= 1;
-  return b;
-}
+// NEXT-2 event-key capacity: two keys per record of a sub-call (records of
+// one attribute call are processed in sub-calls of at most fq_recs) plus
+// the carried keys of an API that continues across (sub-)calls.
+uint64_t freq_cap(const drgpum_ctx* c) { return 3 * c->fq_recs; }
+uint64_t freq_max_tiles(const drgpum_ctx* c) { return (freq_cap(c) + kFreqTileKeys - 1) / kFreqTileKeys; }
+uint32_t bits_for(uint64_t v) { uint32_t b = 0; while (b < 64 && (v >> b)) ++b; return b; }
 
 // Build everything derived from (objects, kinds) on the host.
 drgpum_status build_tables(drgpum_ctx* c) {
@@ -299,6 +297,8 @@ drgpum_status build_tables(drgpum_ctx* c) {
   uint64_t eb = 0;
   for (uint64_t i = 0; i < n; ++i) { c->elem_base[i] = eb; eb += c->objs[i].size / c->objs[i].elem_size; }
   c->n_elem_total = eb;
+  c->fq_pos_bits = std::max<uint32_t>(1, bits_for(2 * eb));        // NEXT-2 keys: 2*element (+1)
+  c->fq_digits = (c->fq_pos_bits + bits_for(c->n_acc) + 7) / 8;      // radix passes over (rank, pos)
   c->slot_base.assign(n, 0);
   uint64_t sb = 0;
   for (uint64_t i = 0; i < n; ++i) { c->slot_base[i] = sb; sb += c->n_hit[i]; }
@@ -355,34 +355,22 @@ drgpum_status compute_layout(drgpum_ctx* c) {
     L.sa_end = off;                           // [sa_owner, sa_end) is zeroed per trace
     L.sa_q = put(sizeof(SaRange) * c->sa_q_cap);
   }
-  L.fq_cells = L.fq_acc = L.fq_state = L.fq_q = L.fq_end = off;
-  L.fq_slot_base = L.fq_out_count = L.fq_out_first = off;
-  L.fq_ctl = L.fq_run_start = L.fq_segs = L.fq_seg_of_ts = L.fq_seg_touch = L.fq_seg_off = off;
-  L.fq_seg_logcap = L.fq_solo = L.fq_batch_first = L.fq_batch_extent = off;
-  L.fq_slot_recs = L.fq_slot_touch = L.fq_slot_list = L.fq_table = off;
+  L.fq_acc = L.fq_state = L.fq_ctl = L.fq_end = L.fq_acc_q = L.fq_slot_base = off;
+  L.fq_out_count = L.fq_out_first = L.fq_keys0 = L.fq_keys1 = L.fq_hist = L.fq_offs = L.fq_part = off;
   if (c->features & DRGPUM_FEATURE_FREQUENCY) {
-    L.fq_cells = put(8 * c->n_elem_total);
     L.fq_acc = put(24 * c->n_slots);
     L.fq_state = put(16);
-    L.fq_q = put(sizeof(FreqChunk) * c->sa_q_cap);
-    L.fq_end = off;                           // [fq_cells, fq_end) is zeroed per trace
+    L.fq_ctl = put(8 * 272);
+    L.fq_end = off;                           // [fq_acc, fq_end) is zeroed per trace
+    L.fq_acc_q = put(24 * c->n_slots);
     L.fq_slot_base = put(8 * n);
-    L.fq_ctl = put(sizeof(FreqCtl));
-    L.fq_run_start = put(8 * (uint64_t(c->n_api) + 1));
-    L.fq_segs = put(8 * (uint64_t(c->n_api) + 2));
-    L.fq_seg_of_ts = put(4 * (uint64_t(c->n_api) + 1));
-    L.fq_seg_touch = put(8 * (uint64_t(c->n_api) + 1));
-    L.fq_seg_off = put(8 * (uint64_t(c->n_api) + 1));
-    L.fq_seg_logcap = put(uint64_t(c->n_api) + 1);
-    L.fq_solo = put(4 * (uint64_t(c->n_api) + 1));
-    L.fq_batch_first = put(4 * (uint64_t(kFreqMaxBatches) + 1));
-    L.fq_batch_extent = put(8 * uint64_t(kFreqMaxBatches));
-    L.fq_slot_recs = put(4 * c->n_slots);
-    L.fq_slot_touch = put(8 * c->n_slots);
-    L.fq_slot_list = put(sizeof(FreqSlotSeg) * c->n_slots);
-    L.fq_table = put(2 * sizeof(FreqEntry) * freq_budget(c));
     L.fq_out_count = put(4 * n);
     L.fq_out_first = put(4 * n);
+    L.fq_keys0 = put(8 * freq_cap(c));
+    L.fq_keys1 = put(8 * freq_cap(c));
+    L.fq_hist = put(4 * 256 * freq_max_tiles(c));
+    L.fq_offs = put(4 * 256 * freq_max_tiles(c));
+    L.fq_part = put(4 * (2 * freq_max_tiles(c) + 64));
   }
   L.total = off;
   return DRGPUM_OK;
@@ -438,7 +426,7 @@ drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s, bool dense) {
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     CK(cudaMemsetAsync(ctx->ws + ctx->L.sa_owner, 0, ctx->L.sa_end - ctx->L.sa_owner, s));
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
-    CK(cudaMemsetAsync(ctx->ws + ctx->L.fq_cells, 0, ctx->L.fq_end - ctx->L.fq_cells, s));
+    CK(cudaMemsetAsync(ctx->ws + ctx->L.fq_acc, 0, ctx->L.fq_end - ctx->L.fq_acc, s));
   ctx->final_valid = false;
   ctx->owned = ctx->gathered = false;
   return DRGPUM_OK;
@@ -473,30 +461,31 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
 FreqParams fq_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   FreqParams q;
   q.a = attr_params(c, recs, n);
-  q.cells = at<unsigned long long>(c, c->L.fq_cells);
   q.elem_base = at<uint64_t>(c, c->L.sa_elem_base);
   q.slot_base = at<uint64_t>(c, c->L.fq_slot_base);
   q.acc = at<unsigned long long>(c, c->L.fq_acc);
-  q.q = at<FreqChunk>(c, c->L.fq_q);
-  q.q_cap = c->sa_q_cap;
+  q.acc_q = at<unsigned long long>(c, c->L.fq_acc_q);
   q.state = at<uint32_t>(c, c->L.fq_state);
-  q.ctl = at<FreqCtl>(c, c->L.fq_ctl);
-  q.run_start = at<uint64_t>(c, c->L.fq_run_start);
-  q.segs = at<uint64_t>(c, c->L.fq_segs);
-  q.seg_of_ts = at<uint32_t>(c, c->L.fq_seg_of_ts);
-  q.seg_touch = at<unsigned long long>(c, c->L.fq_seg_touch);
-  q.seg_off = at<uint64_t>(c, c->L.fq_seg_off);
-  q.seg_logcap = at<uint8_t>(c, c->L.fq_seg_logcap);
-  q.solo = at<uint32_t>(c, c->L.fq_solo);
-  q.batch_first = at<uint32_t>(c, c->L.fq_batch_first);
-  q.batch_extent = at<unsigned long long>(c, c->L.fq_batch_extent);
-  q.max_batches = kFreqMaxBatches;
-  q.slot_recs = at<uint32_t>(c, c->L.fq_slot_recs);
-  q.slot_touch = at<unsigned long long>(c, c->L.fq_slot_touch);
-  q.slot_list = at<FreqSlotSeg>(c, c->L.fq_slot_list);
-  q.table = at<FreqEntry>(c, c->L.fq_table);
-  q.budget = freq_budget(c);
+  q.ctl = at<unsigned long long>(c, c->L.fq_ctl);
+  q.keys0 = at<uint64_t>(c, c->L.fq_keys0);
+  q.keys1 = at<uint64_t>(c, c->L.fq_keys1);
+  q.cap = freq_cap(c);
+  q.hist = at<uint32_t>(c, c->L.fq_hist);
+  q.offs = at<uint32_t>(c, c->L.fq_offs);
+  q.part = at<uint32_t>(c, c->L.fq_part);
+  q.max_tiles = freq_max_tiles(c);
+  q.n_obj = c->n_obj;
+  q.pos_bits = c->fq_pos_bits;
+  q.n_digits = c->fq_digits;
   return q;
+}
+
+// the NEXT-2 pass over n device records, in sub-calls of at most fq_recs
+int launch_frequency_calls(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n, cudaStream_t s) {
+  int launches = 0;
+  for (uint64_t i = 0; i < n; i += c->fq_recs)
+    launches += launch_frequency(fq_params(c, recs + i, std::min(c->fq_recs, n - i)), c->num_sms, s);
+  return launches;
 }
 
 SaParams sa_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
@@ -568,7 +557,10 @@ DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx* ctx, uint32_t features)
   if (features & ~uint32_t(DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY))
     return fail(ctx, DRGPUM_EINVAL, "unknown feature bits");
   ctx->features = features;
-  return compute_layout(ctx);
+  drgpum_status r = compute_layout(ctx);
+  if (r == DRGPUM_OK && (features & DRGPUM_FEATURE_FREQUENCY) && 8 * ctx->fq_digits > 64 + 7)
+    return fail(ctx, DRGPUM_EINVAL, "frequency analysis: (API rank, 2 x element) keys exceed 64 bits");
+  return r;
 }
 
 DRGPUM_API drgpum_status drgpum_set_queue_capacity(drgpum_ctx* ctx, uint32_t range_entries,
@@ -580,6 +572,16 @@ DRGPUM_API drgpum_status drgpum_set_queue_capacity(drgpum_ctx* ctx, uint32_t ran
     return fail(ctx, DRGPUM_EINVAL, "queue capacity above 2^24 entries");
   if (range_entries) ctx->rq_cap = range_entries;
   if (aux_entries) ctx->sa_q_cap = aux_entries;
+  return compute_layout(ctx);
+}
+
+DRGPUM_API drgpum_status drgpum_set_frequency_capacity(drgpum_ctx* ctx, uint64_t records_per_call) {
+  if (!ctx) return DRGPUM_EINVAL;
+  if (ctx->state != S_LOADED)
+    return fail(ctx, DRGPUM_ESTATE, "set_frequency_capacity must follow objects_load and precede workspace_bind");
+  if (records_per_call < 1024 || records_per_call > (1ull << 31))
+    return fail(ctx, DRGPUM_EINVAL, "records_per_call outside [1024, 2^31]");
+  ctx->fq_recs = records_per_call;
   return compute_layout(ctx);
 }
 
@@ -644,7 +646,11 @@ static drgpum_status frequency_ready(drgpum_ctx* ctx, cudaStream_t st) {
   CK(cudaMemcpyAsync(state, ctx->ws + ctx->L.fq_state, 8, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   if (state[0] & 1) return fail(ctx, DRGPUM_EINVAL, "frequency analysis needs records in API (timestamp) order");
-  if (state[0]) return fail(ctx, DRGPUM_ENOMEM, "frequency analysis: per-call table plan overflow (split the call)");
+  if (state[0]) return fail(ctx, DRGPUM_ENOMEM, "frequency analysis: one API's events exceed the key capacity "
+                            "(drgpum_set_frequency_capacity)");
+  // the sums including the API carried at the end of the last call
+  ctx->launches += launch_frequency_query(fq_params(ctx, nullptr, 0), ctx->n_slots, ctx->num_sms, st);
+  CK(cudaGetLastError());
   return DRGPUM_OK;
 }
 
@@ -655,7 +661,7 @@ DRGPUM_API drgpum_status drgpum_frequency(drgpum_ctx* ctx, uint32_t pct, uint32_
   drgpum_status r = frequency_ready(ctx, st);
   if (r != DRGPUM_OK) return r;
   FreqReduceParams q;
-  q.acc = at<unsigned long long>(ctx, ctx->L.fq_acc);
+  q.acc = at<unsigned long long>(ctx, ctx->L.fq_acc_q);
   q.slot_base = at<uint64_t>(ctx, ctx->L.fq_slot_base);
   q.n_hit = at<uint32_t>(ctx, ctx->L.n_hit);
   q.objs = at<DevObj>(ctx, ctx->L.objs);
@@ -682,7 +688,7 @@ DRGPUM_API drgpum_status drgpum_frequency_slots(drgpum_ctx* ctx, uint64_t* h_acc
   if (r != DRGPUM_OK) return r;
   *n_slots = ctx->n_slots;
   if (h_acc && ctx->n_slots) {
-    CK(cudaMemcpyAsync(h_acc, ctx->ws + ctx->L.fq_acc, 24 * ctx->n_slots, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(h_acc, ctx->ws + ctx->L.fq_acc_q, 24 * ctx->n_slots, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
   }
   return DRGPUM_OK;
@@ -696,7 +702,7 @@ DRGPUM_API drgpum_status drgpum_slice_frequency(drgpum_ctx* ctx, uint32_t pct, u
   if (r != DRGPUM_OK) return r;
   std::vector<uint64_t> acc(3 * ctx->n_slots);
   if (ctx->n_slots) {
-    CK(cudaMemcpyAsync(acc.data(), ctx->ws + ctx->L.fq_acc, 24 * ctx->n_slots, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(acc.data(), ctx->ws + ctx->L.fq_acc_q, 24 * ctx->n_slots, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
   }
   // [R22b] per object: over the group's accessing APIs A, F_A = S1 of slot
@@ -744,7 +750,6 @@ DRGPUM_API drgpum_status drgpum_workspace_bind(drgpum_ctx* ctx, void* d_ws, uint
   if (s != DRGPUM_OK) return s;
   // per-device kernel attributes and occupancy, kept in the context
   ctx->attr_occ = attribute_occupancy();
-  ctx->freq_occ = frequency_occupancy();
   CK(cudaGetLastError());
   cudaStream_t st = as_stream(stream);
   ctx->ws = static_cast<uint8_t*>(d_ws);
@@ -806,7 +811,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_re
   if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
     ctx->launches += launch_structured(sa_params(ctx, d_recs, n), ctx->num_sms, as_stream(stream));
   if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
-    ctx->launches += launch_frequency(fq_params(ctx, d_recs, n), ctx->n_slots, ctx->num_sms, ctx->freq_occ, as_stream(stream));
+    ctx->launches += launch_frequency_calls(ctx, d_recs, n, as_stream(stream));
   ctx->final_valid = false;
   CK(cudaGetLastError());
   return DRGPUM_OK;
@@ -847,7 +852,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
     if (ctx->features & DRGPUM_FEATURE_STRUCTURED)
       ctx->launches += launch_structured(sa_params(ctx, stage[b], m), ctx->num_sms, st);
     if (ctx->features & DRGPUM_FEATURE_FREQUENCY)
-      ctx->launches += launch_frequency(fq_params(ctx, stage[b], m), ctx->n_slots, ctx->num_sms, ctx->freq_occ, st);
+      ctx->launches += launch_frequency_calls(ctx, stage[b], m, st);
     CK(cudaEventRecord(ctx->ev_used[b], st));
   }
   CK(cudaStreamSynchronize(ctx->copy_stream));

@@ -98,40 +98,38 @@ struct SaParams {
   const uint8_t* in_group;   // [n_api] 1 = the API takes part in the pass [R23]
 };
 
-// NEXT-2 non-uniform access frequency pass (optional feature).
-struct FreqChunk { uint64_t g_lo, g_hi, slot; uint32_t tag, seg; };   // 32 B wide-record chunk
-struct FreqEntry { unsigned long long key, cnt; };                     // 16 B per-API hash entry
-struct FreqSlotSeg { uint64_t slot; uint32_t seg, pad; };
-struct FreqCtl {                 // per call, zeroed before the scan
-  unsigned long long n_segs, end_valid, n_list, q_count, n_batches, n_solo, pad0, pad1;
-};
-constexpr uint8_t kFreqSolo = 0xFF;
-constexpr uint32_t kFreqMaxBatches = 65536;    // seg_logcap: segment counted in the element cells, alone
+// NEXT-2 non-uniform access frequency pass (optional feature), sort-based:
+// every attributed record becomes the element interval it touches, as two
+// event keys (rank << pos_bits) | (2*g0) and (rank << pos_bits) | (2*g1+1)
+// (g = global element index, rank = access-API rank); adjacent disjoint
+// intervals of a warp's consecutive records are merged first.  An LSD radix
+// sort orders the keys by (API, element); a scan of the +1 / -1 events gives
+// every element's count within its API, and each run of equal count c over
+// len elements adds (len, c*len, c*c*len) to its (object, API) slot.  The
+// API of the call's last records may continue in the next call: its events
+// are carried over, sorted, and swept when the next call (or a query)
+// completes it.
+constexpr uint32_t kFreqTileKeys = 4096;        // radix-sort tile (256 threads x 16 keys)
+constexpr uint32_t kFreqScanItems = 2048;       // entries per block of the digit-offset scan
 struct FreqParams {
-  AttrParams a;                  // records, object table, index, rank table
-  unsigned long long* cells;     // [sum n_elem] (API tag << 32) | count within that API (solo segments)
+  AttrParams a;                  // records of this (sub-)call, object table, index, rank table
   const uint64_t* elem_base;     // [n_obj] first global element of each object
   const uint64_t* slot_base;     // [n_obj] first (object, access API) slot of each object
-  unsigned long long* acc;       // [n_slots][3]: n touched elements, S1 = sum f, S2 = sum f^2
-  FreqChunk* q;                  // wide-record chunk queue
-  uint32_t q_cap;
-  uint32_t max_batches;
-  uint32_t* state;               // [0] records not sorted by ts, [1] last ts of the previous call
-  FreqCtl* ctl;
-  uint64_t* run_start;           // [n_api + 1] run start per ts; [n_api] = start of the invalid tail
-  uint64_t* segs;                // [n_api + 2] segment starts, then the end of the valid records
-  uint32_t* seg_of_ts;           // [n_api] segment index of each ts with records in this call
-  unsigned long long* seg_touch; // [n_api + 1] element touches that need the segment's hash table
-  uint64_t* seg_off;             // [n_api + 1] table offset (entries) inside its batch's region
-  uint8_t* seg_logcap;           // [n_api + 1] log2 table capacity, 0 = no table, kFreqSolo
-  uint32_t* solo;                // [n_api + 1] solo segments in trace order
-  uint32_t* batch_first;         // [max_batches + 1] first segment of each batch (kNone if empty)
-  unsigned long long* batch_extent;  // [max_batches] table entries the batch uses
-  uint32_t* slot_recs;           // [n_slots] records per (object, API) slot in this call
-  unsigned long long* slot_touch;    // [n_slots] element touches per slot in this call
-  FreqSlotSeg* slot_list;        // [n_slots] slots touched in this call, with their segment
-  FreqEntry* table;              // [2 * budget] per-API hash tables of one batch
-  uint64_t budget;               // table entries per batch (power of two)
+  unsigned long long* acc;       // [n_slots][3] completed APIs: n, S1 = sum f, S2 = sum f^2
+  unsigned long long* acc_q;     // [n_slots][3] acc + the carried API (written by queries)
+  uint32_t* state;               // [0] bit0 records out of order, bit1 event capacity exceeded;
+                                 // [1] last timestamp of the previous call + 1 (0 = none)
+  unsigned long long* ctl;       // [0] keys in the current buffer, [1] current buffer, [2] split,
+                                 // [3] skip flag of the current radix pass, [4..260) digit totals
+  uint64_t* keys0;               // event keys, ping-pong buffers of cap keys
+  uint64_t* keys1;
+  uint64_t cap;
+  uint32_t* hist;                // [256 * max_tiles] per-tile digit counts
+  uint32_t* offs;                // [256 * max_tiles] exclusive digit offsets (scanned)
+  uint32_t* part;                // [scan blocks] block sums of offs, then of the sweep
+  uint64_t max_tiles;
+  uint64_t n_obj;
+  uint32_t pos_bits, n_digits;
 };
 struct FreqReduceParams {
   const unsigned long long* acc;
@@ -213,10 +211,11 @@ struct GatherParams {
 // Set the kernels' attributes on the CURRENT device and return their
 // resident blocks per SM (called by workspace_bind; cached in the context).
 int attribute_occupancy();
-int frequency_occupancy();
 int launch_attribute(const AttrParams& p, int num_sms, int occ, cudaStream_t s);   // p.rq_slot alternates per call
 int launch_structured(const SaParams& p, int num_sms, cudaStream_t s);
-int launch_frequency(const FreqParams& p, uint64_t n_slots, int num_sms, int occ, cudaStream_t s);
+int launch_frequency(const FreqParams& p, int num_sms, cudaStream_t s);
+// queries: acc_q = acc + the carried API's contributions
+int launch_frequency_query(const FreqParams& p, uint64_t n_slots, int num_sms, cudaStream_t s);
 int launch_frequency_reduce(const FreqReduceParams& p, int num_sms, cudaStream_t s);
 int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s);
 int launch_fill_u32(uint32_t* p, uint32_t v, uint64_t n, cudaStream_t s);

@@ -39,7 +39,7 @@ class Session:
     """
 
     def __init__(self, objects, kinds, device=None, structured=False, frequency=False, workspace_alloc=None,
-                 queue_capacity=None):
+                 queue_capacity=None, frequency_capacity=None):
         if not torch.cuda.is_available():
             raise RuntimeError("drgpum Session needs a CUDA device (there is no CPU fallback)")
         self.L = _lib.load()
@@ -60,6 +60,8 @@ class Session:
         feats = (_lib.FEATURE_STRUCTURED if structured else 0) | (_lib.FEATURE_FREQUENCY if frequency else 0)
         if feats:
             check(self._h, self.L.drgpum_set_features(self._h, feats))
+        if frequency_capacity is not None:   # NEXT-2 records per sub-call
+            check(self._h, self.L.drgpum_set_frequency_capacity(self._h, int(frequency_capacity)))
         if queue_capacity is not None:   # (range entries, aux entries); tests drive the overflow paths
             check(self._h, self.L.drgpum_set_queue_capacity(self._h, *queue_capacity))
         nbytes = ctypes.c_uint64()

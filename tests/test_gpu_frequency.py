@@ -13,9 +13,9 @@ def _sorted(recs):
     return recs[np.argsort(recs["meta"] & 0x7FFFFFFF, kind="stable")]
 
 
-def _check(objs, kinds, recs, chunks=1, pct=20, queue_capacity=None):
+def _check(objs, kinds, recs, chunks=1, pct=20, frequency_capacity=None):
     from paper_conf_asplos_linzs23_b200 import Session
-    s = Session(objs, kinds, frequency=True, queue_capacity=queue_capacity)
+    s = Session(objs, kinds, frequency=True, frequency_capacity=frequency_capacity)
     d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
     b = np.linspace(0, len(recs), chunks + 1).astype(np.int64)
     for x, y in zip(b, b[1:]):
@@ -107,10 +107,24 @@ def test_dependency_chain(seed, chunks):
 
 
 @pytest.mark.parametrize("seed", range(4))
-def test_wide_record_queue_overflow(seed):
-    """Wide records that do not fit the chunk queue (capacity 1) are counted
-    in place by the warp that found them (frequency.cu queue_range)."""
+def test_sub_calls_and_carried_apis(seed):
+    """A small key capacity splits every call into many sub-calls: the API
+    running across each sub-call boundary is carried (sorted keys moved to
+    the other buffer) and completed by the next sub-call or by the query."""
     p = build_tiny(seed)
-    _check(p.objects, p.kinds, _sorted(gen_all_records(p)), queue_capacity=(0, 1))
+    _check(p.objects, p.kinds, _sorted(gen_all_records(p)), frequency_capacity=2048, chunks=3)
     c = build_config("C1")
-    _check(c.objects, c.kinds, _sorted(gen_all_records(c)), queue_capacity=(0, 1))
+    _check(c.objects, c.kinds, _sorted(gen_all_records(c)), frequency_capacity=1 << 16)
+    objs, kinds, r = _chain_program(seed)
+    _check(objs, kinds, r, chunks=1 + seed, frequency_capacity=4096)
+
+
+def test_api_larger_than_capacity_is_refused():
+    """One API whose events exceed the key capacity: ENOMEM at the query
+    (never a silent partial count)."""
+    from paper_conf_asplos_linzs23_b200 import Session, DrgpumError
+    c = build_config("C1")
+    s = Session(c.objects, c.kinds, frequency=True, frequency_capacity=1024)
+    s.attribute(torch.from_numpy(_sorted(gen_all_records(c)).view(np.uint8)).cuda())
+    with pytest.raises(DrgpumError, match="ENOMEM|capacity"):
+        s.frequency()
