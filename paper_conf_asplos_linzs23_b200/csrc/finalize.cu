@@ -495,7 +495,89 @@ constexpr uint32_t kSmemAcc = 8192;
 
 constexpr int kFinThreads = 256;
 
-template <bool kStaged>
+
+// A6 stats + A7 patterns of object o from its bitmap monoid and hit-row
+// summary (one thread)
+__device__ __forceinline__ void emit_object(const FinalParams& p, uint64_t o, const DevObj& ob,
+                                            const BitMonoid& bm, const HitM& hm) {
+  drgpum_object_stats_t* stats = static_cast<drgpum_object_stats_t*>(p.stats);
+  drgpum_pattern_report_t* reps = static_cast<drgpum_pattern_report_t*>(p.reports);
+  // ---- stats (A6)
+  const uint64_t n = (ob.end - ob.base) >> ob.shift;
+  const uint32_t first = p.first[o], last = p.last[o];
+  drgpum_object_stats_t st;
+  st.n_elems = n;
+  st.accessed = bm.pop;
+  st.span_lo = bm.lo;   // kNoPos == UINT64_MAX
+  st.span_hi = bm.hi;
+  st.largest_unaccessed_run = bm.best;
+  st.t_first = first;
+  st.t_last = last;
+  st.n_access_apis = hm.cnt;
+  st._pad = 0;
+  stats[o] = st;
+  // cross-check of the two liveness folds (atomics vs hit rows), and of
+  // bitmap vs hit row (an object with accessed elements has accessing APIs)
+  const bool consistent = bm.len >= n && (bm.pop == 0 || bm.hi < n) &&
+      (hm.cnt ? (first == hm.first_ts && last == hm.last_ts && bm.pop > 0)
+              : (first == kNever && last == 0 && bm.pop == 0));
+  if (!consistent) atomicAdd(&p.ctr[C_CONSISTENCY], 1ull);
+  // ---- patterns (A7)
+  drgpum_pattern_report_t r;
+  r.flags = 0; r.ea_distance = 0; r.ld_distance = 0; r.ti_ranges = 0;
+  r.ti_max_idle = 0; r.dw_pairs = 0; r.ti_total_idle = 0;
+  const bool used = hm.cnt > 0;
+  const bool leak = ob.t_free == kNever;
+  if (!used) r.flags |= DRGPUM_UA;
+  if (leak) r.flags |= DRGPUM_ML;
+  if (used) {
+    if (hm.first_ts - ob.t_alloc >= 2) { r.flags |= DRGPUM_EA; r.ea_distance = hm.first_ts - ob.t_alloc; }
+    if (!leak && ob.t_free - hm.last_ts >= 2) { r.flags |= DRGPUM_LD; r.ld_distance = ob.t_free - hm.last_ts; }
+    r.ti_ranges = hm.ti_cnt; r.ti_max_idle = hm.ti_max; r.ti_total_idle = hm.ti_sum;
+    r.dw_pairs = hm.dw;
+    if (hm.ti_cnt) r.flags |= DRGPUM_TI;
+    if (hm.dw) r.flags |= DRGPUM_DW;
+  }
+  using u128 = unsigned __int128;
+  if (u128(bm.pop) * 100u < u128(p.oa_pct) * n) {
+    r.flags |= DRGPUM_OA;
+    const uint64_t unacc = n - bm.pop;
+    if (unacc == 0 || u128(unacc - bm.best) * 100u < u128(p.frag_pct) * unacc)
+      r.flags |= DRGPUM_OA_ACTIONABLE;
+  }
+  reps[o] = r;
+}
+
+// sequential fold of hit words [w_lo, w_hi) of an object (one lane)
+struct HitFold {
+  uint32_t cnt = 0, f_ts = 0, f_fl = 0, l_ts = 0, l_fl = 0, ti_cnt = 0, ti_max = 0, ti_sum = 0, dw = 0;
+  __device__ __forceinline__ void add(uint32_t ts, uint32_t fl, uint32_t x_ti) {
+    if (cnt == 0) {
+      f_ts = ts; f_fl = fl;
+    } else {
+      const uint32_t gap = ts - l_ts - 1;               // APIs strictly between (R6)
+      if (gap >= x_ti) { ++ti_cnt; ti_max = max(ti_max, gap); ti_sum += gap; }
+      if (l_fl == 3u && fl == 3u) ++dw;                 // Def 3.7, R12
+    }
+    l_ts = ts; l_fl = fl; ++cnt;
+  }
+  template <typename TS, typename CS>
+  __device__ __forceinline__ void words(const uint32_t* row, uint32_t w_lo, uint32_t w_hi, uint32_t r_lo,
+                                        const TS& acc_ts, const CS& acc_cs, uint32_t x_ti) {
+    for (uint32_t wi = w_lo; wi < w_hi; ++wi) {
+      uint32_t w = row[wi];
+      while (w) {
+        const uint32_t j = uint32_t(__ffs(w) - 1) >> 1;    // API slot inside this word
+        const uint32_t pair = (w >> (2 * j)) & 3u;         // bit0 read, bit1 write
+        w &= ~(3u << (2 * j));
+        const uint32_t rank = r_lo + wi * 16 + j;
+        add(acc_ts[rank], (pair >> 1) | (uint32_t(acc_cs[rank]) << 1), x_ti);   // bit0 write, bit1 copy/set
+      }
+    }
+  }
+};
+
+template <bool kStaged, bool kLane>
 __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const FinalParams p) {
   extern __shared__ uint4 s_acc4[];     // [n_acc] ts (padded to 16 B), then [n_acc] cs bytes
   const uint32_t* acc_ts = p.acc_ts;
@@ -515,119 +597,84 @@ __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const Fina
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  drgpum_object_stats_t* stats = static_cast<drgpum_object_stats_t*>(p.stats);
-  drgpum_pattern_report_t* reps = static_cast<drgpum_pattern_report_t*>(p.reports);
-  for (uint64_t o = p.o_lo + gwarp; o < p.o_hi; o += nwarps) {
-    // ---- bitmap groups of o, in order (one load for a single-group object)
-    const uint32_t t0 = p.group_off[o], t1 = p.group_off[o + 1];
-    BitMonoid bm = bm_identity();
-    if (t1 - t0 == 1) {
-      bm = p.group_part[t0];
-    } else {
-      for (uint32_t tb = t0; tb < t1; tb += 32) {
-        BitMonoid m = (tb + lane < t1) ? p.group_part[tb + lane] : bm_identity();
+  // 32 objects per warp step.  Small objects -- one bitmap group and a hit
+  // row of at most kLaneHitWords words (C5's 10^6 objects) -- are finalized
+  // by their own lane, 32 at once (their loads are independent, so the warp
+  // overlaps 32 objects' latencies instead of walking them one by one); the
+  // others one after the other by the whole warp.
+  // kLane = false (mostly large objects, C2): one object per warp step.
+  const uint32_t step = kLane ? 32u : 1u;
+  for (uint64_t o0 = p.o_lo + gwarp * step; o0 < p.o_hi; o0 += nwarps * step) {
+    const uint64_t ol = o0 + lane;
+    bool small = false;
+    if (kLane && ol < p.o_hi) {
+      const uint32_t t0 = p.group_off[ol], t1 = p.group_off[ol + 1];
+      const uint32_t nw = (2 * p.n_hit[ol] + 31) / 32;
+      small = t1 - t0 <= 1 && nw <= kLaneHitWords;
+      if (small) {
+        const DevObj ob = p.objs[ol];
+        const BitMonoid bm = t1 > t0 ? p.group_part[t0] : bm_identity();
+        HitFold f;
+        f.words(p.orw + ob.hit_word, 0, nw, ob.r_lo, acc_ts, acc_cs, p.ti_min_idle);
+        HitM hm = hit_identity();
+        if (f.cnt) hm = HitM{f.cnt, f.f_ts, f.l_ts, 0, f.ti_cnt, f.ti_max, f.dw, f.ti_sum};
+        emit_object(p, ol, ob, bm, hm);
+      }
+    }
+    uint32_t big = kLane ? __ballot_sync(FULL_MASK, ol < p.o_hi && !small) : 1u;
+    while (big) {
+      const uint64_t o = o0 + uint32_t(__ffs(big) - 1);
+      big &= big - 1;
+      // ---- bitmap groups of o, in order
+      const uint32_t t0 = p.group_off[o], t1 = p.group_off[o + 1];
+      BitMonoid bm = bm_identity();
+      if (t1 - t0 == 1) {
+        bm = p.group_part[t0];
+      } else {
+        for (uint32_t tb = t0; tb < t1; tb += 32) {
+          BitMonoid m = (tb + lane < t1) ? p.group_part[tb + lane] : bm_identity();
 #pragma unroll
-        for (int d = 1; d < 32; d <<= 1) m = bm_cat(m, bm_shfl_down(m, d));
-        if (lane == 0) bm = bm_cat(bm, m);
-      }
-    }
-    // ---- hit row of o: 2 bits per access API inside its lifetime.  Each
-    // lane folds a contiguous run of hit words in order (count, first / last
-    // accessing API with its write / copy-set flags, TI gaps and DW pairs
-    // inside the run); the lanes are then joined at their boundaries: the
-    // gap / pair between a lane's first API and the previous non-empty
-    // lane's last one (one indexed shuffle), and warp sums / maxima.
-    const DevObj ob = p.objs[o];
-    const uint32_t nh = p.n_hit[o];
-    const uint32_t nwords = (2 * nh + 31) / 32;
-    const uint32_t per = (nwords + 31) / 32;
-    const uint32_t wlo = min(nwords, lane * per), whi = min(nwords, wlo + per);
-    uint32_t cnt = 0, f_ts = 0, f_fl = 0, l_ts = 0, l_fl = 0, ti_cnt = 0, ti_max = 0, ti_sum = 0, dw = 0;
-    for (uint32_t wi = wlo; wi < whi; ++wi) {
-      uint32_t w = p.orw[ob.hit_word + wi];
-      while (w) {
-        const uint32_t j = uint32_t(__ffs(w) - 1) >> 1;    // API slot inside this word
-        const uint32_t pair = (w >> (2 * j)) & 3u;         // bit0 read, bit1 write
-        w &= ~(3u << (2 * j));
-        const uint32_t rank = ob.r_lo + wi * 16 + j;
-        const uint32_t ts = acc_ts[rank];
-        const uint32_t fl = (pair >> 1) | (uint32_t(acc_cs[rank]) << 1);   // bit0 write, bit1 copy/set
-        if (cnt == 0) {
-          f_ts = ts; f_fl = fl;
-        } else {
-          const uint32_t gap = ts - l_ts - 1;               // APIs strictly between (R6)
-          if (gap >= p.ti_min_idle) { ++ti_cnt; ti_max = max(ti_max, gap); ti_sum += gap; }
-          if (l_fl == 3u && fl == 3u) ++dw;                 // Def 3.7, R12
+          for (int d = 1; d < 32; d <<= 1) m = bm_cat(m, bm_shfl_down(m, d));
+          if (lane == 0) bm = bm_cat(bm, m);
         }
-        l_ts = ts; l_fl = fl; ++cnt;
       }
-    }
-    const uint32_t nz = __ballot_sync(FULL_MASK, cnt != 0);
-    HitM hm = hit_identity();
-    if (nz) {
-      const uint32_t below = nz & ((1u << lane) - 1u);
-      const int pl = below ? 31 - __clz(below) : lane;
-      const uint32_t p_ts = __shfl_sync(FULL_MASK, l_ts, pl);
-      const uint32_t p_fl = __shfl_sync(FULL_MASK, l_fl, pl);
-      if (cnt && below) {
-        const uint32_t gap = f_ts - p_ts - 1;
-        if (gap >= p.ti_min_idle) { ++ti_cnt; ti_max = max(ti_max, gap); ti_sum += gap; }
-        if (p_fl == 3u && f_fl == 3u) ++dw;
+      // ---- hit row of o: 2 bits per access API inside its lifetime.  Each
+      // lane folds a contiguous run of hit words in order (count, first /
+      // last accessing API with its write / copy-set flags, TI gaps and DW
+      // pairs inside the run); the lanes are then joined at their
+      // boundaries: the gap / pair between a lane's first API and the
+      // previous non-empty lane's last one (one indexed shuffle), and warp
+      // sums / maxima.
+      const DevObj ob = p.objs[o];
+      const uint32_t nwords = (2 * p.n_hit[o] + 31) / 32;
+      const uint32_t per = (nwords + 31) / 32;
+      const uint32_t wlo = min(nwords, lane * per), whi = min(nwords, wlo + per);
+      HitFold f;
+      f.words(p.orw + ob.hit_word, wlo, whi, ob.r_lo, acc_ts, acc_cs, p.ti_min_idle);
+      const uint32_t nz = __ballot_sync(FULL_MASK, f.cnt != 0);
+      HitM hm = hit_identity();
+      if (nz) {
+        const uint32_t below = nz & ((1u << lane) - 1u);
+        const int pl = below ? 31 - __clz(below) : lane;
+        const uint32_t p_ts = __shfl_sync(FULL_MASK, f.l_ts, pl);
+        const uint32_t p_fl = __shfl_sync(FULL_MASK, f.l_fl, pl);
+        uint32_t ti_cnt = f.ti_cnt, ti_max = f.ti_max, ti_sum = f.ti_sum, dw = f.dw;
+        if (f.cnt && below) {
+          const uint32_t gap = f.f_ts - p_ts - 1;
+          if (gap >= p.ti_min_idle) { ++ti_cnt; ti_max = max(ti_max, gap); ti_sum += gap; }
+          if (p_fl == 3u && f.f_fl == 3u) ++dw;
+        }
+        const int fl0 = __ffs(nz) - 1, fl1 = 31 - __clz(nz);
+        hm.cnt = __reduce_add_sync(FULL_MASK, f.cnt);
+        hm.first_ts = __shfl_sync(FULL_MASK, f.f_ts, fl0);
+        hm.last_ts = __shfl_sync(FULL_MASK, f.l_ts, fl1);
+        hm.ti_cnt = __reduce_add_sync(FULL_MASK, ti_cnt);
+        hm.ti_max = __reduce_max_sync(FULL_MASK, ti_max);
+        hm.ti_sum = __reduce_add_sync(FULL_MASK, ti_sum);   // sum of disjoint gaps < n_api < 2^31
+        hm.dw = __reduce_add_sync(FULL_MASK, dw);
       }
-      const int fl0 = __ffs(nz) - 1, fl1 = 31 - __clz(nz);
-      hm.cnt = __reduce_add_sync(FULL_MASK, cnt);
-      hm.first_ts = __shfl_sync(FULL_MASK, f_ts, fl0);
-      hm.last_ts = __shfl_sync(FULL_MASK, l_ts, fl1);
-      hm.ti_cnt = __reduce_add_sync(FULL_MASK, ti_cnt);
-      hm.ti_max = __reduce_max_sync(FULL_MASK, ti_max);
-      hm.ti_sum = __reduce_add_sync(FULL_MASK, ti_sum);   // sum of disjoint gaps < n_api < 2^31
-      hm.dw = __reduce_add_sync(FULL_MASK, dw);
+      if (lane == 0) emit_object(p, o, ob, bm, hm);
     }
-    if (lane != 0) continue;
-    // ---- stats (A6)
-    const uint64_t n = (ob.end - ob.base) >> ob.shift;
-    const uint32_t first = p.first[o], last = p.last[o];
-    drgpum_object_stats_t st;
-    st.n_elems = n;
-    st.accessed = bm.pop;
-    st.span_lo = bm.lo;   // kNoPos == UINT64_MAX
-    st.span_hi = bm.hi;
-    st.largest_unaccessed_run = bm.best;
-    st.t_first = first;
-    st.t_last = last;
-    st.n_access_apis = hm.cnt;
-    st._pad = 0;
-    stats[o] = st;
-    // cross-check of the two liveness folds (atomics vs hit rows), and of
-    // bitmap vs hit row (an object with accessed elements has accessing APIs)
-    const bool consistent = bm.len >= n && (bm.pop == 0 || bm.hi < n) &&
-        (hm.cnt ? (first == hm.first_ts && last == hm.last_ts && bm.pop > 0)
-                : (first == kNever && last == 0 && bm.pop == 0));
-    if (!consistent) atomicAdd(&p.ctr[C_CONSISTENCY], 1ull);
-    // ---- patterns (A7)
-    drgpum_pattern_report_t r;
-    r.flags = 0; r.ea_distance = 0; r.ld_distance = 0; r.ti_ranges = 0;
-    r.ti_max_idle = 0; r.dw_pairs = 0; r.ti_total_idle = 0;
-    const bool used = hm.cnt > 0;
-    const bool leak = ob.t_free == kNever;
-    if (!used) r.flags |= DRGPUM_UA;
-    if (leak) r.flags |= DRGPUM_ML;
-    if (used) {
-      if (hm.first_ts - ob.t_alloc >= 2) { r.flags |= DRGPUM_EA; r.ea_distance = hm.first_ts - ob.t_alloc; }
-      if (!leak && ob.t_free - hm.last_ts >= 2) { r.flags |= DRGPUM_LD; r.ld_distance = ob.t_free - hm.last_ts; }
-      r.ti_ranges = hm.ti_cnt; r.ti_max_idle = hm.ti_max; r.ti_total_idle = hm.ti_sum;
-      r.dw_pairs = hm.dw;
-      if (hm.ti_cnt) r.flags |= DRGPUM_TI;
-      if (hm.dw) r.flags |= DRGPUM_DW;
-    }
-    using u128 = unsigned __int128;
-    if (u128(bm.pop) * 100u < u128(p.oa_pct) * n) {
-      r.flags |= DRGPUM_OA;
-      const uint64_t unacc = n - bm.pop;
-      if (unacc == 0 || u128(unacc - bm.best) * 100u < u128(p.frag_pct) * unacc)
-        r.flags |= DRGPUM_OA_ACTIONABLE;
-    }
-    reps[o] = r;
   }
 }
 
@@ -648,14 +695,21 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
     group_reduce_kernel<true><<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
   else
     group_reduce_kernel<false><<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
-  constexpr unsigned wpb = kFinThreads / 32;   // one warp per object
-  const uint64_t ob = (no + wpb - 1) / wpb;
+  // lane-parallel small objects when they are the majority (host count,
+  // FinalParams::n_small), else one object per warp
+  const bool lane = 2 * p.n_small > no;
+  const unsigned opb = lane ? kFinThreads : kFinThreads / 32;
+  const uint64_t ob = (no + opb - 1) / opb;
   unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
   if (g2 == 0) g2 = 1;
-  if (p.n_acc <= kSmemAcc)
-    object_finalize_kernel<true><<<g2, kFinThreads, 16 * ((p.n_acc + 3) / 4 + (p.n_acc + 15) / 16), s>>>(p);
-  else
-    object_finalize_kernel<false><<<g2, kFinThreads, 0, s>>>(p);
+  const size_t sm = 16 * ((p.n_acc + 3) / 4 + (p.n_acc + 15) / 16);
+  if (p.n_acc <= kSmemAcc) {
+    if (lane) object_finalize_kernel<true, true><<<g2, kFinThreads, sm, s>>>(p);
+    else object_finalize_kernel<true, false><<<g2, kFinThreads, sm, s>>>(p);
+  } else {
+    if (lane) object_finalize_kernel<false, true><<<g2, kFinThreads, 0, s>>>(p);
+    else object_finalize_kernel<false, false><<<g2, kFinThreads, 0, s>>>(p);
+  }
   return 3;
 }
 

@@ -76,6 +76,7 @@ struct drgpum_ctx {
   std::vector<uint32_t> tile_off;
   std::vector<Group> groups;
   std::vector<uint32_t> group_off;
+  std::vector<uint64_t> small_prefix;   // finalize: prefix count of lane-foldable objects
   std::vector<drgpum_object_layout_t> layout;
   uint64_t bitmap_words = 0, hit_words = 0;
   uint32_t rq_cap = 1u << 20;
@@ -264,6 +265,7 @@ drgpum_status build_tables(drgpum_ctx* c) {
   c->tile_off[n] = (uint32_t)c->tiles.size();
   c->groups.clear();
   c->group_off.assign(n + 1, 0);
+  c->small_prefix.clear();
   for (uint64_t i = 0; i < n; ++i) {
     c->group_off[i] = (uint32_t)c->groups.size();
     for (uint32_t t = c->tile_off[i]; t < c->tile_off[i + 1]; t += kGroupTiles)
@@ -529,6 +531,8 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   tmp.objs.assign(h_objs, h_objs + n_obj);
   tmp.kinds.assign(h_api_kinds, h_api_kinds + n_api);
   tmp.rq_cap = ctx->rq_cap;
+  tmp.sa_q_cap = ctx->sa_q_cap;
+  tmp.fq_recs = ctx->fq_recs;
   s = build_tables(&tmp);
   if (s != DRGPUM_OK) { ctx->err = tmp.err; return s; }
   ctx->n_obj = tmp.n_obj; ctx->n_api = tmp.n_api; ctx->n_acc = tmp.n_acc;
@@ -537,9 +541,10 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   ctx->cand.swap(tmp.cand); ctx->l1.swap(tmp.l1); ctx->l1_stride = tmp.l1_stride;
   ctx->acc_rank.swap(tmp.acc_rank); ctx->acc_ts.swap(tmp.acc_ts); ctx->acc_cs.swap(tmp.acc_cs);
   ctx->n_hit.swap(tmp.n_hit); ctx->tiles.swap(tmp.tiles); ctx->tile_off.swap(tmp.tile_off);
-  ctx->groups.swap(tmp.groups); ctx->group_off.swap(tmp.group_off);
+  ctx->groups.swap(tmp.groups); ctx->group_off.swap(tmp.group_off); ctx->small_prefix.clear();
   ctx->elem_base.swap(tmp.elem_base); ctx->n_elem_total = tmp.n_elem_total;
   ctx->slot_base.swap(tmp.slot_base); ctx->n_slots = tmp.n_slots;
+  ctx->fq_pos_bits = tmp.fq_pos_bits; ctx->fq_digits = tmp.fq_digits;
   ctx->features = 0;
   ctx->layout.swap(tmp.layout);
   ctx->bitmap_words = tmp.bitmap_words; ctx->hit_words = tmp.hit_words;
@@ -1065,6 +1070,13 @@ DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_threshold
   p.t_hi = ctx->tile_off[p.o_hi];
   p.g_lo = ctx->group_off[p.o_lo];
   p.g_hi = ctx->group_off[p.o_hi];
+  if (ctx->small_prefix.size() != ctx->n_obj + 1) {   // objects object_finalize folds lane by lane
+    ctx->small_prefix.assign(ctx->n_obj + 1, 0);
+    for (uint64_t o = 0; o < ctx->n_obj; ++o)
+      ctx->small_prefix[o + 1] = ctx->small_prefix[o] +
+          (ctx->group_off[o + 1] - ctx->group_off[o] <= 1 && (2ull * ctx->n_hit[o] + 31) / 32 <= kLaneHitWords);
+  }
+  p.n_small = ctx->small_prefix[p.o_hi] - ctx->small_prefix[p.o_lo];
   ctx->launches += launch_finalize(p, ctx->num_sms, st);
   ctx->gathered = false;
   CK(cudaGetLastError());

@@ -167,7 +167,9 @@ struct FinalParams {
   // the objects this call finalizes ([0, n_obj) unless an owned merge
   // narrowed it) and their tiles / groups
   uint64_t o_lo, o_hi, t_lo, t_hi, g_lo, g_hi;
+  uint64_t n_small;          // objects in [o_lo, o_hi) with one bitmap group and <= kLaneHitWords hit words
 };
+constexpr uint32_t kLaneHitWords = 128;   // hit rows a single lane folds in object_finalize (<= 2048 APIs)
 
 // Peer-memory merge (B7'): workspace base pointers of every rank, indexed by rank.
 constexpr uint32_t kMaxPeers = 64;
