@@ -113,12 +113,32 @@ __global__ void __launch_bounds__(kFT) freq_order_kernel(const __grid_constant__
   }
 }
 
+// Keys are staged per warp in shared memory and flushed 256 at a time with
+// ONE atomic on the global key count (a per-tile atomic on that single
+// address serialised the kernel: 3e6 same-address atomics on C2).
+constexpr uint32_t kEvBuf = 256;
+__device__ __forceinline__ void ev_flush(const FreqParams& q, uint64_t* out, const uint64_t* buf, uint32_t cnt,
+                                         int lane) {
+  unsigned long long base = 0;
+  if (lane == 0 && cnt) base = atomicAdd(&q.ctl[0], (unsigned long long)cnt);
+  base = __shfl_sync(FULL_MASK, base, 0);
+  if (!cnt) return;
+  if (base + cnt > q.cap) {                          // capacity exceeded: flagged, results invalid
+    if (lane == 0) atomicOr(q.state, 2u);
+    return;
+  }
+  for (uint32_t j = lane; j < cnt; j += 32) out[base + j] = buf[j];
+}
+
 __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant__ FreqParams q) {
   __shared__ uint64_t s_l1[kL1MaxKeys];
+  __shared__ uint64_t s_ev[kFT / 32][kEvBuf];
   const AttrParams& p = q.a;
   for (uint32_t j = threadIdx.x; j < p.n_l1; j += blockDim.x) s_l1[j] = p.l1[j];
   __syncthreads();
   const int lane = threadIdx.x & 31;
+  uint64_t* buf = s_ev[threadIdx.x >> 5];
+  uint32_t nbuf = 0;
   uint64_t* out = keys_buf(q, uint32_t(q.ctl[1]));
   // each warp walks one contiguous chunk (lane caches stay on one object)
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
@@ -152,18 +172,20 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
     const uint32_t hb = __ballot_sync(FULL_MASK, head), tb = __ballot_sync(FULL_MASK, tail);
     const uint32_t cnt = __popc(hb) + __popc(tb);
     if (!cnt) continue;
-    unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(&q.ctl[0], (unsigned long long)cnt);
-    base = __shfl_sync(FULL_MASK, base, 0);
-    if (base + cnt > q.cap) {                        // capacity exceeded: flagged, results invalid
-      if (lane == 0) atomicOr(q.state, 2u);
-      continue;
+    if (nbuf + cnt > kEvBuf) {                       // warp-uniform
+      __syncwarp();
+      ev_flush(q, out, buf, nbuf, lane);
+      __syncwarp();
+      nbuf = 0;
     }
     const uint32_t lt = (1u << lane) - 1u;
     const uint64_t hi = uint64_t(rank) << q.pos_bits;
-    if (head) out[base + __popc(hb & lt)] = hi | (2 * g0);
-    if (tail) out[base + __popc(hb) + __popc(tb & lt)] = hi | (2 * g1 + 1);
+    if (head) buf[nbuf + __popc(hb & lt)] = hi | (2 * g0);
+    if (tail) buf[nbuf + __popc(hb) + __popc(tb & lt)] = hi | (2 * g1 + 1);
+    nbuf += cnt;
   }
+  __syncwarp();
+  ev_flush(q, out, buf, nbuf, lane);
 }
 
 // ---------------------------------------------------------------- 2. radix sort
@@ -179,10 +201,15 @@ __global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ 
     s_h[threadIdx.x] = 0;
     __syncthreads();
     const uint64_t t0 = tile * kFreqTileKeys;
+    const int lane = threadIdx.x & 31;
 #pragma unroll 4
     for (uint32_t k = 0; k < kFreqTileKeys / kFT; ++k) {
       const uint64_t idx = t0 + k * kFT + threadIdx.x;
-      if (idx < n) atomicAdd(&s_h[(src[idx] >> shift) & 255u], 1u);
+      // warp-aggregated: sorted-ish keys share digits, so one shared atomic
+      // per distinct digit of the warp instead of 32 on one counter
+      const uint32_t dg = idx < n ? uint32_t(src[idx] >> shift) & 255u : 256u + uint32_t(lane);
+      const uint32_t peers = __match_any_sync(FULL_MASK, dg);
+      if (dg < 256u && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&s_h[dg], uint32_t(__popc(peers)));
     }
     __syncthreads();
     const uint32_t v = s_h[threadIdx.x];
