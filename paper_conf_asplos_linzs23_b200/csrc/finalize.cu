@@ -697,7 +697,9 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
     group_reduce_kernel<false><<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
   // lane-parallel small objects when they are the majority (host count,
   // FinalParams::n_small), else one object per warp
-  const bool lane = 2 * p.n_small > no;
+  // (only with enough objects to give every SM's warps 32 each: C5's 10^6;
+  // C2 / C4 keep one object per warp, 7 / ~1500 us)
+  const bool lane = 2 * p.n_small > no && no >= uint64_t(num_sms) * 32 * 32;
   const unsigned opb = lane ? kFinThreads : kFinThreads / 32;
   const uint64_t ob = (no + opb - 1) / opb;
   unsigned g2 = (unsigned)(ob < uint64_t(num_sms) * 16 ? ob : uint64_t(num_sms) * 16);
@@ -759,25 +761,13 @@ __global__ void __launch_bounds__(256) reset_touched_kernel(uint32_t* __restrict
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  // 32 tiles per warp step: each lane checks one tile's object (independent
-  // loads), then the warp zeroes the touched ones
-  for (uint64_t t0 = gwarp * 32; t0 < n_tiles; t0 += nwarps * 32) {
-    const uint64_t t = t0 + lane;
-    Tile tl{0, 0, 0, 0, 0};
-    bool touched = false;
-    if (t < n_tiles) {
-      tl = tiles[t];
-      touched = __ldg(first + tl.obj) != kNever;
-    }
-    uint32_t m = __ballot_sync(FULL_MASK, touched);
-    while (m) {
-      const int j = __ffs(m) - 1;
-      m &= m - 1;
-      const uint64_t wlo = __shfl_sync(FULL_MASK, tl.word_lo, j);
-      const uint32_t nv = (__shfl_sync(FULL_MASK, tl.n_words, j) + 3) / 4;
-      uint4* v = reinterpret_cast<uint4*>(orw + wlo);
-      for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
-    }
+  // one warp per tile (the zeroing is the work: up to 1024 words each)
+  for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
+    const Tile tl = tiles[t];
+    if (__ldg(first + tl.obj) == kNever) continue;   // warp-uniform
+    uint4* v = reinterpret_cast<uint4*>(orw + tl.word_lo);
+    const uint32_t nv = (tl.n_words + 3) / 4;
+    for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
   }
   for (uint64_t o0 = gwarp * 32; o0 < n_obj; o0 += nwarps * 32) {   // hit rows, 32 objects per step
     const uint64_t o = o0 + lane;
@@ -802,8 +792,8 @@ __global__ void __launch_bounds__(256) reset_touched_kernel(uint32_t* __restrict
 int launch_reset_touched(uint32_t* orw, const Tile* tiles, uint64_t n_tiles, const DevObj* objs,
                          const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, int num_sms,
                          cudaStream_t s) {
-  const uint64_t work = (n_tiles > n_obj ? n_tiles : n_obj) / 32;
-  if (!work && !n_tiles) return 0;
+  const uint64_t work = n_tiles > n_obj / 32 ? n_tiles : n_obj / 32;
+  if (!n_tiles && !n_obj) return 0;
   uint64_t b = (work + 7) / 8 + 1;
   if (b > uint64_t(num_sms) * 16) b = uint64_t(num_sms) * 16;
   reset_touched_kernel<<<(unsigned)b, 256, 0, s>>>(orw, tiles, n_tiles, objs, n_hit, first, n_obj);

@@ -103,16 +103,6 @@ __device__ __forceinline__ uint64_t n_keys(const FreqParams& q) {
 }
 
 // ---------------------------------------------------------------- 1. events
-__global__ void __launch_bounds__(kFT) freq_order_kernel(const __grid_constant__ FreqParams q) {
-  const AttrParams& p = q.a;
-  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
-  for (uint64_t i = tid; i < p.n; i += nth) {
-    const uint32_t t = ts_of(p, i);
-    if (i ? t < ts_of(p, i - 1) : (q.state[1] && uint64_t(t) + 1 < q.state[1])) atomicOr(q.state, 1u);
-  }
-}
-
 // Keys are staged per warp in shared memory and flushed 256 at a time with
 // ONE atomic on the global key count (a per-tile atomic on that single
 // address serialised the kernel: 3e6 same-address atomics on C2).
@@ -146,17 +136,22 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
   const uint64_t chunk = ((p.n + nwarps - 1) / nwarps + 31) / 32 * 32;
   const uint64_t w_lo = min(p.n, gw * chunk), w_hi = min(p.n, w_lo + chunk);
   LaneObj c;
+  // timestamp order (across the calls too): the record before this warp's
+  // chunk, or the previous call's last timestamp
+  uint32_t prev_t = w_lo < w_hi ? (w_lo ? ts_of(p, w_lo - 1) : (q.state[1] ? q.state[1] - 1u : 0u)) : 0u;
+  bool unsorted = false;
   for (uint64_t i0 = w_lo; i0 < w_hi; i0 += 32) {     // warp-uniform trip count
     const uint64_t i = i0 + lane;
     bool valid = false;
     uint64_t g0 = 0, g1 = 0;
     uint32_t rank = kNone;
-    if (i < w_hi) {
-      const uint32_t t = ts_of(p, i);
-      if (t < p.n_api) {
-        rank = __ldg(p.acc_rank + t);
-        valid = rank != kNone && resolve(q, s_l1, c, i, t, g0, g1);
-      }
+    const uint32_t t = i < w_hi ? ts_of(p, i) : 0xFFFFFFFFu;
+    const uint32_t tq = __shfl_up_sync(FULL_MASK, t, 1);
+    unsorted |= i < w_hi && t < (lane ? tq : prev_t);
+    prev_t = __shfl_sync(FULL_MASK, t, 31);   // the last lane's (a full tile, or the chunk end)
+    if (i < w_hi && t < p.n_api) {
+      rank = __ldg(p.acc_rank + t);
+      valid = rank != kNone && resolve(q, s_l1, c, i, t, g0, g1);
     }
     // merge chains of adjacent, disjoint intervals of one object and API
     const uint32_t obj = valid ? c.obj : kNone;
@@ -186,6 +181,7 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
   }
   __syncwarp();
   ev_flush(q, out, buf, nbuf, lane);
+  if (__any_sync(FULL_MASK, unsorted) && lane == 0) atomicOr(q.state, 1u);
 }
 
 // ---------------------------------------------------------------- 2. radix sort
@@ -202,14 +198,19 @@ __global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ 
     __syncthreads();
     const uint64_t t0 = tile * kFreqTileKeys;
     const int lane = threadIdx.x & 31;
-#pragma unroll 4
-    for (uint32_t k = 0; k < kFreqTileKeys / kFT; ++k) {
+    constexpr uint32_t kI = kFreqTileKeys / kFT;
+    uint32_t dk[kI];
+#pragma unroll
+    for (uint32_t k = 0; k < kI; ++k) {              // all of the tile's loads in flight at once
       const uint64_t idx = t0 + k * kFT + threadIdx.x;
+      dk[k] = idx < n ? uint32_t(__ldcs(src + idx) >> shift) & 255u : 256u + uint32_t(lane);
+    }
+#pragma unroll
+    for (uint32_t k = 0; k < kI; ++k) {
       // warp-aggregated: sorted-ish keys share digits, so one shared atomic
       // per distinct digit of the warp instead of 32 on one counter
-      const uint32_t dg = idx < n ? uint32_t(src[idx] >> shift) & 255u : 256u + uint32_t(lane);
-      const uint32_t peers = __match_any_sync(FULL_MASK, dg);
-      if (dg < 256u && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&s_h[dg], uint32_t(__popc(peers)));
+      const uint32_t peers = __match_any_sync(FULL_MASK, dk[k]);
+      if (dk[k] < 256u && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&s_h[dk[k]], uint32_t(__popc(peers)));
     }
     __syncthreads();
     const uint32_t v = s_h[threadIdx.x];
@@ -332,13 +333,21 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
     s_start[threadIdx.x] = block_excl_scan(cnt, s_w, tot);
     s_run[threadIdx.x] = 0;
     const uint64_t t0 = tile * kFreqTileKeys;
-    for (uint32_t sub = 0; sub < kFreqTileKeys / kFT; ++sub) {
+    constexpr uint32_t kI = kFreqTileKeys / kFT;
+    uint64_t kr[kI];
+#pragma unroll
+    for (uint32_t k = 0; k < kI; ++k) {              // all of the tile's loads in flight at once
+      const uint64_t idx = t0 + k * kFT + threadIdx.x;
+      kr[k] = idx < n ? __ldcs(src + idx) : 0ull;
+    }
+#pragma unroll
+    for (uint32_t sub = 0; sub < kI; ++sub) {
 #pragma unroll
       for (int w = 0; w < kFT / 32; ++w) s_wc[w][threadIdx.x] = 0;
       __syncthreads();
       const uint64_t idx = t0 + sub * kFT + threadIdx.x;
       const bool valid = idx < n;
-      const uint64_t key = valid ? src[idx] : 0ull;
+      const uint64_t key = kr[sub];
       const uint32_t dg = uint32_t(key >> shift) & 255u;
       const uint32_t peers = __match_any_sync(FULL_MASK, valid ? dg : 256u + uint32_t(lane));
       const uint32_t rk = __popc(peers & lt);
@@ -508,11 +517,8 @@ static void sweep(const FreqParams& q, unsigned long long* acc, uint32_t mode, i
 int launch_frequency(const FreqParams& q, int num_sms, cudaStream_t s) {
   if (q.a.n == 0) return 0;
   int launches = 0;
-  uint64_t b = (q.a.n + 255) / 256;
-  if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
-  freq_order_kernel<<<(unsigned)b, kFT, 0, s>>>(q);
-  freq_events_kernel<<<unsigned(num_sms) * 8, kFT, 0, s>>>(q);
-  launches += 2;
+  freq_events_kernel<<<unsigned(num_sms) * 8, kFT, 0, s>>>(q);   // also checks the timestamp order
+  launches += 1;
   radix_sort(q, num_sms, s, launches);
   sweep(q, q.acc, 0, num_sms, s, launches);
   freq_carry_kernel<<<unsigned(num_sms) * 4, kFT, 0, s>>>(q);
@@ -532,32 +538,38 @@ int launch_frequency_query(const FreqParams& q, uint64_t n_slots, int num_sms, c
 }
 
 // per object: the APIs at which it matches NUAF, and the first of them
+// (one warp per object, lanes over its slots)
 __global__ void __launch_bounds__(256) frequency_reduce_kernel(const FreqReduceParams q) {
-  for (uint64_t o = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; o < q.n_obj;
-       o += uint64_t(gridDim.x) * blockDim.x) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t gw = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  using u128 = unsigned __int128;
+  for (uint64_t o = gw; o < q.n_obj; o += nw) {
     const uint64_t sb = q.slot_base[o];
     const uint32_t nh = q.n_hit[o], r_lo = q.objs[o].r_lo;
-    uint32_t cnt = 0, first = kNever;
-    using u128 = unsigned __int128;
-    for (uint32_t k = 0; k < nh; ++k) {
+    uint32_t cnt = 0, first_k = 0xFFFFFFFFu;
+    for (uint32_t k = lane; k < nh; k += 32) {
       const unsigned long long* a = q.acc + 3 * (sb + k);
       const u128 n = a[0], s1 = a[1], s2 = a[2];
-      if (!s1) continue;
       // CV^2 = (n*S2 - S1^2)/S1^2 > (pct/100)^2
-      if ((n * s2 - s1 * s1) * 10000u > u128(q.pct) * q.pct * s1 * s1) {
+      if (s1 && (n * s2 - s1 * s1) * 10000u > u128(q.pct) * q.pct * s1 * s1) {
         ++cnt;
-        if (first == kNever) first = q.acc_ts[r_lo + k];
+        first_k = min(first_k, k);
       }
     }
-    q.out_count[o] = cnt;
-    q.out_first[o] = first;
+    cnt = __reduce_add_sync(FULL_MASK, cnt);
+    first_k = __reduce_min_sync(FULL_MASK, first_k);
+    if (lane == 0) {
+      q.out_count[o] = cnt;
+      q.out_first[o] = first_k == 0xFFFFFFFFu ? kNever : q.acc_ts[r_lo + first_k];
+    }
   }
 }
 
 int launch_frequency_reduce(const FreqReduceParams& q, int num_sms, cudaStream_t s) {
   if (q.n_obj == 0) return 0;
-  uint64_t b = (q.n_obj + 255) / 256;
-  if (b > uint64_t(num_sms) * 8) b = uint64_t(num_sms) * 8;
+  uint64_t b = (q.n_obj + 7) / 8;
+  if (b > uint64_t(num_sms) * 16) b = uint64_t(num_sms) * 16;
   frequency_reduce_kernel<<<(unsigned)b, 256, 0, s>>>(q);
   return 1;
 }
