@@ -41,6 +41,7 @@ namespace drgpum {
 constexpr int kFT = 256;                       // threads per block, every kernel here
 constexpr uint32_t kSweepItems = 8;            // keys per thread in the sweep
 constexpr uint32_t kSweepChunk = kFT * kSweepItems;
+constexpr uint32_t kSweepSample = 2048;        // object bases staged per block for the sweep's search
 
 __device__ __forceinline__ uint32_t ts_of(const AttrParams& p, uint64_t i) { return __ldcs(&p.recs[i].w) & 0x7FFFFFFFu; }
 
@@ -185,6 +186,18 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
 }
 
 // ---------------------------------------------------------------- 2. radix sort
+// Lanes holding the same 9-bit value (bit 8 = "no key"): nine ballots
+// instead of MATCH.ANY (which issues far slower in these loops).
+__device__ __forceinline__ uint32_t peers9(uint32_t v) {
+  uint32_t m = FULL_MASK;
+#pragma unroll
+  for (int b = 0; b < 9; ++b) {
+    const uint32_t x = __ballot_sync(FULL_MASK, (v >> b) & 1u);
+    m &= ((v >> b) & 1u) ? x : ~x;
+  }
+  return m;
+}
+
 // (a) tile histograms of digit d, digit-major: hist[digit * ntiles + tile];
 // totals per digit for the skip test
 __global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
@@ -193,24 +206,28 @@ __global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ 
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
   const uint64_t* src = keys_buf(q, buf_before(q, d));
   const uint32_t shift = 8 * d;
+  const int lane = threadIdx.x & 31;
+  constexpr uint32_t kI = kFreqTileKeys / kFT;
   for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     s_h[threadIdx.x] = 0;
     __syncthreads();
     const uint64_t t0 = tile * kFreqTileKeys;
-    const int lane = threadIdx.x & 31;
-    constexpr uint32_t kI = kFreqTileKeys / kFT;
     uint32_t dk[kI];
 #pragma unroll
     for (uint32_t k = 0; k < kI; ++k) {              // all of the tile's loads in flight at once
       const uint64_t idx = t0 + k * kFT + threadIdx.x;
-      dk[k] = idx < n ? uint32_t(__ldcs(src + idx) >> shift) & 255u : 256u + uint32_t(lane);
+      dk[k] = idx < n ? uint32_t(__ldcs(src + idx) >> shift) & 255u : 256u;
     }
 #pragma unroll
     for (uint32_t k = 0; k < kI; ++k) {
-      // warp-aggregated: sorted-ish keys share digits, so one shared atomic
-      // per distinct digit of the warp instead of 32 on one counter
-      const uint32_t peers = __match_any_sync(FULL_MASK, dk[k]);
-      if (dk[k] < 256u && (peers & ((1u << lane) - 1u)) == 0) atomicAdd(&s_h[dk[k]], uint32_t(__popc(peers)));
+      // the whole warp on one digit (the high digits of sorted-ish keys):
+      // one shared atomic; otherwise one per key (conflicts are rare then)
+      const uint32_t d0 = __shfl_sync(FULL_MASK, dk[k], 0);
+      if (__all_sync(FULL_MASK, dk[k] == d0)) {
+        if (lane == 0 && d0 < 256u) atomicAdd(&s_h[d0], 32u);
+      } else if (dk[k] < 256u) {
+        atomicAdd(&s_h[dk[k]], 1u);
+      }
     }
     __syncthreads();
     const uint32_t v = s_h[threadIdx.x];
@@ -309,13 +326,15 @@ __global__ void __launch_bounds__(1024) freq_part_scan_kernel(const __grid_const
   }
 }
 
-// (d) stable scatter of pass d: each tile's keys are ranked by digit in
-// shared memory (warp match + per-warp digit counts in warp order, 16
-// sub-chunks of 256 keys in key order), then stored digit run by digit run
+// (d) stable scatter of pass d.  Tile = 4096 keys; warp w ranks its 512
+// keys [512w, 512w+512) in 16 rounds of 32 (key order = round-major, lane
+// minor) against a per-warp digit counter -- no block barrier inside; one
+// block-wide combine turns the warps' digit counts into per-warp offsets;
+// keys go to shared memory in digit order and leave it run by run.
 __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
   __shared__ uint64_t s_keys[kFreqTileKeys];
-  __shared__ uint32_t s_wc[kFT / 32][256];
-  __shared__ uint32_t s_start[256], s_run[256], s_goff[256], s_w[kFT / 32];
+  __shared__ uint32_t s_wc[kFT / 32][256];           // per-warp digit counts, then offsets
+  __shared__ uint32_t s_start[256], s_goff[256], s_w[kFT / 32];
   if (q.ctl[8 + d]) return;                          // every key has the same digit: pass skipped
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
@@ -325,53 +344,69 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
   const uint32_t shift = 8 * d;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t lt = (1u << lane) - 1u;
+  constexpr uint32_t kR = kFreqTileKeys / kFT;       // 16 rounds of 32 keys per warp
+  uint32_t* wc = s_wc[warp];
   for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const uint64_t e = uint64_t(threadIdx.x) * ntiles + tile;
     const uint32_t cnt = q.hist[e];
     s_goff[threadIdx.x] = q.offs[e] + q.part[e / kFreqScanItems];
     uint32_t tot;
-    s_start[threadIdx.x] = block_excl_scan(cnt, s_w, tot);
-    s_run[threadIdx.x] = 0;
-    const uint64_t t0 = tile * kFreqTileKeys;
-    constexpr uint32_t kI = kFreqTileKeys / kFT;
-    uint64_t kr[kI];
+    s_start[threadIdx.x] = block_excl_scan(cnt, s_w, tot);   // (syncs: the previous tile is written out)
 #pragma unroll
-    for (uint32_t k = 0; k < kI; ++k) {              // all of the tile's loads in flight at once
-      const uint64_t idx = t0 + k * kFT + threadIdx.x;
-      kr[k] = idx < n ? __ldcs(src + idx) : 0ull;
+    for (int k = 0; k < 8; ++k) wc[lane + 32 * k] = 0;
+    __syncwarp();
+    const uint64_t w0 = tile * kFreqTileKeys + uint64_t(warp) * (kR * 32);
+    uint64_t kr[kR];
+#pragma unroll
+    for (uint32_t r = 0; r < kR; ++r) {              // all of the warp's loads in flight at once
+      const uint64_t idx = w0 + r * 32 + lane;
+      kr[r] = idx < n ? __ldcs(src + idx) : ~0ull;
     }
+    uint32_t rank[kR];
 #pragma unroll
-    for (uint32_t sub = 0; sub < kI; ++sub) {
-#pragma unroll
-      for (int w = 0; w < kFT / 32; ++w) s_wc[w][threadIdx.x] = 0;
-      __syncthreads();
-      const uint64_t idx = t0 + sub * kFT + threadIdx.x;
-      const bool valid = idx < n;
-      const uint64_t key = kr[sub];
-      const uint32_t dg = uint32_t(key >> shift) & 255u;
-      const uint32_t peers = __match_any_sync(FULL_MASK, valid ? dg : 256u + uint32_t(lane));
-      const uint32_t rk = __popc(peers & lt);
-      if (valid && rk == 0) s_wc[warp][dg] = __popc(peers);
-      __syncthreads();
-      uint32_t run = s_run[threadIdx.x];
-#pragma unroll
-      for (int w = 0; w < kFT / 32; ++w) {
-        const uint32_t v = s_wc[w][threadIdx.x];
-        s_wc[w][threadIdx.x] = run;
-        run += v;
+    for (uint32_t r = 0; r < kR; ++r) {
+      const bool valid = kr[r] != ~0ull;
+      const uint32_t dg = valid ? uint32_t(kr[r] >> shift) & 255u : 256u;
+      const uint32_t d0 = __shfl_sync(FULL_MASK, dg, 0);
+      if (__all_sync(FULL_MASK, dg == d0)) {          // one digit for the round (common on high digits)
+        if (d0 < 256u) {
+          rank[r] = wc[d0] + uint32_t(lane);
+          __syncwarp();
+          if (lane == 0) wc[d0] += 32u;
+        }
+      } else {
+        const uint32_t peers = peers9(dg);
+        if (valid) rank[r] = wc[dg] + __popc(peers & lt);
+        __syncwarp();
+        if (valid && (peers & lt) == 0) wc[dg] += __popc(peers);
       }
-      s_run[threadIdx.x] = run;
-      __syncthreads();
-      if (valid) s_keys[s_start[dg] + s_wc[warp][dg] + rk] = key;
-      __syncthreads();
+      __syncwarp();
     }
+    __syncthreads();
+    // per digit: exclusive prefix of the warps' counts (thread = digit)
+    uint32_t run = 0;
+#pragma unroll
+    for (int w = 0; w < kFT / 32; ++w) {
+      const uint32_t v = s_wc[w][threadIdx.x];
+      s_wc[w][threadIdx.x] = run;
+      run += v;
+    }
+    __syncthreads();
+#pragma unroll
+    for (uint32_t r = 0; r < kR; ++r) {
+      if (kr[r] == ~0ull) continue;
+      const uint32_t dg = uint32_t(kr[r] >> shift) & 255u;
+      s_keys[s_start[dg] + wc[dg] + rank[r]] = kr[r];
+    }
+    __syncthreads();
+    const uint64_t t0 = tile * kFreqTileKeys;
     const uint32_t tn = uint32_t(min(uint64_t(kFreqTileKeys), n - t0));
     for (uint32_t j = threadIdx.x; j < tn; j += kFT) {
       const uint64_t key = s_keys[j];
       const uint32_t dg = uint32_t(key >> shift) & 255u;
       dst[s_goff[dg] + (j - s_start[dg])] = key;
     }
-    __syncthreads();
+    __syncthreads();   // s_keys / s_goff / s_start are rewritten by the next tile
   }
 }
 
@@ -425,6 +460,12 @@ struct SlotSum {
 __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__ FreqParams q,
                                                          unsigned long long* acc) {
   __shared__ uint32_t s_w[kFT / 32];
+  __shared__ uint64_t s_eb[kSweepSample];            // element base of every stride-th object
+  const uint32_t n_obj = uint32_t(q.n_obj);
+  const uint32_t stride = (n_obj + kSweepSample - 1) / kSweepSample;   // >= 1
+  const uint32_t n_samp = (n_obj + stride - 1) / stride;
+  for (uint32_t i = threadIdx.x; i < n_samp; i += kFT) s_eb[i] = q.elem_base[uint64_t(i) * stride];
+  __syncthreads();
   const uint64_t split = q.ctl[2];
   const uint64_t* k = keys_buf(q, buf_before(q, q.n_digits));
   const uint64_t nb = (split + kSweepChunk - 1) / kSweepChunk;
@@ -451,8 +492,10 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
       const uint64_t x0 = (p0 + 1) >> 1, x1 = (p1 + 1) >> 1;
       if (x1 <= x0) continue;
       const uint64_t len = x1 - x0;
-      if (!(x0 >= c_lo && x0 < c_hi)) {             // object of element x0: binary search
-        uint32_t lo = 0, hi = uint32_t(q.n_obj);
+      if (!(x0 >= c_lo && x0 < c_hi)) {             // object of element x0: shared sample, then global
+        uint32_t a = 0, bb = n_samp;
+        while (bb - a > 1) { const uint32_t m = (a + bb) >> 1; if (s_eb[m] <= x0) a = m; else bb = m; }
+        uint32_t lo = a * stride, hi = min(n_obj, lo + stride);
         while (hi - lo > 1) { const uint32_t m = (lo + hi) >> 1; if (q.elem_base[m] <= x0) lo = m; else hi = m; }
         const DevObj dv = q.a.objs[lo];
         c_lo = q.elem_base[lo];
