@@ -462,7 +462,7 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
   __shared__ uint32_t s_w[kFT / 32];
   __shared__ uint64_t s_eb[kSweepSample];            // element base of every stride-th object
   const uint32_t n_obj = uint32_t(q.n_obj);
-  const uint32_t stride = (n_obj + kSweepSample - 1) / kSweepSample;   // >= 1
+  const uint32_t stride = n_obj ? (n_obj + kSweepSample - 1) / kSweepSample : 1u;
   const uint32_t n_samp = (n_obj + stride - 1) / stride;
   for (uint32_t i = threadIdx.x; i < n_samp; i += kFT) s_eb[i] = q.elem_base[uint64_t(i) * stride];
   __syncthreads();
