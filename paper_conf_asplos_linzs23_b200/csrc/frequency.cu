@@ -42,6 +42,9 @@ constexpr int kFT = 256;                       // threads per block, every kerne
 constexpr uint32_t kSweepItems = 8;            // keys per thread in the sweep
 constexpr uint32_t kSweepChunk = kFT * kSweepItems;
 constexpr uint32_t kSweepSample = 2048;        // object bases staged per block for the sweep's search
+constexpr uint32_t kBins = 1u << kFreqRadixBits;  // digit values per radix pass
+constexpr uint32_t kBPT = kBins / kFT;            // bins per thread
+static_assert(kBins % kFT == 0, "bins are spread evenly over the threads");
 
 __device__ __forceinline__ uint32_t ts_of(const AttrParams& p, uint64_t i) { return __ldcs(&p.recs[i].w) & 0x7FFFFFFFu; }
 
@@ -186,12 +189,12 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
 }
 
 // ---------------------------------------------------------------- 2. radix sort
-// Lanes holding the same 9-bit value (bit 8 = "no key"): nine ballots
-// instead of MATCH.ANY (which issues far slower in these loops).
-__device__ __forceinline__ uint32_t peers9(uint32_t v) {
+// Lanes holding the same (kFreqRadixBits + 1)-bit value (the top bit = "no
+// key"): one ballot per bit.
+__device__ __forceinline__ uint32_t peers_of(uint32_t v) {
   uint32_t m = FULL_MASK;
 #pragma unroll
-  for (int b = 0; b < 9; ++b) {
+  for (int b = 0; b <= int(kFreqRadixBits); ++b) {
     const uint32_t x = __ballot_sync(FULL_MASK, (v >> b) & 1u);
     m &= ((v >> b) & 1u) ? x : ~x;
   }
@@ -201,22 +204,23 @@ __device__ __forceinline__ uint32_t peers9(uint32_t v) {
 // (a) tile histograms of digit d, digit-major: hist[digit * ntiles + tile];
 // totals per digit for the skip test
 __global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
-  __shared__ uint32_t s_h[256];
+  __shared__ uint32_t s_h[kBins];
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
   const uint64_t* src = keys_buf(q, buf_before(q, d));
-  const uint32_t shift = 8 * d;
+  const uint32_t shift = kFreqRadixBits * d;
   const int lane = threadIdx.x & 31;
   constexpr uint32_t kI = kFreqTileKeys / kFT;
   for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    s_h[threadIdx.x] = 0;
+#pragma unroll
+    for (uint32_t b = 0; b < kBPT; ++b) s_h[threadIdx.x + b * kFT] = 0;
     __syncthreads();
     const uint64_t t0 = tile * kFreqTileKeys;
     uint32_t dk[kI];
 #pragma unroll
     for (uint32_t k = 0; k < kI; ++k) {              // all of the tile's loads in flight at once
       const uint64_t idx = t0 + k * kFT + threadIdx.x;
-      dk[k] = idx < n ? uint32_t(__ldcs(src + idx) >> shift) & 255u : 256u;
+      dk[k] = idx < n ? uint32_t(__ldcs(src + idx) >> shift) & (kBins - 1) : kBins;
     }
 #pragma unroll
     for (uint32_t k = 0; k < kI; ++k) {
@@ -224,15 +228,19 @@ __global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ 
       // one shared atomic; otherwise one per key (conflicts are rare then)
       const uint32_t d0 = __shfl_sync(FULL_MASK, dk[k], 0);
       if (__all_sync(FULL_MASK, dk[k] == d0)) {
-        if (lane == 0 && d0 < 256u) atomicAdd(&s_h[d0], 32u);
-      } else if (dk[k] < 256u) {
+        if (lane == 0 && d0 < kBins) atomicAdd(&s_h[d0], 32u);
+      } else if (dk[k] < kBins) {
         atomicAdd(&s_h[dk[k]], 1u);
       }
     }
     __syncthreads();
-    const uint32_t v = s_h[threadIdx.x];
-    q.hist[uint64_t(threadIdx.x) * ntiles + tile] = v;
-    if (v) atomicAdd(&q.ctl[16 + threadIdx.x], (unsigned long long)v);
+#pragma unroll
+    for (uint32_t b = 0; b < kBPT; ++b) {
+      const uint32_t bin = threadIdx.x + b * kFT;
+      const uint32_t v = s_h[bin];
+      q.hist[uint64_t(bin) * ntiles + tile] = v;
+      if (v) atomicAdd(&q.ctl[16 + bin], (unsigned long long)v);
+    }
     __syncthreads();
   }
 }
@@ -266,11 +274,11 @@ __global__ void __launch_bounds__(kFT) freq_scan_kernel(const __grid_constant__ 
   __shared__ uint32_t s_w[kFT / 32];
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
-  const uint64_t E = 256 * ntiles;
+  const uint64_t E = uint64_t(kBins) * ntiles;
   const uint64_t nb = (E + kFreqScanItems - 1) / kFreqScanItems;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     bool skip = n == 0;
-    for (int k = 0; k < 256 && !skip; ++k) skip = q.ctl[16 + k] == n;
+    for (uint32_t k = 0; k < kBins && !skip; ++k) skip = q.ctl[16 + k] == n;
     q.ctl[8 + d] = skip ? 1ull : 0ull;
   }
   constexpr uint32_t kI = kFreqScanItems / kFT;
@@ -301,7 +309,7 @@ __global__ void __launch_bounds__(1024) freq_part_scan_kernel(const __grid_const
     if (q.ctl[8 + d]) return;
     const uint64_t n = n_keys(q);
     const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
-    nb = (256 * ntiles + kFreqScanItems - 1) / kFreqScanItems;
+    nb = (uint64_t(kBins) * ntiles + kFreqScanItems - 1) / kFreqScanItems;
   } else {
     nb = (q.ctl[2] + kSweepChunk - 1) / kSweepChunk;
   }
@@ -333,27 +341,35 @@ __global__ void __launch_bounds__(1024) freq_part_scan_kernel(const __grid_const
 // keys go to shared memory in digit order and leave it run by run.
 __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
   __shared__ uint64_t s_keys[kFreqTileKeys];
-  __shared__ uint32_t s_wc[kFT / 32][256];           // per-warp digit counts, then offsets
-  __shared__ uint32_t s_start[256], s_goff[256], s_w[kFT / 32];
+  __shared__ uint16_t s_wc[kFT / 32][kBins];          // per-warp digit counts, then offsets (<= 4096)
+  __shared__ uint32_t s_start[kBins], s_goff[kBins], s_w[kFT / 32];
   if (q.ctl[8 + d]) return;                          // every key has the same digit: pass skipped
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
   const uint32_t src_b = buf_before(q, d);
   const uint64_t* src = keys_buf(q, src_b);
   uint64_t* dst = keys_buf(q, src_b ^ 1u);
-  const uint32_t shift = 8 * d;
+  const uint32_t shift = kFreqRadixBits * d;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t lt = (1u << lane) - 1u;
   constexpr uint32_t kR = kFreqTileKeys / kFT;       // 16 rounds of 32 keys per warp
-  uint32_t* wc = s_wc[warp];
+  uint16_t* wc = s_wc[warp];
   for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const uint64_t e = uint64_t(threadIdx.x) * ntiles + tile;
-    const uint32_t cnt = q.hist[e];
-    s_goff[threadIdx.x] = q.offs[e] + q.part[e / kFreqScanItems];
-    uint32_t tot;
-    s_start[threadIdx.x] = block_excl_scan(cnt, s_w, tot);   // (syncs: the previous tile is written out)
+    // the tile's digit counts (thread t: bins t*kBPT ..) -> local starts and global offsets
+    uint32_t cnt[kBPT], csum = 0;
 #pragma unroll
-    for (int k = 0; k < 8; ++k) wc[lane + 32 * k] = 0;
+    for (uint32_t b = 0; b < kBPT; ++b) {
+      const uint64_t e = uint64_t(threadIdx.x * kBPT + b) * ntiles + tile;
+      cnt[b] = q.hist[e];
+      s_goff[threadIdx.x * kBPT + b] = q.offs[e] + q.part[e / kFreqScanItems];
+      csum += cnt[b];
+    }
+    uint32_t tot;
+    uint32_t st = block_excl_scan(csum, s_w, tot);   // (syncs: the previous tile is written out)
+#pragma unroll
+    for (uint32_t b = 0; b < kBPT; ++b) { s_start[threadIdx.x * kBPT + b] = st; st += cnt[b]; }
+#pragma unroll
+    for (uint32_t k = 0; k < kBins / 32; ++k) wc[lane + 32 * k] = 0;
     __syncwarp();
     const uint64_t w0 = tile * kFreqTileKeys + uint64_t(warp) * (kR * 32);
     uint64_t kr[kR];
@@ -366,36 +382,40 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
 #pragma unroll
     for (uint32_t r = 0; r < kR; ++r) {
       const bool valid = kr[r] != ~0ull;
-      const uint32_t dg = valid ? uint32_t(kr[r] >> shift) & 255u : 256u;
+      const uint32_t dg = valid ? uint32_t(kr[r] >> shift) & (kBins - 1) : kBins;
       const uint32_t d0 = __shfl_sync(FULL_MASK, dg, 0);
       if (__all_sync(FULL_MASK, dg == d0)) {          // one digit for the round (common on high digits)
-        if (d0 < 256u) {
+        if (d0 < kBins) {
           rank[r] = wc[d0] + uint32_t(lane);
           __syncwarp();
-          if (lane == 0) wc[d0] += 32u;
+          if (lane == 0) wc[d0] = uint16_t(wc[d0] + 32u);
         }
       } else {
-        const uint32_t peers = peers9(dg);
+        const uint32_t peers = peers_of(dg);
         if (valid) rank[r] = wc[dg] + __popc(peers & lt);
         __syncwarp();
-        if (valid && (peers & lt) == 0) wc[dg] += __popc(peers);
+        if (valid && (peers & lt) == 0) wc[dg] = uint16_t(wc[dg] + __popc(peers));
       }
       __syncwarp();
     }
     __syncthreads();
-    // per digit: exclusive prefix of the warps' counts (thread = digit)
-    uint32_t run = 0;
+    // per digit: exclusive prefix of the warps' counts
 #pragma unroll
-    for (int w = 0; w < kFT / 32; ++w) {
-      const uint32_t v = s_wc[w][threadIdx.x];
-      s_wc[w][threadIdx.x] = run;
-      run += v;
+    for (uint32_t b = 0; b < kBPT; ++b) {
+      const uint32_t bin = threadIdx.x + b * kFT;
+      uint32_t run = 0;
+#pragma unroll
+      for (int w = 0; w < kFT / 32; ++w) {
+        const uint32_t v = s_wc[w][bin];
+        s_wc[w][bin] = uint16_t(run);
+        run += v;
+      }
     }
     __syncthreads();
 #pragma unroll
     for (uint32_t r = 0; r < kR; ++r) {
       if (kr[r] == ~0ull) continue;
-      const uint32_t dg = uint32_t(kr[r] >> shift) & 255u;
+      const uint32_t dg = uint32_t(kr[r] >> shift) & (kBins - 1);
       s_keys[s_start[dg] + wc[dg] + rank[r]] = kr[r];
     }
     __syncthreads();
@@ -403,7 +423,7 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
     const uint32_t tn = uint32_t(min(uint64_t(kFreqTileKeys), n - t0));
     for (uint32_t j = threadIdx.x; j < tn; j += kFT) {
       const uint64_t key = s_keys[j];
-      const uint32_t dg = uint32_t(key >> shift) & 255u;
+      const uint32_t dg = uint32_t(key >> shift) & (kBins - 1);
       dst[s_goff[dg] + (j - s_start[dg])] = key;
     }
     __syncthreads();   // s_keys / s_goff / s_start are rewritten by the next tile
@@ -433,10 +453,13 @@ __global__ void __launch_bounds__(kFT) freq_sweep_sum_kernel(const __grid_consta
   const uint64_t* k = keys_buf(q, buf_before(q, q.n_digits));
   const uint64_t nb = (split + kSweepChunk - 1) / kSweepChunk;
   for (uint64_t b = blockIdx.x; b < nb; b += gridDim.x) {
-    const uint64_t i0 = b * kSweepChunk + uint64_t(threadIdx.x) * kSweepItems;
+    const uint64_t c0 = b * kSweepChunk;
     int s = 0;
 #pragma unroll
-    for (uint32_t j = 0; j < kSweepItems; ++j) if (i0 + j < split) s += ev_sign(k[i0 + j]);
+    for (uint32_t j = 0; j < kSweepItems; ++j) {     // coalesced: the order does not matter for a sum
+      const uint64_t i = c0 + j * kFT + threadIdx.x;
+      if (i < split) s += ev_sign(__ldcs(k + i));
+    }
     uint32_t total;
     block_excl_scan(uint32_t(s), s_w, total);
     if (threadIdx.x == 0) q.part[b] = total;
@@ -461,6 +484,7 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
                                                          unsigned long long* acc) {
   __shared__ uint32_t s_w[kFT / 32];
   __shared__ uint64_t s_eb[kSweepSample];            // element base of every stride-th object
+  __shared__ uint64_t s_k[kSweepChunk + 1];
   const uint32_t n_obj = uint32_t(q.n_obj);
   const uint32_t stride = n_obj ? (n_obj + kSweepSample - 1) / kSweepSample : 1u;
   const uint32_t n_samp = (n_obj + stride - 1) / stride;
@@ -474,11 +498,21 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
   uint32_t c_rlo = 0;
   SlotSum ss;
   for (uint64_t b = blockIdx.x; b < nb; b += gridDim.x) {
-    const uint64_t i0 = b * kSweepChunk + uint64_t(threadIdx.x) * kSweepItems;
+    // the chunk (+ the next key) through shared memory: coalesced loads,
+    // then every thread its kSweepItems consecutive keys
+    const uint64_t c0 = b * kSweepChunk;
+#pragma unroll
+    for (uint32_t j = 0; j < kSweepItems; ++j) {
+      const uint64_t i = c0 + j * kFT + threadIdx.x;
+      s_k[j * kFT + threadIdx.x] = i < split ? __ldcs(k + i) : ~0ull;
+    }
+    if (threadIdx.x == 0) s_k[kSweepChunk] = c0 + kSweepChunk < split ? k[c0 + kSweepChunk] : ~0ull;
+    __syncthreads();
     uint64_t kk[kSweepItems + 1];
     int s = 0;
 #pragma unroll
-    for (uint32_t j = 0; j <= kSweepItems; ++j) kk[j] = i0 + j < split ? k[i0 + j] : ~0ull;
+    for (uint32_t j = 0; j <= kSweepItems; ++j) kk[j] = s_k[threadIdx.x * kSweepItems + j];
+    __syncthreads();
 #pragma unroll
     for (uint32_t j = 0; j < kSweepItems; ++j) if (kk[j] != ~0ull) s += ev_sign(kk[j]);
     uint32_t total;
@@ -538,7 +572,7 @@ __global__ void freq_carry_ctl_kernel(const __grid_constant__ FreqParams q) {
 static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& launches) {
   const unsigned g = unsigned(num_sms) * 4;
   for (uint32_t d = 0; d < q.n_digits; ++d) {
-    cudaMemsetAsync(q.ctl + 16, 0, 8 * 256, s);
+    cudaMemsetAsync(q.ctl + 16, 0, 8 * kBins, s);
     freq_hist_kernel<<<g, kFT, 0, s>>>(q, d);
     freq_scan_kernel<<<g, kFT, 0, s>>>(q, d);
     freq_part_scan_kernel<<<1, 1024, 0, s>>>(q, 0, d);

@@ -300,7 +300,7 @@ drgpum_status build_tables(drgpum_ctx* c) {
   for (uint64_t i = 0; i < n; ++i) { c->elem_base[i] = eb; eb += c->objs[i].size / c->objs[i].elem_size; }
   c->n_elem_total = eb;
   c->fq_pos_bits = std::max<uint32_t>(1, bits_for(2 * eb));        // NEXT-2 keys: 2*element (+1)
-  c->fq_digits = (c->fq_pos_bits + bits_for(c->n_acc) + 7) / 8;      // radix passes over (rank, pos)
+  c->fq_digits = (c->fq_pos_bits + bits_for(c->n_acc) + kFreqRadixBits - 1) / kFreqRadixBits;   // radix passes
   c->slot_base.assign(n, 0);
   uint64_t sb = 0;
   for (uint64_t i = 0; i < n; ++i) { c->slot_base[i] = sb; sb += c->n_hit[i]; }
@@ -362,7 +362,7 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   if (c->features & DRGPUM_FEATURE_FREQUENCY) {
     L.fq_acc = put(24 * c->n_slots);
     L.fq_state = put(16);
-    L.fq_ctl = put(8 * 272);
+    L.fq_ctl = put(8 * kFreqCtlWords);
     L.fq_end = off;                           // [fq_acc, fq_end) is zeroed per trace
     L.fq_acc_q = put(24 * c->n_slots);
     L.fq_slot_base = put(8 * n);
@@ -370,9 +370,9 @@ drgpum_status compute_layout(drgpum_ctx* c) {
     L.fq_out_first = put(4 * n);
     L.fq_keys0 = put(8 * freq_cap(c));
     L.fq_keys1 = put(8 * freq_cap(c));
-    L.fq_hist = put(4 * 256 * freq_max_tiles(c));
-    L.fq_offs = put(4 * 256 * freq_max_tiles(c));
-    L.fq_part = put(4 * (2 * freq_max_tiles(c) + 64));
+    L.fq_hist = put(4ull * (1u << kFreqRadixBits) * freq_max_tiles(c));
+    L.fq_offs = put(4ull * (1u << kFreqRadixBits) * freq_max_tiles(c));
+    L.fq_part = put(4 * (4 * freq_max_tiles(c) + 64));
   }
   L.total = off;
   return DRGPUM_OK;
@@ -563,7 +563,7 @@ DRGPUM_API drgpum_status drgpum_set_features(drgpum_ctx* ctx, uint32_t features)
     return fail(ctx, DRGPUM_EINVAL, "unknown feature bits");
   ctx->features = features;
   drgpum_status r = compute_layout(ctx);
-  if (r == DRGPUM_OK && (features & DRGPUM_FEATURE_FREQUENCY) && 8 * ctx->fq_digits > 64 + 7)
+  if (r == DRGPUM_OK && (features & DRGPUM_FEATURE_FREQUENCY) && ctx->fq_pos_bits + bits_for(ctx->n_acc) > 64)
     return fail(ctx, DRGPUM_EINVAL, "frequency analysis: (API rank, 2 x element) keys exceed 64 bits");
   return r;
 }

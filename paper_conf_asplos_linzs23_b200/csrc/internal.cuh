@@ -110,6 +110,8 @@ struct SaParams {
 // are carried over, sorted, and swept when the next call (or a query)
 // completes it.
 constexpr uint32_t kFreqTileKeys = 4096;        // radix-sort tile (256 threads x 16 keys)
+constexpr uint32_t kFreqRadixBits = 9;          // digit width of the LSD passes (512 bins)
+constexpr uint32_t kFreqCtlWords = 16 + (1u << kFreqRadixBits);   // control words (u64)
 constexpr uint32_t kFreqScanItems = 2048;       // entries per block of the digit-offset scan
 struct FreqParams {
   AttrParams a;                  // records of this (sub-)call, object table, index, rank table
@@ -120,12 +122,12 @@ struct FreqParams {
   uint32_t* state;               // [0] bit0 records out of order, bit1 event capacity exceeded;
                                  // [1] last timestamp of the previous call + 1 (0 = none)
   unsigned long long* ctl;       // [0] keys in the current buffer, [1] current buffer, [2] split,
-                                 // [3] skip flag of the current radix pass, [4..260) digit totals
+                                 // [8..16) skip flag per radix pass, [16..) digit totals
   uint64_t* keys0;               // event keys, ping-pong buffers of cap keys
   uint64_t* keys1;
   uint64_t cap;
-  uint32_t* hist;                // [256 * max_tiles] per-tile digit counts
-  uint32_t* offs;                // [256 * max_tiles] exclusive digit offsets (scanned)
+  uint32_t* hist;                // [bins * max_tiles] per-tile digit counts
+  uint32_t* offs;                // [bins * max_tiles] exclusive digit offsets (scanned)
   uint32_t* part;                // [scan blocks] block sums of offs, then of the sweep
   uint64_t max_tiles;
   uint64_t n_obj;
