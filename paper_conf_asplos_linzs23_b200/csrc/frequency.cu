@@ -268,33 +268,38 @@ __device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* s_w, u
   return before + x - v;
 }
 
-// (b) exclusive scan of hist (digit-major) in blocks of kFreqScanItems -> offs,
-// block sums -> part; block 0 also decides whether pass d can be skipped
-__global__ void __launch_bounds__(kFT) freq_scan_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
-  __shared__ uint32_t s_w[kFT / 32];
+// (b') digit offsets of pass d in one kernel: warp = digit; its global start
+// is the sum of the lower digits' totals, then a warp scan runs along its
+// row of tile counts (hist is digit-major: the row is contiguous)
+__global__ void __launch_bounds__(kFT) freq_offsets_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
-  const uint64_t E = uint64_t(kBins) * ntiles;
-  const uint64_t nb = (E + kFreqScanItems - 1) / kFreqScanItems;
+  const int lane = threadIdx.x & 31;
+  const uint32_t dg = blockIdx.x * (kFT / 32) + (threadIdx.x >> 5);
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     bool skip = n == 0;
     for (uint32_t k = 0; k < kBins && !skip; ++k) skip = q.ctl[16 + k] == n;
     q.ctl[8 + d] = skip ? 1ull : 0ull;
   }
-  constexpr uint32_t kI = kFreqScanItems / kFT;
-  for (uint64_t b = blockIdx.x; b < nb; b += gridDim.x) {
-    const uint64_t e0 = b * kFreqScanItems + uint64_t(threadIdx.x) * kI;
-    uint32_t v[kI], sum = 0;
+  if (dg >= kBins) return;
+  unsigned long long base = 0;
+  for (uint32_t k = lane; k < dg; k += 32) base += q.ctl[16 + k];
 #pragma unroll
-    for (uint32_t k = 0; k < kI; ++k) { v[k] = e0 + k < E ? q.hist[e0 + k] : 0u; sum += v[k]; }
-    uint32_t total;
-    uint32_t run = block_excl_scan(sum, s_w, total);
+  for (int o = 16; o; o >>= 1) base += __shfl_xor_sync(FULL_MASK, base, o);
+  const uint32_t* row = q.hist + uint64_t(dg) * ntiles;
+  uint32_t* orow = q.offs + uint64_t(dg) * ntiles;
+  uint32_t carry = uint32_t(base);
+  for (uint64_t c0 = 0; c0 < ntiles; c0 += 32) {
+    const uint64_t i = c0 + lane;
+    const uint32_t v = i < ntiles ? row[i] : 0u;
+    uint32_t x = v;
 #pragma unroll
-    for (uint32_t k = 0; k < kI; ++k) {
-      if (e0 + k < E) q.offs[e0 + k] = run;
-      run += v[k];
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL_MASK, x, o);
+      if (lane >= o) x += y;
     }
-    if (threadIdx.x == 0) q.part[b] = total;
+    if (i < ntiles) orow[i] = carry + x - v;
+    carry += __shfl_sync(FULL_MASK, x, 31);
   }
 }
 
@@ -361,7 +366,7 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
     for (uint32_t b = 0; b < kBPT; ++b) {
       const uint64_t e = uint64_t(threadIdx.x * kBPT + b) * ntiles + tile;
       cnt[b] = q.hist[e];
-      s_goff[threadIdx.x * kBPT + b] = q.offs[e] + q.part[e / kFreqScanItems];
+      s_goff[threadIdx.x * kBPT + b] = q.offs[e];
       csum += cnt[b];
     }
     uint32_t tot;
@@ -574,10 +579,9 @@ static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& la
   for (uint32_t d = 0; d < q.n_digits; ++d) {
     cudaMemsetAsync(q.ctl + 16, 0, 8 * kBins, s);
     freq_hist_kernel<<<g, kFT, 0, s>>>(q, d);
-    freq_scan_kernel<<<g, kFT, 0, s>>>(q, d);
-    freq_part_scan_kernel<<<1, 1024, 0, s>>>(q, 0, d);
+    freq_offsets_kernel<<<kBins / (kFT / 32), kFT, 0, s>>>(q, d);
     freq_scatter_kernel<<<g, kFT, 0, s>>>(q, d);
-    launches += 4;
+    launches += 3;
   }
 }
 
