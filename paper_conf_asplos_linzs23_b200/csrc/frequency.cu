@@ -268,38 +268,40 @@ __device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* s_w, u
   return before + x - v;
 }
 
-// (b') digit offsets of pass d in one kernel: warp = digit; its global start
-// is the sum of the lower digits' totals, then a warp scan runs along its
-// row of tile counts (hist is digit-major: the row is contiguous)
+// (b') digit offsets of pass d: one block per digit; its global start is the
+// sum of the lower digits' totals, then a block scan along its row of tile
+// counts (hist is digit-major: the row is contiguous), each thread a
+// contiguous segment of the row
 __global__ void __launch_bounds__(kFT) freq_offsets_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
+  __shared__ uint32_t s_w[kFT / 32];
+  __shared__ unsigned long long s_base;
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
-  const int lane = threadIdx.x & 31;
-  const uint32_t dg = blockIdx.x * (kFT / 32) + (threadIdx.x >> 5);
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
+  const uint32_t dg = blockIdx.x;
+  if (dg == 0 && threadIdx.x == 0) {
     bool skip = n == 0;
     for (uint32_t k = 0; k < kBins && !skip; ++k) skip = q.ctl[16 + k] == n;
     q.ctl[8 + d] = skip ? 1ull : 0ull;
   }
-  if (dg >= kBins) return;
-  unsigned long long base = 0;
-  for (uint32_t k = lane; k < dg; k += 32) base += q.ctl[16 + k];
+  if (threadIdx.x < 32) {
+    unsigned long long b = 0;
+    for (uint32_t k = threadIdx.x; k < dg; k += 32) b += q.ctl[16 + k];
 #pragma unroll
-  for (int o = 16; o; o >>= 1) base += __shfl_xor_sync(FULL_MASK, base, o);
+    for (int o = 16; o; o >>= 1) b += __shfl_xor_sync(FULL_MASK, b, o);
+    if (threadIdx.x == 0) s_base = b;
+  }
   const uint32_t* row = q.hist + uint64_t(dg) * ntiles;
   uint32_t* orow = q.offs + uint64_t(dg) * ntiles;
-  uint32_t carry = uint32_t(base);
-  for (uint64_t c0 = 0; c0 < ntiles; c0 += 32) {
-    const uint64_t i = c0 + lane;
-    const uint32_t v = i < ntiles ? row[i] : 0u;
-    uint32_t x = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL_MASK, x, o);
-      if (lane >= o) x += y;
-    }
-    if (i < ntiles) orow[i] = carry + x - v;
-    carry += __shfl_sync(FULL_MASK, x, 31);
+  const uint64_t seg = (ntiles + kFT - 1) / kFT;
+  const uint64_t lo = min(ntiles, uint64_t(threadIdx.x) * seg), hi = min(ntiles, lo + seg);
+  uint32_t sum = 0;
+  for (uint64_t i = lo; i < hi; ++i) sum += row[i];
+  uint32_t tot;
+  uint32_t run = block_excl_scan(sum, s_w, tot) + uint32_t(s_base);   // (its syncs publish s_base)
+  for (uint64_t i = lo; i < hi; ++i) {
+    const uint32_t v = row[i];
+    orow[i] = run;
+    run += v;
   }
 }
 
@@ -579,7 +581,7 @@ static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& la
   for (uint32_t d = 0; d < q.n_digits; ++d) {
     cudaMemsetAsync(q.ctl + 16, 0, 8 * kBins, s);
     freq_hist_kernel<<<g, kFT, 0, s>>>(q, d);
-    freq_offsets_kernel<<<kBins / (kFT / 32), kFT, 0, s>>>(q, d);
+    freq_offsets_kernel<<<kBins, kFT, 0, s>>>(q, d);
     freq_scatter_kernel<<<g, kFT, 0, s>>>(q, d);
     launches += 3;
   }
