@@ -292,16 +292,34 @@ __global__ void __launch_bounds__(kFT) freq_offsets_kernel(const __grid_constant
   }
   const uint32_t* row = q.hist + uint64_t(dg) * ntiles;
   uint32_t* orow = q.offs + uint64_t(dg) * ntiles;
-  const uint64_t seg = (ntiles + kFT - 1) / kFT;
-  const uint64_t lo = min(ntiles, uint64_t(threadIdx.x) * seg), hi = min(ntiles, lo + seg);
-  uint32_t sum = 0;
-  for (uint64_t i = lo; i < hi; ++i) sum += row[i];
-  uint32_t tot;
-  uint32_t run = block_excl_scan(sum, s_w, tot) + uint32_t(s_base);   // (its syncs publish s_base)
-  for (uint64_t i = lo; i < hi; ++i) {
-    const uint32_t v = row[i];
-    orow[i] = run;
-    run += v;
+  // the row in chunks of kFT * 16 counts through shared memory: coalesced
+  // loads / stores, each thread a contiguous 16-count segment for the scan
+  constexpr uint32_t kPer = 16, kChunk = kFT * kPer;
+  __shared__ uint32_t s_row[kChunk];
+  __syncthreads();                                   // s_base
+  uint32_t carry = uint32_t(s_base);
+  for (uint64_t c0 = 0; c0 < ntiles; c0 += kChunk) {
+#pragma unroll
+    for (uint32_t j = 0; j < kPer; ++j) {
+      const uint64_t i = c0 + j * kFT + threadIdx.x;
+      s_row[j * kFT + threadIdx.x] = i < ntiles ? row[i] : 0u;
+    }
+    __syncthreads();
+    uint32_t v[kPer], sum = 0;
+#pragma unroll
+    for (uint32_t j = 0; j < kPer; ++j) { v[j] = s_row[threadIdx.x * kPer + j]; sum += v[j]; }
+    uint32_t tot;
+    uint32_t run = carry + block_excl_scan(sum, s_w, tot);
+#pragma unroll
+    for (uint32_t j = 0; j < kPer; ++j) { s_row[threadIdx.x * kPer + j] = run; run += v[j]; }
+    __syncthreads();
+#pragma unroll
+    for (uint32_t j = 0; j < kPer; ++j) {
+      const uint64_t i = c0 + j * kFT + threadIdx.x;
+      if (i < ntiles) orow[i] = s_row[j * kFT + threadIdx.x];
+    }
+    carry += tot;
+    __syncthreads();
   }
 }
 
