@@ -71,10 +71,9 @@ struct LaneObj {
 
 // the global element interval [g0, g1] record i touches, false if it touches
 // no live object (or is malformed); c caches the object between records
-__device__ __forceinline__ bool resolve(const FreqParams& q, const uint64_t* l1, LaneObj& c, uint64_t i,
+__device__ __forceinline__ bool resolve(const FreqParams& q, const uint64_t* l1, LaneObj& c, const uint4& r,
                                         uint32_t t, uint64_t& g0, uint64_t& g1) {
   const AttrParams& p = q.a;
-  const uint4 r = __ldcs(p.recs + i);                 // streamed once
   const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
   const uint32_t size = r.z;
   if (size == 0 || addr > ~0ull - size) return false;
@@ -149,13 +148,14 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
     bool valid = false;
     uint64_t g0 = 0, g1 = 0;
     uint32_t rank = kNone;
-    const uint32_t t = i < w_hi ? ts_of(p, i) : 0xFFFFFFFFu;
+    const uint4 rec = i < w_hi ? __ldcs(p.recs + i) : make_uint4(0, 0, 0, 0xFFFFFFFFu);   // streamed once
+    const uint32_t t = i < w_hi ? (rec.w & 0x7FFFFFFFu) : 0xFFFFFFFFu;
     const uint32_t tq = __shfl_up_sync(FULL_MASK, t, 1);
     unsorted |= i < w_hi && t < (lane ? tq : prev_t);
     prev_t = __shfl_sync(FULL_MASK, t, 31);   // the last lane's (a full tile, or the chunk end)
     if (i < w_hi && t < p.n_api) {
       rank = __ldg(p.acc_rank + t);
-      valid = rank != kNone && resolve(q, s_l1, c, i, t, g0, g1);
+      valid = rank != kNone && resolve(q, s_l1, c, rec, t, g0, g1);
     }
     // merge chains of adjacent, disjoint intervals of one object and API
     const uint32_t obj = valid ? c.obj : kNone;
@@ -278,10 +278,11 @@ __global__ void __launch_bounds__(kFT) freq_offsets_kernel(const __grid_constant
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
   const uint32_t dg = blockIdx.x;
-  if (dg == 0 && threadIdx.x == 0) {
-    bool skip = n == 0;
-    for (uint32_t k = 0; k < kBins && !skip; ++k) skip = q.ctl[16 + k] == n;
-    q.ctl[8 + d] = skip ? 1ull : 0ull;
+  if (dg == 0) {                                      // skip the pass if one digit holds every key
+    bool hit = n == 0;
+    for (uint32_t k = threadIdx.x; k < kBins; k += kFT) hit |= q.ctl[16 + k] == n;
+    hit = __syncthreads_or(hit);
+    if (threadIdx.x == 0) q.ctl[8 + d] = hit ? 1ull : 0ull;
   }
   if (threadIdx.x < 32) {
     unsigned long long b = 0;
@@ -509,7 +510,7 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
                                                          unsigned long long* acc) {
   __shared__ uint32_t s_w[kFT / 32];
   __shared__ uint64_t s_eb[kSweepSample];            // element base of every stride-th object
-  __shared__ uint64_t s_k[kSweepChunk + 1];
+  __shared__ uint64_t s_k[kSweepChunk + kSweepChunk / 8 + 2];   // padded: 1 word per 8
   const uint32_t n_obj = uint32_t(q.n_obj);
   const uint32_t stride = n_obj ? (n_obj + kSweepSample - 1) / kSweepSample : 1u;
   const uint32_t n_samp = (n_obj + stride - 1) / stride;
@@ -529,14 +530,18 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
 #pragma unroll
     for (uint32_t j = 0; j < kSweepItems; ++j) {
       const uint64_t i = c0 + j * kFT + threadIdx.x;
-      s_k[j * kFT + threadIdx.x] = i < split ? __ldcs(k + i) : ~0ull;
+      const uint32_t li = j * kFT + threadIdx.x;
+      s_k[li + (li >> 3)] = i < split ? __ldcs(k + i) : ~0ull;
     }
-    if (threadIdx.x == 0) s_k[kSweepChunk] = c0 + kSweepChunk < split ? k[c0 + kSweepChunk] : ~0ull;
+    if (threadIdx.x == 0) s_k[kSweepChunk + kSweepChunk / 8] = c0 + kSweepChunk < split ? k[c0 + kSweepChunk] : ~0ull;
     __syncthreads();
     uint64_t kk[kSweepItems + 1];
     int s = 0;
 #pragma unroll
-    for (uint32_t j = 0; j <= kSweepItems; ++j) kk[j] = s_k[threadIdx.x * kSweepItems + j];
+    for (uint32_t j = 0; j <= kSweepItems; ++j) {
+      const uint32_t li = threadIdx.x * kSweepItems + j;   // li >> 3 == thread (+1 for the next key)
+      kk[j] = s_k[li + (li >> 3)];
+    }
     __syncthreads();
 #pragma unroll
     for (uint32_t j = 0; j < kSweepItems; ++j) if (kk[j] != ~0ull) s += ev_sign(kk[j]);
