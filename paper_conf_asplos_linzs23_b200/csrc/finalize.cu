@@ -564,14 +564,26 @@ struct HitFold {
   template <typename TS, typename CS>
   __device__ __forceinline__ void words(const uint32_t* row, uint32_t w_lo, uint32_t w_hi, uint32_t r_lo,
                                         const TS& acc_ts, const CS& acc_cs, uint32_t x_ti) {
-    for (uint32_t wi = w_lo; wi < w_hi; ++wi) {
-      uint32_t w = row[wi];
+    constexpr uint32_t kB = 8;                          // words loaded per round trip
+    for (uint32_t wb = w_lo; wb < w_hi; wb += kB) {
+      uint32_t ws[kB];
+#pragma unroll
+      for (uint32_t j = 0; j < kB; ++j) ws[j] = wb + j < w_hi ? row[wb + j] : 0u;
+      uint32_t any = 0;
+#pragma unroll
+      for (uint32_t j = 0; j < kB; ++j) any |= ws[j];
+      if (!any) continue;                               // untouched stretch (unused objects: all of it)
+#pragma unroll
+      for (uint32_t j = 0; j < kB; ++j) {
+      const uint32_t wi = wb + j;
+      uint32_t w = ws[j];
       while (w) {
         const uint32_t j = uint32_t(__ffs(w) - 1) >> 1;    // API slot inside this word
         const uint32_t pair = (w >> (2 * j)) & 3u;         // bit0 read, bit1 write
         w &= ~(3u << (2 * j));
         const uint32_t rank = r_lo + wi * 16 + j;
         add(acc_ts[rank], (pair >> 1) | (uint32_t(acc_cs[rank]) << 1), x_ti);   // bit0 write, bit1 copy/set
+      }
       }
     }
   }
