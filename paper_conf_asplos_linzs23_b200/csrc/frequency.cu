@@ -599,8 +599,11 @@ __global__ void freq_carry_ctl_kernel(const __grid_constant__ FreqParams q) {
 }
 
 // ---------------------------------------------------------------- launchers
+#ifndef DRGPUM_FQ_GRID
+#define DRGPUM_FQ_GRID 4
+#endif
 static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& launches) {
-  const unsigned g = unsigned(num_sms) * 4;
+  const unsigned g = unsigned(num_sms) * DRGPUM_FQ_GRID;
   for (uint32_t d = 0; d < q.n_digits; ++d) {
     cudaMemsetAsync(q.ctl + 16, 0, 8 * kBins, s);
     freq_hist_kernel<<<g, kFT, 0, s>>>(q, d);

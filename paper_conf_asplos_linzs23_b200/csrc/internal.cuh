@@ -109,7 +109,10 @@ struct SaParams {
 // API of the call's last records may continue in the next call: its events
 // are carried over, sorted, and swept when the next call (or a query)
 // completes it.
-constexpr uint32_t kFreqTileKeys = 4096;        // radix-sort tile (256 threads x 16 keys)
+#ifndef DRGPUM_FQ_TILE
+#define DRGPUM_FQ_TILE 4096
+#endif
+constexpr uint32_t kFreqTileKeys = DRGPUM_FQ_TILE;   // radix-sort tile (256 threads x 16 keys)
 constexpr uint32_t kFreqRadixBits = 9;          // digit width of the LSD passes (512 bins)
 constexpr uint32_t kFreqCtlWords = 16 + (1u << kFreqRadixBits);   // control words (u64)
 constexpr uint32_t kFreqScanItems = 2048;       // entries per block of the digit-offset scan
