@@ -1,0 +1,8 @@
+#!/bin/bash
+TAG=${1:-na}; OUT=gpurun_out/$TAG; mkdir -p $OUT
+python -c "import __graft_entry__ as g; g.build()" > $OUT/build.log 2>&1 || { tail -30 $OUT/build.log; exit 1; }
+for c in ${CFGS:-C5 C2}; do
+  skip=1; [ $c = C5 ] && skip=22
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:attribute_kernel -s $skip -c 1 -o $OUT/attr_$c \
+    python tools/ncu_one.py --config $c > $OUT/ncu_attr_$c.log 2>&1; echo "attr $c rc=$?"
+done
