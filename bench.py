@@ -584,8 +584,11 @@ def next_rows(prog, d_recs, plain_attr_ms, reps=5):
     stream = torch.cuda.current_stream()
     N = prog.n_records
     out = {}
+    # NEXT-2 processes a call in sub-calls of at most frequency_capacity
+    # records; one sub-call per (1e8-record) call here
     for name, kw, query in (("NEXT-3 structured access", {"structured": True}, lambda s: s.structured()),
-                            ("NEXT-2 non-uniform access frequency", {"frequency": True},
+                            ("NEXT-2 non-uniform access frequency",
+                             {"frequency": True, "frequency_capacity": min(N, 1 << 27)},
                              lambda s: s.frequency(20))):
         s = Session(prog.objects, prog.kinds, **kw)
         for _ in range(2):

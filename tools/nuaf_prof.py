@@ -9,7 +9,8 @@ from paper_conf_asplos_linzs23_b200 import Session
 
 w = bench.Workload(sys.argv[1] if len(sys.argv) > 1 else "C2")
 d = w.d_recs[:16 * w.n_local]
-s = Session(w.prog.objects, w.prog.kinds, frequency=True)
+cap = int(sys.argv[2]) if len(sys.argv) > 2 else None
+s = Session(w.prog.objects, w.prog.kinds, frequency=True, frequency_capacity=cap)
 for _ in range(2):
     s.reset(); s.attribute(d); s.frequency(20)
 torch.cuda.synchronize()
