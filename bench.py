@@ -71,10 +71,12 @@ def args_():
     ap.add_argument("--config", default="C5", choices=sorted(WORKLOADS))
     ap.add_argument("--records", type=int, default=None, help="override the record count")
     ap.add_argument("--e2e-steps", type=int, default=None)
-    ap.add_argument("--merge", default="owned", choices=["owned", "peers", "nccl"],
+    ap.add_argument("--merge", default="owned", choices=["owned", "owned-nvls", "peers", "nccl"],
                     help="N>1 exchange step over torch symmetric memory (NVLink P2P): owned = "
                          "drgpum_merge_peers_owned + per-rank finalize of its objects + "
-                         "drgpum_gather_peers; peers = drgpum_merge_peers (every rank gets the "
+                         "drgpum_gather_peers; owned-nvls = the same with objects several ranks "
+                         "touched read through the NVSwitch multicast mapping (NVLS OR, when the "
+                         "box provides one); peers = drgpum_merge_peers (every rank gets the "
                          "whole merged shadow, finalizes everything); nccl = all-to-all + "
                          "merge_or + all-gather")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -283,13 +285,19 @@ class Workload:
             self.chunks = [(0, self.n_local)]
         torch.cuda.synchronize()
         self.sm, self.merge_note = None, "none (1 rank)"
+        self.nvls = merge == "owned-nvls"
+        if self.nvls:
+            merge = "owned"
         if world > 1 and merge in ("peers", "owned"):
             from paper_conf_asplos_linzs23_b200.parallel import SymmetricMerge
             try:
                 self.sm = SymmetricMerge()
                 self.s = Session(self.prog.objects, self.prog.kinds, workspace_alloc=self.sm.alloc)
-                self.merge_note = ("drgpum_merge_peers_owned + finalize of the owned objects + "
-                                   "drgpum_gather_peers over torch symmetric memory (NVLink P2P)"
+                mc = self.sm.multicast_ptr() if self.nvls else 0
+                self.merge_note = (("drgpum_merge_peers_owned" + ("_nvls (NVSwitch multicast OR)" if mc else "") +
+                                    " + finalize of the owned objects + "
+                                    "drgpum_gather_peers over torch symmetric memory (NVLink P2P)" +
+                                    (" [nvls requested, no multicast mapping]" if self.nvls and not mc else ""))
                                    if merge == "owned" else
                                    "drgpum_merge_peers over torch symmetric memory (one kernel per rank, NVLink P2P)")
             except Exception as e:   # symmetric memory unavailable: the NCCL exchange instead, said so
@@ -308,7 +316,7 @@ class Workload:
         if self.world > 1:
             from paper_conf_asplos_linzs23_b200.parallel import merge_session
             if self.owned:
-                self.sm.merge_owned(self.s)
+                self.sm.merge_owned(self.s, nvls=self.nvls)
             elif self.sm is not None:
                 self.sm.merge(self.s)
             else:

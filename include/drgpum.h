@@ -317,6 +317,19 @@ DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx *ctx, void *const *h_peer
 DRGPUM_API drgpum_status drgpum_merge_peers_owned(drgpum_ctx *ctx, void *const *h_peer_ws,
     uint32_t n_peers, uint32_t rank, void *stream);
 
+/* The same owned merge with NVLS (NVLink SHARP, SURVEY §8(e) "B200-native
+ * stretch"): d_mc_ws is the NVSwitch multicast mapping of the ranks'
+ * workspaces (torch symmetric memory's multicast_ptr; the workspace is the
+ * symmetric buffer from its start).  Owned bitmap tiles and hit rows that at
+ * least two OTHER ranks touched are read with multimem.ld_reduce...or, the
+ * switch ORing every rank's copy (one read per word instead of one per
+ * touching peer); the rest as drgpum_merge_peers_owned.  Needs NVSwitch
+ * multicast (a multi-GPU NVLink box); untested on a single GPU, where torch
+ * gives no multicast mapping.  EINVAL for a NULL / unaligned d_mc_ws, else
+ * as drgpum_merge_peers_owned. */
+DRGPUM_API drgpum_status drgpum_merge_peers_owned_nvls(drgpum_ctx *ctx, void *const *h_peer_ws,
+    uint32_t n_peers, uint32_t rank, void *d_mc_ws, void *stream);
+
 /* After drgpum_merge_peers_owned + drgpum_finalize on every rank (and a
  * barrier): stores this rank's objects' stats and pattern reports into every
  * peer's workspace and adds its consistency-violation count into every peer's

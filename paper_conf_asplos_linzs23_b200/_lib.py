@@ -65,7 +65,7 @@ EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_set_features", "drgpu
            "drgpum_workspace_size",
            "drgpum_workspace_bind", "drgpum_reset", "drgpum_trace_attribute",
            "drgpum_trace_attribute_host", "drgpum_shadow_view", "drgpum_object_layout",
-           "drgpum_merge_or", "drgpum_merge_peers", "drgpum_merge_peers_owned", "drgpum_gather_peers", "drgpum_finalize", "drgpum_object_stats", "drgpum_patterns",
+           "drgpum_merge_or", "drgpum_merge_peers", "drgpum_merge_peers_owned", "drgpum_merge_peers_owned_nvls", "drgpum_gather_peers", "drgpum_finalize", "drgpum_object_stats", "drgpum_patterns",
            "drgpum_consistency_errors", "drgpum_path_stats", "drgpum_redundant_pairs",
            "drgpum_redundant_alloc", "drgpum_kahn_levels", "drgpum_dependency_graph",
            "drgpum_patterns_topo", "drgpum_last_error", "drgpum_destroy",
@@ -98,6 +98,7 @@ def load():
         "drgpum_merge_or": ([P, P, U32, U64, U64, U64, P], I),
         "drgpum_merge_peers": ([P, P, U32, U32, P], I),
         "drgpum_merge_peers_owned": ([P, P, U32, U32, P], I),
+        "drgpum_merge_peers_owned_nvls": ([P, P, U32, U32, P, P], I),
         "drgpum_gather_peers": ([P, P, U32, U32, P], I),
         "drgpum_finalize": ([P, ctypes.POINTER(Thresholds), P], I),
         "drgpum_object_stats": ([P, P, ctypes.POINTER(Counters), P], I),

@@ -923,6 +923,19 @@ int launch_merge_owned(const MergeOwnedParams& q, int num_sms, cudaStream_t s) {
   return 1;
 }
 
+// NVLS (NVLink SHARP): one load through the multicast mapping returns the OR
+// of every rank's copy, reduced in the NVSwitch.
+__device__ __forceinline__ uint64_t mc_or64(const void* a) {
+  uint64_t v;
+  asm volatile("multimem.ld_reduce.relaxed.sys.global.or.b64 %0, [%1];" : "=l"(v) : "l"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t mc_or32(const void* a) {
+  uint32_t v;
+  asm volatile("multimem.ld_reduce.relaxed.sys.global.or.b32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+  return v;
+}
+
 // B7'' sparse: the owned merge reading only what a peer wrote.  A peer's
 // words of object o are nonzero only if its first[o] is set (every bit is
 // attributed or merged together with a first-use fold), so kernel 1 (one
@@ -960,10 +973,15 @@ __global__ void __launch_bounds__(256) merge_owned_objects_kernel(const MergeOwn
     if ((mask & ~(1ull << q.rank)) == 0) continue;   // nobody else touched o
     const uint64_t hw = q.objs[o].hit_word;
     const uint32_t nw = (2 * q.n_hit[o] + 31) / 32;
+    const bool nvls = q.mc && __popcll(mask & ~(1ull << q.rank)) >= 2;   // the switch ORs the copies
     for (uint32_t i = lane; i < nw; i += 32) {
       uint32_t v = 0;
-      for (unsigned long long m = mask; m; m &= m - 1)
-        v |= __ldcg(reinterpret_cast<const uint32_t*>(q.peer[__ffsll(m) - 1] + q.or_off) + hw + i);
+      if (nvls) {
+        v = mc_or32(q.mc + q.or_off + 4 * (hw + i));
+      } else {
+        for (unsigned long long m = mask; m; m &= m - 1)
+          v |= __ldcg(reinterpret_cast<const uint32_t*>(q.peer[__ffsll(m) - 1] + q.or_off) + hw + i);
+      }
       reinterpret_cast<uint32_t*>(own + q.or_off)[hw + i] = v;
     }
   }
@@ -987,6 +1005,15 @@ __global__ void __launch_bounds__(256) merge_owned_tiles_kernel(const MergeOwned
     const unsigned long long mask = q.pmask[tl.obj];
     if ((mask & ~(1ull << q.rank)) == 0) continue;   // warp-uniform: local words are final
     const uint32_t nv = (tl.n_words + 3) / 4;
+    if (q.mc && __popcll(mask & ~(1ull << q.rank)) >= 2) {   // NVLS: one reduced load per 8 B
+      const uint8_t* mp = q.mc + q.or_off + 4 * tl.word_lo;
+      for (uint32_t i = lane; i < nv; i += 32) {
+        const uint64_t a = mc_or64(mp + 16 * i), b = mc_or64(mp + 16 * i + 8);
+        reinterpret_cast<uint4*>(own + q.or_off + 4 * tl.word_lo)[i] =
+            make_uint4(uint32_t(a), uint32_t(a >> 32), uint32_t(b), uint32_t(b >> 32));
+      }
+      continue;
+    }
     for (uint32_t i = lane; i < nv; i += 32) {
       uint4 v = make_uint4(0, 0, 0, 0);
       for (unsigned long long m = mask; m; m &= m - 1) {

@@ -968,8 +968,24 @@ DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx* ctx, void* const* h_peer
   return DRGPUM_OK;
 }
 
+static drgpum_status merge_owned_impl(drgpum_ctx* ctx, void* const* h_peer_ws, uint32_t n_peers,
+                                      uint32_t rank, void* d_mc, void* stream);
+
 DRGPUM_API drgpum_status drgpum_merge_peers_owned(drgpum_ctx* ctx, void* const* h_peer_ws,
                                                   uint32_t n_peers, uint32_t rank, void* stream) {
+  return merge_owned_impl(ctx, h_peer_ws, n_peers, rank, nullptr, stream);
+}
+
+DRGPUM_API drgpum_status drgpum_merge_peers_owned_nvls(drgpum_ctx* ctx, void* const* h_peer_ws,
+                                                       uint32_t n_peers, uint32_t rank, void* d_mc_ws,
+                                                       void* stream) {
+  if (ctx && (!d_mc_ws || reinterpret_cast<uintptr_t>(d_mc_ws) % kAlign))
+    return fail(ctx, DRGPUM_EINVAL, "merge_peers_owned_nvls: multicast address NULL or not 256-B aligned");
+  return merge_owned_impl(ctx, h_peer_ws, n_peers, rank, d_mc_ws, stream);
+}
+
+static drgpum_status merge_owned_impl(drgpum_ctx* ctx, void* const* h_peer_ws, uint32_t n_peers,
+                                      uint32_t rank, void* d_mc, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers_owned before workspace_bind");
   if (drgpum_status _d = set_device(ctx)) return _d;
@@ -993,6 +1009,7 @@ DRGPUM_API drgpum_status drgpum_merge_peers_owned(drgpum_ctx* ctx, void* const* 
   q.objs = at<DevObj>(ctx, ctx->L.objs);
   q.n_hit = at<uint32_t>(ctx, ctx->L.n_hit);
   q.pmask = at<unsigned long long>(ctx, ctx->L.pmask);
+  q.mc = static_cast<uint8_t*>(d_mc);
 #if DRGPUM_SPARSE_MERGE
   ctx->launches += launch_merge_owned_sparse(q, ctx->num_sms, as_stream(stream));
 #else

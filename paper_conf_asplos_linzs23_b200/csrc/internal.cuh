@@ -202,6 +202,7 @@ struct MergeOwnedParams {
   const DevObj* objs;
   const uint32_t* n_hit;
   unsigned long long* pmask;   // [n_obj] (this workspace)
+  uint8_t* mc;                 // NVLS multicast mapping of the workspaces (nullptr: peer loads only)
 };
 
 // Gather (B7''): rank r stores bytes [lo, hi) of the stats and of the

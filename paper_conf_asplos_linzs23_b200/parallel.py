@@ -116,12 +116,22 @@ class SymmetricMerge:
         session.merge_peers(self.peer_ptrs(), h.rank, stream)
         h.barrier(channel=0)            # every slice is merged everywhere
 
-    def merge_owned(self, session, stream=None):
+    def multicast_ptr(self):
+        """The NVSwitch multicast mapping of the workspaces (0 if none)."""
+        return int(getattr(self.handle, "multicast_ptr", 0) or 0)
+
+    def merge_owned(self, session, stream=None, nvls=False):
         """Owned merge: afterwards this rank holds the merged shadow of its
-        objects only; follow with session.finalize() and gather()."""
+        objects only; follow with session.finalize() and gather().  nvls:
+        objects several ranks touched are read through the multicast mapping
+        (NVLS in-switch OR) when the box provides one."""
         h = self.handle
         h.barrier(channel=0)            # every rank's attribution is done
-        session.merge_peers_owned(self.peer_ptrs(), h.rank, stream)
+        mc = self.multicast_ptr() if nvls else 0
+        if mc:
+            session.merge_peers_owned_nvls(self.peer_ptrs(), h.rank, mc, stream)
+        else:
+            session.merge_peers_owned(self.peer_ptrs(), h.rank, stream)
         h.barrier(channel=0)            # every rank's objects are merged
 
     def gather(self, session, stream=None):

@@ -287,6 +287,14 @@ class Session:
         check(self._h, self.L.drgpum_merge_peers_owned(self._h, arr, len(peer_ptrs), rank,
                                                        _stream_handle(stream)))
 
+    def merge_peers_owned_nvls(self, peer_ptrs, rank, mc_ptr, stream=None):
+        """drgpum_merge_peers_owned_nvls: the owned merge, objects touched by
+        several ranks read through the NVSwitch multicast mapping mc_ptr."""
+        arr = (ctypes.c_void_p * len(peer_ptrs))(*[ctypes.c_void_p(int(x)) for x in peer_ptrs])
+        check(self._h, self.L.drgpum_merge_peers_owned_nvls(self._h, arr, len(peer_ptrs), rank,
+                                                            ctypes.c_void_p(int(mc_ptr)),
+                                                            _stream_handle(stream)))
+
     def gather_peers(self, peer_ptrs, rank, stream=None):
         """drgpum_gather_peers: share this rank's finalized stats / reports."""
         arr = (ctypes.c_void_p * len(peer_ptrs))(*[ctypes.c_void_p(int(x)) for x in peer_ptrs])
