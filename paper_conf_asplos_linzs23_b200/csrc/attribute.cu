@@ -303,13 +303,15 @@ struct alignas(16) WarpSmem {
   uint32_t scratch[kScratchWords > 0 ? kScratchWords : 4];   // small-object bitmap copy
   uint64_t sc_base;                    // global word of scratch[0], kNoScratch if unbound
   uint64_t full[kStages];              // one mbarrier per stage
-  uint64_t f_pos, f_hi;                // lane 0: rest of the current chunk [f_pos, f_hi)
+  uint64_t f_src;                      // lane 0: global address of the chunk's next record
+  uint32_t f_left, f_last;             // lane 0: records left in the chunk; 1 if it ends the launch
   uint32_t cnt[kStages];               // records in each stage (0 = end of work)
   uint32_t pad;
   WarpCounts wc;
 };
-constexpr uint32_t kOffFull = offsetof(WarpSmem, full), kOffPos = offsetof(WarpSmem, f_pos),
-                   kOffHi = offsetof(WarpSmem, f_hi), kOffCnt = offsetof(WarpSmem, cnt),
+constexpr uint32_t kOffFull = offsetof(WarpSmem, full), kOffSrc = offsetof(WarpSmem, f_src),
+                   kOffLeft = offsetof(WarpSmem, f_left), kOffLast = offsetof(WarpSmem, f_last),
+                   kOffCnt = offsetof(WarpSmem, cnt),
                    kOffWc = offsetof(WarpSmem, wc), kOffScratch = offsetof(WarpSmem, scratch),
                    kOffScBase = offsetof(WarpSmem, sc_base);
 static_assert(offsetof(WarpCounts, aff_w) == offsetof(WarpCounts, aff_u) + 4, "aff_u / aff_w adjacent");
@@ -892,29 +894,39 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
   uint32_t f_next = kStatic ? blockIdx.x * (kAttrThreads / 32) + (threadIdx.x >> 5) : kNone;
   auto ticket = [&]() { return take_ticket(&p.ctr[C_WORK]) + (kStatic ? n_warps : 0u); };
   auto fetch = [&](int s) {   // lane 0: fill slot s with the next <= 128 records, or mark the end
-    uint64_t f_pos = lds64(wsm + kOffPos), f_hi = lds64(wsm + kOffHi);
-    if (f_pos == f_hi) {
+    // per stage: records left (u32) and the next record's address (u64) --
+    // a new chunk only every 64 stages; no 64-bit position arithmetic
+    uint32_t left = lds32<kOffLeft>(wsm);
+    uint64_t src;
+    if (left == 0) {
+      uint64_t lo, hi;
       do {   // skip empty chunks (only possible at the end or in a tiny static part)
         const uint32_t kc = f_next == kNone ? ticket() : f_next;
         f_next = kNone;
-        f_pos = min(chunk_start(kc, p.n, n_warps), p.n);
-        f_hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps), p.n);
-      } while (f_pos == f_hi && f_pos < p.n);
-      if (f_pos >= p.n) f_pos = f_hi = p.n;
-      sts64(wsm + kOffHi, f_hi);
+        lo = min(chunk_start(kc, p.n, n_warps), p.n);
+        hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps), p.n);
+      } while (lo == hi && lo < p.n);
+      if (lo >= p.n) lo = hi = p.n;
+      left = uint32_t(hi - lo);
+      src = reinterpret_cast<uint64_t>(p.recs + lo);
+      sts32(wsm + kOffLast, hi >= p.n ? 1u : 0u);
+    } else {
+      src = lds64(wsm + kOffSrc);
     }
-    const uint32_t cnt = uint32_t(min(uint64_t(kWarpRecords), f_hi - f_pos));
+    const uint32_t cnt = min(uint32_t(kWarpRecords), left);
     sts32(wsm + kOffCnt + 4 * s, cnt);
     const uint32_t bar = wsm + kOffFull + 8 * s;
     if (cnt) {
       mbar_arrive_expect_tx(bar, cnt * 16);
-      tma_load_1d(wsm + s * (kWarpRecords * 16), p.recs + f_pos, cnt * 16, bar, evict_first_policy());
-      f_pos += cnt;
-      sts64(wsm + kOffPos, f_pos);
+      tma_load_1d(wsm + s * (kWarpRecords * 16), reinterpret_cast<const void*>(src), cnt * 16, bar,
+                  evict_first_policy());
+      sts64(wsm + kOffSrc, src + 16ull * cnt);
+      left -= cnt;
+      sts32(wsm + kOffLeft, left);
       // the next chunk's ticket is taken when this one has at most two stages
       // left: its latency hides behind them, and no warp holds a reservation
       // long enough to unbalance the end of the launch
-      if (f_next == kNone && f_hi - f_pos <= 2 * kWarpRecords && f_hi < p.n)
+      if (left <= 2 * kWarpRecords && f_next == kNone && !lds32<kOffLast>(wsm))
         f_next = ticket();
     } else {
       mbar_arrive(bar);   // end of work: complete the phase with cnt = 0
@@ -927,8 +939,9 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
   my->t_alloc = 0; my->t_free = 0; my->r_lo = 0; my->shift = 0; my->obj = kNone; my->meta = kNever;
   if (lane == 0) {
     *slow_counts() = WarpCounts{0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
-    sts64(wsm + kOffPos, 0);
-    sts64(wsm + kOffHi, 0);
+    sts64(wsm + kOffSrc, 0);
+    sts32(wsm + kOffLeft, 0);
+    sts32(wsm + kOffLast, 0);
     sts64(wsm + kOffScBase, kNoScratch);
     for (int s = 0; s < kStages; ++s) mbar_init(wsm + kOffFull + 8 * s, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
