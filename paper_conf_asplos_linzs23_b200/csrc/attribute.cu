@@ -72,6 +72,9 @@ constexpr int kWarpRecords = kTilesPerWarp * 32;             // 128 records = 2 
 #ifndef DRGPUM_STATIC
 #define DRGPUM_STATIC 0
 #endif
+#ifndef DRGPUM_FETCH_V2
+#define DRGPUM_FETCH_V2 1   // per-stage fetch bookkeeping as records-left + next address (A/B macro)
+#endif
 #ifndef DRGPUM_TAIL
 #define DRGPUM_TAIL 1   // guided tail (below): C2 0.389 -> 0.381 ms with kBigPct 85; C3 within noise
 #endif
@@ -893,6 +896,7 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
   // lane 0: ticket of the next chunk, taken two stages ahead (static: its own range first)
   uint32_t f_next = kStatic ? blockIdx.x * (kAttrThreads / 32) + (threadIdx.x >> 5) : kNone;
   auto ticket = [&]() { return take_ticket(&p.ctr[C_WORK]) + (kStatic ? n_warps : 0u); };
+#if DRGPUM_FETCH_V2
   auto fetch = [&](int s) {   // lane 0: fill slot s with the next <= 128 records, or mark the end
     // per stage: records left (u32) and the next record's address (u64) --
     // a new chunk only every 64 stages; no 64-bit position arithmetic
@@ -933,6 +937,39 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
     }
   };
 
+#else
+  // A/B reference: 64-bit [f_pos, f_hi) kept in the f_src / (f_left, f_last) words
+  auto fetch = [&](int s) {   // lane 0: fill slot s with the next <= 128 records, or mark the end
+    uint64_t f_pos = lds64(wsm + kOffSrc), f_hi = lds64(wsm + kOffLeft);
+    if (f_pos == f_hi) {
+      do {   // skip empty chunks (only possible at the end or in a tiny static part)
+        const uint32_t kc = f_next == kNone ? ticket() : f_next;
+        f_next = kNone;
+        f_pos = min(chunk_start(kc, p.n, n_warps), p.n);
+        f_hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps), p.n);
+      } while (f_pos == f_hi && f_pos < p.n);
+      if (f_pos >= p.n) f_pos = f_hi = p.n;
+      sts64(wsm + kOffLeft, f_hi);
+    }
+    const uint32_t cnt = uint32_t(min(uint64_t(kWarpRecords), f_hi - f_pos));
+    sts32(wsm + kOffCnt + 4 * s, cnt);
+    const uint32_t bar = wsm + kOffFull + 8 * s;
+    if (cnt) {
+      mbar_arrive_expect_tx(bar, cnt * 16);
+      tma_load_1d(wsm + s * (kWarpRecords * 16), p.recs + f_pos, cnt * 16, bar, evict_first_policy());
+      f_pos += cnt;
+      sts64(wsm + kOffSrc, f_pos);
+      // the next chunk's ticket is taken when this one has at most two stages
+      // left: its latency hides behind them, and no warp holds a reservation
+      // long enough to unbalance the end of the launch
+      if (f_next == kNone && f_hi - f_pos <= 2 * kWarpRecords && f_hi < p.n)
+        f_next = ticket();
+    } else {
+      mbar_arrive(bar);   // end of work: complete the phase with cnt = 0
+    }
+  };
+
+#endif
   for (uint32_t i = lane; i < kScratchWords; i += 32) sts32(wsm + kOffScratch + 4 * i, 0);
   SlowCache* my = slow_cache();
   my->base = 0; my->size = 0; my->bm_word = 0; my->hit_word = 0;
