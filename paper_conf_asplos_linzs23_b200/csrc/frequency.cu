@@ -100,6 +100,9 @@ __device__ __forceinline__ uint32_t buf_before(const FreqParams& q, uint32_t d) 
   for (uint32_t k = 0; k < d; ++k) b ^= q.ctl[8 + k] ? 0u : 1u;
   return b;
 }
+__device__ __forceinline__ unsigned long long* digit_totals(const FreqParams& q, uint32_t d) {
+  return q.ctl + kFreqCtlTot + uint64_t(d) * kBins;
+}
 __device__ __forceinline__ uint64_t n_keys(const FreqParams& q) {
   const unsigned long long n = q.ctl[0];
   return n < q.cap ? n : q.cap;
@@ -239,7 +242,7 @@ __global__ void __launch_bounds__(kFT) freq_hist_kernel(const __grid_constant__ 
       const uint32_t bin = threadIdx.x + b * kFT;
       const uint32_t v = s_h[bin];
       q.hist[uint64_t(bin) * ntiles + tile] = v;
-      if (v) atomicAdd(&q.ctl[16 + bin], (unsigned long long)v);
+      if (v) atomicAdd(digit_totals(q, d) + bin, (unsigned long long)v);
     }
     __syncthreads();
   }
@@ -280,13 +283,13 @@ __global__ void __launch_bounds__(kFT) freq_offsets_kernel(const __grid_constant
   const uint32_t dg = blockIdx.x;
   if (dg == 0) {                                      // skip the pass if one digit holds every key
     bool hit = n == 0;
-    for (uint32_t k = threadIdx.x; k < kBins; k += kFT) hit |= q.ctl[16 + k] == n;
+    for (uint32_t k = threadIdx.x; k < kBins; k += kFT) hit |= digit_totals(q, d)[k] == n;
     hit = __syncthreads_or(hit);
     if (threadIdx.x == 0) q.ctl[8 + d] = hit ? 1ull : 0ull;
   }
   if (threadIdx.x < 32) {
     unsigned long long b = 0;
-    for (uint32_t k = threadIdx.x; k < dg; k += 32) b += q.ctl[16 + k];
+    for (uint32_t k = threadIdx.x; k < dg; k += 32) b += digit_totals(q, d)[k];
 #pragma unroll
     for (int o = 16; o; o >>= 1) b += __shfl_xor_sync(FULL_MASK, b, o);
     if (threadIdx.x == 0) s_base = b;
@@ -456,6 +459,168 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
   }
 }
 
+// ---- one-sweep form (default): every pass's digit totals from one read of
+// the keys, then ONE kernel per pass: tiles taken in order from a ticket,
+// ranked as above, their digit counts published and the exclusive prefix over
+// the previous tiles found by decoupled look-back (flag A: the tile's own
+// count, flag P: the inclusive prefix), so no per-pass histogram kernel and
+// no offset scan.
+constexpr uint32_t kFlagA = 1u << 30, kFlagP = 1u << 31, kValMask = kFlagA - 1;
+
+__global__ void __launch_bounds__(kFT) freq_hist_all_kernel(const __grid_constant__ FreqParams q) {
+  __shared__ uint32_t s_h[kFreqMaxDigits][kBins];
+  const uint64_t n = n_keys(q);
+  const uint64_t* src = keys_buf(q, uint32_t(q.ctl[1]));
+  const int lane = threadIdx.x & 31;
+  const uint32_t nd = q.n_digits;
+  for (uint32_t i = threadIdx.x; i < nd * kBins; i += kFT) s_h[i / kBins][i % kBins] = 0;
+  __syncthreads();
+  const uint64_t nth = uint64_t(gridDim.x) * kFT;
+  for (uint64_t i0 = uint64_t(blockIdx.x) * kFT; i0 < n; i0 += nth) {
+    const uint64_t i = i0 + threadIdx.x;
+    const bool valid = i < n;
+    const uint64_t key = valid ? __ldcs(src + i) : 0ull;
+    for (uint32_t d = 0; d < nd; ++d) {
+      const uint32_t dg = valid ? uint32_t(key >> (kFreqRadixBits * d)) & (kBins - 1) : kBins;
+      const uint32_t d0 = __shfl_sync(FULL_MASK, dg, 0);
+      if (__all_sync(FULL_MASK, dg == d0)) {
+        if (lane == 0 && d0 < kBins) atomicAdd(&s_h[d][d0], 32u);
+      } else if (valid) {
+        atomicAdd(&s_h[d][dg], 1u);
+      }
+    }
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < nd * kBins; i += kFT) {
+    const uint32_t v = s_h[i / kBins][i % kBins];
+    if (v) atomicAdd(digit_totals(q, i / kBins) + (i % kBins), (unsigned long long)v);
+  }
+}
+
+// skip flags of every pass (a pass whose digit is the same for every key)
+__global__ void __launch_bounds__(kFT) freq_skip_kernel(const __grid_constant__ FreqParams q) {
+  const uint64_t n = n_keys(q);
+  for (uint32_t d = 0; d < q.n_digits; ++d) {
+    bool hit = n == 0;
+    for (uint32_t k = threadIdx.x; k < kBins; k += kFT) hit |= digit_totals(q, d)[k] == n;
+    hit = __syncthreads_or(hit);
+    if (threadIdx.x == 0) q.ctl[8 + d] = hit ? 1ull : 0ull;
+  }
+}
+
+__global__ void __launch_bounds__(kFT) freq_onesweep_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
+  __shared__ uint64_t s_keys[kFreqTileKeys];
+  __shared__ uint16_t s_wc[kFT / 32][kBins];          // per-warp digit counts, then offsets (<= 4096)
+  __shared__ uint32_t s_start[kBins], s_goff[kBins], s_gstart[kBins], s_w[kFT / 32];
+  __shared__ uint32_t s_tile;
+  if (q.ctl[8 + d]) return;                          // every key has the same digit: pass skipped
+  const uint64_t n = n_keys(q);
+  const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
+  const uint32_t src_b = buf_before(q, d);
+  const uint64_t* src = keys_buf(q, src_b);
+  uint64_t* dst = keys_buf(q, src_b ^ 1u);
+  const uint32_t shift = kFreqRadixBits * d;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  constexpr uint32_t kR = kFreqTileKeys / kFT;
+  uint16_t* wc = s_wc[warp];
+  volatile uint32_t* status = q.hist;                // [tile][bin]
+  {   // global digit starts of this pass (exclusive scan of the totals)
+    const unsigned long long* tot = digit_totals(q, d);
+    uint32_t c[kBPT], cs = 0;
+#pragma unroll
+    for (uint32_t b = 0; b < kBPT; ++b) { c[b] = uint32_t(tot[threadIdx.x * kBPT + b]); cs += c[b]; }
+    uint32_t all;
+    uint32_t st = block_excl_scan(cs, s_w, all);
+#pragma unroll
+    for (uint32_t b = 0; b < kBPT; ++b) { s_gstart[threadIdx.x * kBPT + b] = st; st += c[b]; }
+  }
+  for (;;) {
+    if (threadIdx.x == 0) s_tile = uint32_t(atomicAdd(&q.ctl[16 + d], 1ull));
+    __syncthreads();
+    const uint64_t tile = s_tile;
+    if (tile >= ntiles) break;
+#pragma unroll
+    for (uint32_t k = 0; k < kBins / 32; ++k) wc[lane + 32 * k] = 0;
+    __syncwarp();
+    const uint64_t w0 = tile * kFreqTileKeys + uint64_t(warp) * (kR * 32);
+    uint64_t kr[kR];
+#pragma unroll
+    for (uint32_t r = 0; r < kR; ++r) {
+      const uint64_t idx = w0 + r * 32 + lane;
+      kr[r] = idx < n ? __ldcs(src + idx) : ~0ull;
+    }
+    uint32_t rank[kR];
+#pragma unroll
+    for (uint32_t r = 0; r < kR; ++r) {
+      const bool valid = kr[r] != ~0ull;
+      const uint32_t dg = valid ? uint32_t(kr[r] >> shift) & (kBins - 1) : kBins;
+      const uint32_t d0 = __shfl_sync(FULL_MASK, dg, 0);
+      if (__all_sync(FULL_MASK, dg == d0)) {
+        if (d0 < kBins) {
+          rank[r] = wc[d0] + uint32_t(lane);
+          __syncwarp();
+          if (lane == 0) wc[d0] = uint16_t(wc[d0] + 32u);
+        }
+      } else {
+        const uint32_t peers = peers_of(dg);
+        if (valid) rank[r] = wc[dg] + __popc(peers & lt);
+        __syncwarp();
+        if (valid && (peers & lt) == 0) wc[dg] = uint16_t(wc[dg] + __popc(peers));
+      }
+      __syncwarp();
+    }
+    __syncthreads();
+    // per digit: the tile's count, the warps' offsets, publish, look back
+    uint32_t cnt[kBPT], csum = 0;
+#pragma unroll
+    for (uint32_t b = 0; b < kBPT; ++b) {
+      const uint32_t bin = threadIdx.x * kBPT + b;
+      uint32_t run = 0;
+#pragma unroll
+      for (int w = 0; w < kFT / 32; ++w) {
+        const uint32_t v = s_wc[w][bin];
+        s_wc[w][bin] = uint16_t(run);
+        run += v;
+      }
+      cnt[b] = run;
+      csum += run;
+      __stcg(const_cast<uint32_t*>(status) + tile * kBins + bin, (tile == 0 ? kFlagP : kFlagA) | run);
+    }
+    uint32_t tsum;
+    uint32_t st = block_excl_scan(csum, s_w, tsum);
+#pragma unroll
+    for (uint32_t b = 0; b < kBPT; ++b) {
+      const uint32_t bin = threadIdx.x * kBPT + b;
+      s_start[bin] = st;
+      st += cnt[b];
+      uint32_t excl = 0;
+      for (int64_t pt = int64_t(tile) - 1; pt >= 0;) {   // decoupled look-back
+        const uint32_t v = status[uint64_t(pt) * kBins + bin];
+        if (v & kFlagP) { excl += v & kValMask; break; }
+        if (v & kFlagA) { excl += v & kValMask; --pt; }
+      }
+      if (tile) __stcg(const_cast<uint32_t*>(status) + tile * kBins + bin, kFlagP | (excl + cnt[b]));
+      s_goff[bin] = s_gstart[bin] + excl;
+    }
+    __syncthreads();
+#pragma unroll
+    for (uint32_t r = 0; r < kR; ++r) {
+      if (kr[r] == ~0ull) continue;
+      const uint32_t dg = uint32_t(kr[r] >> shift) & (kBins - 1);
+      s_keys[s_start[dg] + wc[dg] + rank[r]] = kr[r];
+    }
+    __syncthreads();
+    const uint32_t tn = uint32_t(min(uint64_t(kFreqTileKeys), n - tile * kFreqTileKeys));
+    for (uint32_t j = threadIdx.x; j < tn; j += kFT) {
+      const uint64_t key = s_keys[j];
+      const uint32_t dg = uint32_t(key >> shift) & (kBins - 1);
+      dst[s_goff[dg] + (j - s_start[dg])] = key;
+    }
+    __syncthreads();
+  }
+}
+
 // ---------------------------------------------------------------- 3. sweep
 // split = first key of the call's last API (carried to the next call);
 // queries (mode 1) sweep every key
@@ -602,15 +767,29 @@ __global__ void freq_carry_ctl_kernel(const __grid_constant__ FreqParams q) {
 #ifndef DRGPUM_FQ_GRID
 #define DRGPUM_FQ_GRID 4
 #endif
+#ifndef DRGPUM_FQ_ONESWEEP
+#define DRGPUM_FQ_ONESWEEP 1
+#endif
 static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& launches) {
   const unsigned g = unsigned(num_sms) * DRGPUM_FQ_GRID;
+  cudaMemsetAsync(q.ctl + 8, 0, 8 * (kFreqCtlWords - 8), s);   // skip flags, tickets, totals
+#if DRGPUM_FQ_ONESWEEP
+  freq_hist_all_kernel<<<g, kFT, 0, s>>>(q);
+  freq_skip_kernel<<<1, kFT, 0, s>>>(q);
+  launches += 2;
   for (uint32_t d = 0; d < q.n_digits; ++d) {
-    cudaMemsetAsync(q.ctl + 16, 0, 8 * kBins, s);
+    cudaMemsetAsync(q.hist, 0, 4ull * kBins * q.max_tiles, s);   // look-back status
+    freq_onesweep_kernel<<<g, kFT, 0, s>>>(q, d);
+    launches += 1;
+  }
+#else
+  for (uint32_t d = 0; d < q.n_digits; ++d) {
     freq_hist_kernel<<<g, kFT, 0, s>>>(q, d);
     freq_offsets_kernel<<<kBins, kFT, 0, s>>>(q, d);
     freq_scatter_kernel<<<g, kFT, 0, s>>>(q, d);
     launches += 3;
   }
+#endif
 }
 
 static void sweep(const FreqParams& q, unsigned long long* acc, uint32_t mode, int num_sms, cudaStream_t s,

@@ -114,7 +114,11 @@ struct SaParams {
 #endif
 constexpr uint32_t kFreqTileKeys = DRGPUM_FQ_TILE;   // radix-sort tile (256 threads x 16 keys)
 constexpr uint32_t kFreqRadixBits = 9;          // digit width of the LSD passes (512 bins)
-constexpr uint32_t kFreqCtlWords = 16 + (1u << kFreqRadixBits);   // control words (u64)
+// control words (u64): [0..8) counts / buffer / split, [8..16) per-pass skip
+// flags, [16..24) per-pass tile tickets, [32..) per-pass digit totals
+constexpr uint32_t kFreqCtlTot = 32;
+constexpr uint32_t kFreqMaxDigits = 8;
+constexpr uint32_t kFreqCtlWords = kFreqCtlTot + kFreqMaxDigits * (1u << kFreqRadixBits);
 constexpr uint32_t kFreqScanItems = 2048;       // entries per block of the digit-offset scan
 struct FreqParams {
   AttrParams a;                  // records of this (sub-)call, object table, index, rank table
