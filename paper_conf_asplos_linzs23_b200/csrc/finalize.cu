@@ -767,19 +767,50 @@ int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_by
 // one warp per object for the hit rows; only objects with first[o] != NEVER
 // hold nonzero words.  Tiles start 4-word aligned inside 4-word padded
 // bitmaps, so whole 16-B stores cover them.
+template <bool kLane>
 __global__ void __launch_bounds__(256) reset_touched_kernel(uint32_t* __restrict__ orw,
     const Tile* __restrict__ tiles, uint64_t n_tiles, const DevObj* __restrict__ objs,
     const uint32_t* __restrict__ n_hit, const uint32_t* __restrict__ first, uint64_t n_obj) {
   const int lane = threadIdx.x & 31;
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
-  // one warp per tile (the zeroing is the work: up to 1024 words each)
-  for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
-    const Tile tl = tiles[t];
-    if (__ldg(first + tl.obj) == kNever) continue;   // warp-uniform
-    uint4* v = reinterpret_cast<uint4*>(orw + tl.word_lo);
-    const uint32_t nv = (tl.n_words + 3) / 4;
-    for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
+  if (kLane) {
+    // mostly small tiles (C5's 10^6 objects): 32 tiles per warp step, each
+    // lane checks one and zeroes it itself if it is small; large touched
+    // tiles are zeroed by the whole warp
+    for (uint64_t t0 = gwarp * 32; t0 < n_tiles; t0 += nwarps * 32) {
+      const uint64_t t = t0 + lane;
+      bool big = false;
+      if (t < n_tiles) {
+        const Tile tl = tiles[t];
+        if (__ldg(first + tl.obj) != kNever) {
+          const uint32_t nv = (tl.n_words + 3) / 4;
+          if (nv <= 32) {
+            uint4* v = reinterpret_cast<uint4*>(orw + tl.word_lo);
+            for (uint32_t i = 0; i < nv; ++i) v[i] = make_uint4(0, 0, 0, 0);
+          } else {
+            big = true;
+          }
+        }
+      }
+      uint32_t m = __ballot_sync(FULL_MASK, big);
+      while (m) {
+        const Tile tl = tiles[t0 + uint32_t(__ffs(m) - 1)];
+        m &= m - 1;
+        uint4* v = reinterpret_cast<uint4*>(orw + tl.word_lo);
+        const uint32_t nv = (tl.n_words + 3) / 4;
+        for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
+      }
+    }
+  } else {
+    // one warp per tile (the zeroing is the work: up to 1024 words each)
+    for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
+      const Tile tl = tiles[t];
+      if (__ldg(first + tl.obj) == kNever) continue;   // warp-uniform
+      uint4* v = reinterpret_cast<uint4*>(orw + tl.word_lo);
+      const uint32_t nv = (tl.n_words + 3) / 4;
+      for (uint32_t i = lane; i < nv; i += 32) v[i] = make_uint4(0, 0, 0, 0);
+    }
   }
   for (uint64_t o0 = gwarp * 32; o0 < n_obj; o0 += nwarps * 32) {   // hit rows, 32 objects per step
     const uint64_t o = o0 + lane;
@@ -802,13 +833,16 @@ __global__ void __launch_bounds__(256) reset_touched_kernel(uint32_t* __restrict
 }
 
 int launch_reset_touched(uint32_t* orw, const Tile* tiles, uint64_t n_tiles, const DevObj* objs,
-                         const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, int num_sms,
-                         cudaStream_t s) {
+                         const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, bool lane_tiles,
+                         int num_sms, cudaStream_t s) {
   const uint64_t work = n_tiles > n_obj / 32 ? n_tiles : n_obj / 32;
   if (!n_tiles && !n_obj) return 0;
   uint64_t b = (work + 7) / 8 + 1;
   if (b > uint64_t(num_sms) * 16) b = uint64_t(num_sms) * 16;
-  reset_touched_kernel<<<(unsigned)b, 256, 0, s>>>(orw, tiles, n_tiles, objs, n_hit, first, n_obj);
+  if (lane_tiles)
+    reset_touched_kernel<true><<<(unsigned)b, 256, 0, s>>>(orw, tiles, n_tiles, objs, n_hit, first, n_obj);
+  else
+    reset_touched_kernel<false><<<(unsigned)b, 256, 0, s>>>(orw, tiles, n_tiles, objs, n_hit, first, n_obj);
   return 1;
 }
 

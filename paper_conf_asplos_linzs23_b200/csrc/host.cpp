@@ -77,6 +77,7 @@ struct drgpum_ctx {
   std::vector<Group> groups;
   std::vector<uint32_t> group_off;
   std::vector<uint64_t> small_prefix;   // finalize: prefix count of lane-foldable objects
+  uint64_t n_small_tiles = 0;           // tiles of <= 128 words (the sparse reset's lane mode)
   std::vector<drgpum_object_layout_t> layout;
   uint64_t bitmap_words = 0, hit_words = 0;
   uint32_t rq_cap = 1u << 20;
@@ -262,6 +263,8 @@ drgpum_status build_tables(drgpum_ctx* c) {
     bw += align_up(words, 4);
   }
   if (c->tiles.size() >= 0xFFFFFFFFull) return fail(c, DRGPUM_ENOMEM, "too many reduction tiles");
+  c->n_small_tiles = 0;
+  for (const Tile& t : c->tiles) c->n_small_tiles += t.n_words <= 128;
   c->tile_off[n] = (uint32_t)c->tiles.size();
   c->groups.clear();
   c->group_off.assign(n + 1, 0);
@@ -421,7 +424,8 @@ drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s, bool dense) {
     ctx->launches += launch_reset_touched(at<uint32_t>(ctx, ctx->L.orw), at<Tile>(ctx, ctx->L.tiles),
                                           ctx->tiles.size(), at<DevObj>(ctx, ctx->L.objs),
                                           at<uint32_t>(ctx, ctx->L.n_hit), at<uint32_t>(ctx, ctx->L.first),
-                                          ctx->n_obj, ctx->num_sms, s);
+                                          ctx->n_obj, 2 * ctx->n_small_tiles > ctx->tiles.size(),
+                                          ctx->num_sms, s);
     ctx->launches += launch_reset(ctx->ws + ctx->L.first, ctx->L.dyn_end - ctx->L.first, 0, 4 * ctx->n_obj,
                                   ctx->num_sms, s);
   }
@@ -542,6 +546,7 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   ctx->acc_rank.swap(tmp.acc_rank); ctx->acc_ts.swap(tmp.acc_ts); ctx->acc_cs.swap(tmp.acc_cs);
   ctx->n_hit.swap(tmp.n_hit); ctx->tiles.swap(tmp.tiles); ctx->tile_off.swap(tmp.tile_off);
   ctx->groups.swap(tmp.groups); ctx->group_off.swap(tmp.group_off); ctx->small_prefix.clear();
+  ctx->n_small_tiles = tmp.n_small_tiles;
   ctx->elem_base.swap(tmp.elem_base); ctx->n_elem_total = tmp.n_elem_total;
   ctx->slot_base.swap(tmp.slot_base); ctx->n_slots = tmp.n_slots;
   ctx->fq_pos_bits = tmp.fq_pos_bits; ctx->fq_digits = tmp.fq_digits;

@@ -236,8 +236,8 @@ int launch_reset(void* ws, uint64_t bytes, uint64_t first_off, uint64_t first_by
 // objects whose first[] is not NEVER (every attributed or merged bit of an
 // object comes with a first-use fold, so the others are still all zero).
 int launch_reset_touched(uint32_t* orw, const Tile* tiles, uint64_t n_tiles, const DevObj* objs,
-                         const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, int num_sms,
-                         cudaStream_t s);
+                         const uint32_t* n_hit, const uint32_t* first, uint64_t n_obj, bool lane_tiles,
+                         int num_sms, cudaStream_t s);
 int launch_merge_peers(const MergePeersParams& q, int num_sms, cudaStream_t s);
 int launch_merge_owned(const MergeOwnedParams& q, int num_sms, cudaStream_t s);
 int launch_merge_owned_sparse(const MergeOwnedParams& q, int num_sms, cudaStream_t s);
