@@ -42,6 +42,9 @@ constexpr int kFT = 256;                       // threads per block, every kerne
 constexpr uint32_t kSweepItems = 8;            // keys per thread in the sweep
 constexpr uint32_t kSweepChunk = kFT * kSweepItems;
 constexpr uint32_t kSweepSample = 2048;        // object bases staged per block for the sweep's search
+#ifndef DRGPUM_FQ_ONESWEEP
+#define DRGPUM_FQ_ONESWEEP 1   // one-sweep radix passes; digit totals counted where the keys are written
+#endif
 constexpr uint32_t kBins = 1u << kFreqRadixBits;  // digit values per radix pass
 constexpr uint32_t kBPT = kBins / kFT;            // bins per thread
 static_assert(kBins % kFT == 0, "bins are spread evenly over the threads");
@@ -109,12 +112,33 @@ __device__ __forceinline__ uint64_t n_keys(const FreqParams& q) {
 }
 
 // ---------------------------------------------------------------- 1. events
+// Every pass's digit totals, counted where the keys are written (the event
+// kernel, and the carry kernel for the carried keys): per-block shared
+// histograms, flushed once per block.
+struct DigitHist {
+  uint32_t h[kFreqMaxDigits][kBins];
+  __device__ void zero() {
+    for (uint32_t i = threadIdx.x; i < kFreqMaxDigits * kBins; i += blockDim.x) h[i / kBins][i % kBins] = 0;
+  }
+  __device__ void add(uint64_t key, uint32_t nd) {
+    for (uint32_t d = 0; d < nd; ++d) atomicAdd(&h[d][uint32_t(key >> (kFreqRadixBits * d)) & (kBins - 1)], 1u);
+  }
+  __device__ void flush(const FreqParams& q) {
+    for (uint32_t i = threadIdx.x; i < q.n_digits * kBins; i += blockDim.x) {
+      const uint32_t v = h[i / kBins][i % kBins];
+      if (v) atomicAdd(q.ctl + kFreqCtlTot + i, (unsigned long long)v);
+    }
+  }
+};
+
 // Keys are staged per warp in shared memory and flushed 256 at a time with
 // ONE atomic on the global key count (a per-tile atomic on that single
 // address serialised the kernel: 3e6 same-address atomics on C2).
 constexpr uint32_t kEvBuf = 256;
 __device__ __forceinline__ void ev_flush(const FreqParams& q, uint64_t* out, const uint64_t* buf, uint32_t cnt,
-                                         int lane) {
+                                         int lane, DigitHist& dh) {
+  if (DRGPUM_FQ_ONESWEEP)
+    for (uint32_t j = lane; j < cnt; j += 32) dh.add(buf[j], q.n_digits);
   unsigned long long base = 0;
   if (lane == 0 && cnt) base = atomicAdd(&q.ctl[0], (unsigned long long)cnt);
   base = __shfl_sync(FULL_MASK, base, 0);
@@ -128,6 +152,8 @@ __device__ __forceinline__ void ev_flush(const FreqParams& q, uint64_t* out, con
 
 __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant__ FreqParams q) {
   __shared__ uint64_t s_l1[kL1MaxKeys];
+  __shared__ DigitHist s_dh;
+  if (DRGPUM_FQ_ONESWEEP) s_dh.zero();
   __shared__ uint64_t s_ev[kFT / 32][kEvBuf];
   const AttrParams& p = q.a;
   for (uint32_t j = threadIdx.x; j < p.n_l1; j += blockDim.x) s_l1[j] = p.l1[j];
@@ -176,7 +202,7 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
     if (!cnt) continue;
     if (nbuf + cnt > kEvBuf) {                       // warp-uniform
       __syncwarp();
-      ev_flush(q, out, buf, nbuf, lane);
+      ev_flush(q, out, buf, nbuf, lane, s_dh);
       __syncwarp();
       nbuf = 0;
     }
@@ -187,8 +213,12 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
     nbuf += cnt;
   }
   __syncwarp();
-  ev_flush(q, out, buf, nbuf, lane);
+  ev_flush(q, out, buf, nbuf, lane, s_dh);
   if (__any_sync(FULL_MASK, unsorted) && lane == 0) atomicOr(q.state, 1u);
+  if (DRGPUM_FQ_ONESWEEP) {
+    __syncthreads();
+    s_dh.flush(q);
+  }
 }
 
 // ---------------------------------------------------------------- 2. radix sort
@@ -459,43 +489,13 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
   }
 }
 
-// ---- one-sweep form (default): every pass's digit totals from one read of
-// the keys, then ONE kernel per pass: tiles taken in order from a ticket,
+// ---- one-sweep form (default): every pass's digit totals counted where the
+// keys were written (event kernel, carry kernel), then ONE kernel per pass: tiles taken in order from a ticket,
 // ranked as above, their digit counts published and the exclusive prefix over
 // the previous tiles found by decoupled look-back (flag A: the tile's own
 // count, flag P: the inclusive prefix), so no per-pass histogram kernel and
 // no offset scan.
 constexpr uint32_t kFlagA = 1u << 30, kFlagP = 1u << 31, kValMask = kFlagA - 1;
-
-__global__ void __launch_bounds__(kFT) freq_hist_all_kernel(const __grid_constant__ FreqParams q) {
-  __shared__ uint32_t s_h[kFreqMaxDigits][kBins];
-  const uint64_t n = n_keys(q);
-  const uint64_t* src = keys_buf(q, uint32_t(q.ctl[1]));
-  const int lane = threadIdx.x & 31;
-  const uint32_t nd = q.n_digits;
-  for (uint32_t i = threadIdx.x; i < nd * kBins; i += kFT) s_h[i / kBins][i % kBins] = 0;
-  __syncthreads();
-  const uint64_t nth = uint64_t(gridDim.x) * kFT;
-  for (uint64_t i0 = uint64_t(blockIdx.x) * kFT; i0 < n; i0 += nth) {
-    const uint64_t i = i0 + threadIdx.x;
-    const bool valid = i < n;
-    const uint64_t key = valid ? __ldcs(src + i) : 0ull;
-    for (uint32_t d = 0; d < nd; ++d) {
-      const uint32_t dg = valid ? uint32_t(key >> (kFreqRadixBits * d)) & (kBins - 1) : kBins;
-      const uint32_t d0 = __shfl_sync(FULL_MASK, dg, 0);
-      if (__all_sync(FULL_MASK, dg == d0)) {
-        if (lane == 0 && d0 < kBins) atomicAdd(&s_h[d][d0], 32u);
-      } else if (valid) {
-        atomicAdd(&s_h[d][dg], 1u);
-      }
-    }
-  }
-  __syncthreads();
-  for (uint32_t i = threadIdx.x; i < nd * kBins; i += kFT) {
-    const uint32_t v = s_h[i / kBins][i % kBins];
-    if (v) atomicAdd(digit_totals(q, i / kBins) + (i % kBins), (unsigned long long)v);
-  }
-}
 
 // skip flags of every pass (a pass whose digit is the same for every key)
 __global__ void __launch_bounds__(kFT) freq_skip_kernel(const __grid_constant__ FreqParams q) {
@@ -745,13 +745,23 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
 
 // ---------------------------------------------------------------- 4. carry
 __global__ void __launch_bounds__(kFT) freq_carry_kernel(const __grid_constant__ FreqParams q) {
+  __shared__ DigitHist s_dh;                          // the carried keys count toward the next sort
+  if (DRGPUM_FQ_ONESWEEP) s_dh.zero();
+  __syncthreads();
   const uint64_t n = n_keys(q), split = q.ctl[2];
   const uint32_t b = buf_before(q, q.n_digits);
   const uint64_t* src = keys_buf(q, b);
   uint64_t* dst = keys_buf(q, b ^ 1u);
   for (uint64_t i = split + uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n;
-       i += uint64_t(gridDim.x) * blockDim.x)
-    dst[i - split] = src[i];
+       i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t key = src[i];
+    dst[i - split] = key;
+    if (DRGPUM_FQ_ONESWEEP) s_dh.add(key, q.n_digits);
+  }
+  if (DRGPUM_FQ_ONESWEEP) {
+    __syncthreads();
+    s_dh.flush(q);
+  }
 }
 
 __global__ void freq_carry_ctl_kernel(const __grid_constant__ FreqParams q) {
@@ -767,22 +777,20 @@ __global__ void freq_carry_ctl_kernel(const __grid_constant__ FreqParams q) {
 #ifndef DRGPUM_FQ_GRID
 #define DRGPUM_FQ_GRID 4
 #endif
-#ifndef DRGPUM_FQ_ONESWEEP
-#define DRGPUM_FQ_ONESWEEP 1
-#endif
 static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& launches) {
   const unsigned g = unsigned(num_sms) * DRGPUM_FQ_GRID;
-  cudaMemsetAsync(q.ctl + 8, 0, 8 * (kFreqCtlWords - 8), s);   // skip flags, tickets, totals
 #if DRGPUM_FQ_ONESWEEP
-  freq_hist_all_kernel<<<g, kFT, 0, s>>>(q);
+  // digit totals: counted by the event kernel (and the previous call's carry)
+  cudaMemsetAsync(q.ctl + 8, 0, 8 * (kFreqCtlTot - 8), s);   // skip flags, tickets
   freq_skip_kernel<<<1, kFT, 0, s>>>(q);
-  launches += 2;
+  launches += 1;
   for (uint32_t d = 0; d < q.n_digits; ++d) {
     cudaMemsetAsync(q.hist, 0, 4ull * kBins * q.max_tiles, s);   // look-back status
     freq_onesweep_kernel<<<g, kFT, 0, s>>>(q, d);
     launches += 1;
   }
 #else
+  cudaMemsetAsync(q.ctl + 8, 0, 8 * (kFreqCtlWords - 8), s);   // skip flags, tickets, totals
   for (uint32_t d = 0; d < q.n_digits; ++d) {
     freq_hist_kernel<<<g, kFT, 0, s>>>(q, d);
     freq_offsets_kernel<<<kBins, kFT, 0, s>>>(q, d);
@@ -809,6 +817,8 @@ int launch_frequency(const FreqParams& q, int num_sms, cudaStream_t s) {
   launches += 1;
   radix_sort(q, num_sms, s, launches);
   sweep(q, q.acc, 0, num_sms, s, launches);
+  // the next sort's digit totals start with the carried keys
+  cudaMemsetAsync(q.ctl + kFreqCtlTot, 0, 8ull * kFreqMaxDigits * kBins, s);
   freq_carry_kernel<<<unsigned(num_sms) * 4, kFT, 0, s>>>(q);
   freq_carry_ctl_kernel<<<1, 1, 0, s>>>(q);
   return launches + 2;
