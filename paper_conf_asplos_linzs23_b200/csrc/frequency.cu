@@ -137,25 +137,8 @@ struct DigitHist {
 constexpr uint32_t kEvBuf = 256;
 __device__ __forceinline__ void ev_flush(const FreqParams& q, uint64_t* out, const uint64_t* buf, uint32_t cnt,
                                          int lane, DigitHist& dh) {
-  if (DRGPUM_FQ_ONESWEEP) {
-    // the warp's keys, 32 at a time: a digit the whole round shares (the high
-    // digits: one API's keys) is one shared atomic
-    for (uint32_t j0 = 0; j0 < cnt; j0 += 32) {
-      const uint32_t j = j0 + uint32_t(lane);
-      const bool v = j < cnt;
-      const uint64_t key = v ? buf[j] : buf[j0];
-      const uint32_t nv = min(32u, cnt - j0);
-      for (uint32_t d = 0; d < q.n_digits; ++d) {
-        const uint32_t dg = uint32_t(key >> (kFreqRadixBits * d)) & (kBins - 1);
-        const uint32_t d0 = __shfl_sync(FULL_MASK, dg, 0);
-        if (__all_sync(FULL_MASK, dg == d0)) {
-          if (lane == 0) atomicAdd(&dh.h[d][d0], nv);
-        } else if (v) {
-          atomicAdd(&dh.h[d][dg], 1u);
-        }
-      }
-    }
-  }
+  if (DRGPUM_FQ_ONESWEEP)
+    for (uint32_t j = lane; j < cnt; j += 32) dh.add(buf[j], q.n_digits);
   unsigned long long base = 0;
   if (lane == 0 && cnt) base = atomicAdd(&q.ctl[0], (unsigned long long)cnt);
   base = __shfl_sync(FULL_MASK, base, 0);
