@@ -15,9 +15,9 @@ from ._lib import (OBJECT_DTYPE, RECORD_DTYPE, STATS_DTYPE, REPORT_DTYPE, COUNTE
                    LAYOUT_DTYPE, NEVER, EA, LD, UA, ML, TI, DW, OA, OA_ACTIONABLE,
                    FLAG_NAMES, DrgpumError, EXPORTS, LIB_PATH, load, redundant_pairs, kahn_levels,
                    DEP_INTRA, DEP_RAW, DEP_WAW, DEP_WAR)
-from .session import Session
+from .session import Session, pinned_array
 
-__all__ = ["Session", "OBJECT_DTYPE", "RECORD_DTYPE", "STATS_DTYPE", "REPORT_DTYPE",
+__all__ = ["Session", "pinned_array", "OBJECT_DTYPE", "RECORD_DTYPE", "STATS_DTYPE", "REPORT_DTYPE",
            "COUNTERS_DTYPE", "LAYOUT_DTYPE", "NEVER", "EA", "LD", "UA", "ML", "TI", "DW",
            "OA", "OA_ACTIONABLE", "FLAG_NAMES", "DrgpumError", "EXPORTS", "LIB_PATH", "load",
            "redundant_pairs", "kahn_levels", "DEP_INTRA", "DEP_RAW", "DEP_WAW", "DEP_WAR"]

@@ -23,6 +23,25 @@ def _stream_handle(stream):
     return ctypes.c_void_p(s.cuda_stream)
 
 
+def pinned_array(n, dtype):
+    """A numpy array of n ``dtype`` elements in page-locked host memory (a
+    torch pinned allocation, kept alive by the array's base): outputs read
+    into it (``object_stats(out=...)``, ``patterns(out=...)``) copy at the
+    DMA rate instead of through the driver's pageable staging."""
+    dtype = np.dtype(dtype)
+    t = torch.empty(max(1, n) * dtype.itemsize, dtype=torch.uint8, pin_memory=True)
+    a = t.numpy()[:n * dtype.itemsize].view(dtype)
+    return a
+
+
+def _out(out, n, dtype):
+    if out is None:
+        return np.zeros(n, dtype=dtype)
+    if out.dtype != dtype or out.shape != (n,) or not out.flags.c_contiguous:
+        raise ValueError(f"out must be a contiguous {dtype} array of {n} elements")
+    return out
+
+
 def _thresholds(th):
     if th is None:
         return Thresholds(2, 80, 80)
@@ -122,8 +141,8 @@ class Session:
         th = _thresholds(thresholds)
         check(self._h, self.L.drgpum_finalize(self._h, ctypes.byref(th), _stream_handle(stream)))
 
-    def object_stats(self, stream=None):
-        out = np.zeros(self.n_obj, dtype=STATS_DTYPE)
+    def object_stats(self, stream=None, out=None):
+        out = _out(out, self.n_obj, STATS_DTYPE)
         c = Counters()
         check(self._h, self.L.drgpum_object_stats(self._h, _np_ptr(out), ctypes.byref(c),
                                                   _stream_handle(stream)))
@@ -132,8 +151,8 @@ class Session:
             ctr[k] = getattr(c, k)
         return out, ctr
 
-    def patterns(self, thresholds=None, stream=None):
-        out = np.zeros(self.n_obj, dtype=REPORT_DTYPE)
+    def patterns(self, thresholds=None, stream=None, out=None):
+        out = _out(out, self.n_obj, REPORT_DTYPE)
         th = _thresholds(thresholds)
         check(self._h, self.L.drgpum_patterns(self._h, ctypes.byref(th), _np_ptr(out),
                                               _stream_handle(stream)))

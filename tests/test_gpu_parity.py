@@ -158,6 +158,26 @@ def test_reset_gives_a_fresh_trace(c1):
     assert np.array_equal(st1, st2) and c1_ == c2_
 
 
+def test_pinned_result_arrays(c1):
+    """object_stats / patterns into caller-owned page-locked arrays (the e2e
+    leg's form) equal the freshly allocated results, and a wrong out raises."""
+    from paper_conf_asplos_linzs23_b200 import pinned_array, STATS_DTYPE, REPORT_DTYPE
+    p, r = c1
+    s = _session(p.objects, p.kinds)
+    s.attribute(torch.from_numpy(r.view(np.uint8)).cuda())
+    st, ctr = s.object_stats()
+    rep = s.patterns()
+    hs, hr = pinned_array(p.n_obj, STATS_DTYPE), pinned_array(p.n_obj, REPORT_DTYPE)
+    hs.view(np.uint8)[:] = 0xAB       # stale contents must be overwritten
+    st2, ctr2 = s.object_stats(out=hs)
+    assert st2 is hs and np.array_equal(st.view(np.uint8), hs.view(np.uint8)) and ctr == ctr2
+    assert s.patterns(out=hr) is hr and np.array_equal(rep.view(np.uint8), hr.view(np.uint8))
+    with pytest.raises(ValueError):
+        s.object_stats(out=np.zeros(p.n_obj + 1, STATS_DTYPE))
+    with pytest.raises(ValueError):
+        s.patterns(out=np.zeros(p.n_obj, STATS_DTYPE))
+
+
 def test_empty_and_degenerate():
     # no records at all: every object unused
     p = build_tiny(7)
