@@ -1175,49 +1175,102 @@ __device__ __forceinline__ bool sa_claim(uint32_t* owner, uint32_t* overlap, uin
 constexpr uint32_t kSaInline = 64;          // elements claimed by the lane itself
 constexpr uint64_t kSaChunk = 4096;         // queued work item (elements)
 
-__global__ void __launch_bounds__(256) structured_kernel(const __grid_constant__ SaParams q) {
+constexpr uint32_t kSaUnroll = 4;           // records per lane per round (independent chains)
+
+// Queue a large element range (>= kSaInline elements) in kSaChunk pieces for
+// structured_range_kernel; claims in place when the queue is full.
+__device__ __noinline__ bool sa_enqueue(const SaParams& q, uint64_t g0, uint64_t g1, uint32_t tag, uint32_t obj) {
+  const uint64_t nch = (g1 - g0) / kSaChunk + 1;
+  const unsigned long long slot = atomicAdd(q.q_count, (unsigned long long)nch);
+  bool dead = false;
+  for (uint64_t k = 0; k < nch; ++k) {
+    const uint64_t lo = g0 + k * kSaChunk, hi = min(g1, lo + kSaChunk - 1);
+    if (slot + k < q.q_cap) {
+      q.q[slot + k] = SaRange{lo, hi, obj, tag, {0, 0}};
+    } else {
+      for (uint64_t g = lo; g <= hi && !dead; ++g) dead = sa_claim(q.owner, q.overlap, g, tag, obj);
+    }
+  }
+  return dead;
+}
+
+// Every warp owns a contiguous span of records and reads it 32 x kSaUnroll
+// records per round (coalesced, streamed past L2), so a lane's consecutive
+// records are 32 apart -- inside one burst, where its object and API caches
+// hit.  The kSaUnroll records' owner reads are issued together before any
+// CAS, so each lane keeps kSaUnroll independent load chains in flight.
+__global__ void __launch_bounds__(256, 4) structured_kernel(const __grid_constant__ SaParams q) {
   const AttrParams& p = q.a;
-  const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-  const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
-  // per-thread object cache: records of a thread are strided, but bursts are
-  // long, so consecutive records of one thread still share objects
+  const int lane = threadIdx.x & 31;
+  const uint64_t gw = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  constexpr uint64_t kRound = 32ull * kSaUnroll;
+  const uint64_t per = ((p.n + nw - 1) / nw + kRound - 1) / kRound * kRound;
+  const uint64_t w_lo = gw * per, w_hi = min(p.n, w_lo + per);
+  // per-lane object cache (+ whether the cached object is already overlapped)
   uint64_t c_base = 0, c_size = 0, c_eb = 0;
   uint32_t c_ta = 0, c_tf = 0, c_obj = kNone, c_shift = 0;
-  bool c_dead = false;                        // cached object already overlapped: SA decided
-  for (uint64_t i = tid; i < p.n; i += nth) {
-    const uint4 r = p.recs[i];
-    const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
-    const uint32_t size = r.z, ts = r.w & 0x7FFFFFFFu;
-    if (size == 0 || ts >= p.n_api || addr > ~0ull - size) continue;
-    const uint32_t rank = __ldg(p.acc_rank + ts);
-    if (rank == kNone || !__ldg(q.in_group + ts)) continue;
-    if (!(addr - c_base < c_size && ts > c_ta && ts < c_tf)) {
-      const uint32_t o = find_object(p, p.l1, addr, ts);   // level-1 keys from global here
-      if (o == kNone) continue;
-      const DevObj d = p.objs[o];
-      if (ts >= d.t_free) continue;
-      c_base = d.base; c_size = d.end - d.base; c_ta = d.t_alloc; c_tf = d.t_free;
-      c_obj = o; c_shift = d.shift; c_eb = __ldg(q.elem_base + o);
-      c_dead = __ldcg(q.overlap + o) != 0;
+  bool c_dead = false;
+  uint32_t c_ts = ~0u, c_tag = 0;             // per-lane API cache: tag 0 = not in the pass
+  for (uint64_t b = w_lo; b < w_hi; b += kRound) {
+    // another lane or warp may have decided the cached object meanwhile: its
+    // flag is re-read every round (in flight together with the records)
+    const uint32_t ov_now = (c_obj != kNone && !c_dead) ? __ldcg(q.overlap + c_obj) : 0u;
+    uint4 r[kSaUnroll];
+#pragma unroll
+    for (uint32_t k = 0; k < kSaUnroll; ++k) {
+      const uint64_t i = b + k * 32 + uint64_t(lane);
+      r[k] = i < w_hi ? __ldcs(p.recs + i) : make_uint4(0, 0, 0, 0);
     }
-    if (c_dead) continue;
-    const uint64_t off = addr - c_base;
-    const uint64_t end = min(off + size, c_size);
-    const uint64_t e0 = off >> c_shift, e1 = (end - 1) >> c_shift;
-    const uint32_t tag = rank + 1;
-    if (e1 - e0 < kSaInline) {
-      for (uint64_t e = e0; e <= e1 && !c_dead; ++e) c_dead = sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
-      continue;
-    }
-    const uint64_t nch = (e1 - e0) / kSaChunk + 1;
-    const unsigned long long slot = atomicAdd(q.q_count, (unsigned long long)nch);
-    for (uint64_t k = 0; k < nch; ++k) {
-      const uint64_t lo = e0 + k * kSaChunk, hi = min(e1, lo + kSaChunk - 1);
-      if (slot + k < q.q_cap) {
-        q.q[slot + k] = SaRange{c_eb + lo, c_eb + hi, c_obj, tag, {0, 0}};
-      } else {
-        for (uint64_t e = lo; e <= hi && !c_dead; ++e) c_dead = sa_claim(q.owner, q.overlap, c_eb + e, tag, c_obj);
+    if (ov_now) c_dead = true;
+    uint64_t g[kSaUnroll];
+    uint32_t cnt[kSaUnroll], tag[kSaUnroll], obj[kSaUnroll], cur[kSaUnroll];
+#pragma unroll
+    for (uint32_t k = 0; k < kSaUnroll; ++k) {
+      cnt[k] = 0; g[k] = 0; tag[k] = 0; obj[k] = kNone;
+      const uint64_t addr = (uint64_t(r[k].y) << 32) | r[k].x;
+      const uint32_t size = r[k].z, ts = r[k].w & 0x7FFFFFFFu;
+      if (size == 0 || ts >= p.n_api || addr > ~0ull - size) continue;
+      if (ts != c_ts) {
+        const uint32_t rank = __ldg(p.acc_rank + ts);
+        c_ts = ts;
+        c_tag = (rank == kNone || !__ldg(q.in_group + ts)) ? 0u : rank + 1;
       }
+      if (c_tag == 0) continue;
+      if (!(addr - c_base < c_size && ts > c_ta && ts < c_tf)) {
+        const uint32_t o = find_object(p, p.l1, addr, ts);   // level-1 keys from global here
+        if (o == kNone) continue;
+        const DevObj d = p.objs[o];
+        if (ts >= d.t_free) continue;
+        c_base = d.base; c_size = d.end - d.base; c_ta = d.t_alloc; c_tf = d.t_free;
+        c_obj = o; c_shift = d.shift; c_eb = __ldg(q.elem_base + o);
+        c_dead = __ldcg(q.overlap + o) != 0;
+      }
+      if (c_dead) continue;
+      const uint64_t off = addr - c_base;
+      const uint64_t end = min(off + size, c_size);
+      const uint64_t e0 = off >> c_shift, e1 = (end - 1) >> c_shift;
+      if (e1 - e0 >= kSaInline) {
+        c_dead = sa_enqueue(q, c_eb + e0, c_eb + e1, c_tag, c_obj);
+        continue;
+      }
+      g[k] = c_eb + e0; cnt[k] = uint32_t(e1 - e0) + 1; tag[k] = c_tag; obj[k] = c_obj;
+    }
+#pragma unroll
+    for (uint32_t k = 0; k < kSaUnroll; ++k) cur[k] = cnt[k] ? q.owner[g[k]] : 0u;
+#pragma unroll
+    for (uint32_t k = 0; k < kSaUnroll; ++k) {
+      if (cnt[k] == 0) continue;
+      bool dead = false;
+      // first element: the owner value read above (0 -> the CAS decides)
+      uint32_t c0 = cur[k];
+      if (c0 == 0) c0 = atomicCAS(q.owner + g[k], 0u, tag[k]);
+      if (c0 != 0 && c0 != tag[k]) {
+        if (!__ldcg(q.overlap + obj[k])) red_or(q.overlap + obj[k], 1u);
+        dead = true;
+      }
+      for (uint32_t e = 1; e < cnt[k] && !dead; ++e) dead = sa_claim(q.owner, q.overlap, g[k] + e, tag[k], obj[k]);
+      if (dead && obj[k] == c_obj) c_dead = true;
     }
   }
 }
@@ -1242,8 +1295,9 @@ __global__ void __launch_bounds__(256) structured_range_kernel(const __grid_cons
 int launch_structured(const SaParams& q, int num_sms, cudaStream_t s) {
   if (q.a.n == 0) return 0;
   cudaMemsetAsync(q.q_count, 0, sizeof(unsigned long long), s);
-  uint64_t blocks = (q.a.n + 255) / 256;
-  if (blocks > uint64_t(num_sms) * 8) blocks = uint64_t(num_sms) * 8;
+  // one round per warp at least; at most 4 blocks (32 warps) per SM
+  uint64_t blocks = (q.a.n + 8 * 32 * kSaUnroll - 1) / (8 * 32 * kSaUnroll);
+  if (blocks > uint64_t(num_sms) * 4) blocks = uint64_t(num_sms) * 4;
   structured_kernel<<<(unsigned)blocks, 256, 0, s>>>(q);
   structured_range_kernel<<<num_sms * 4, 256, 0, s>>>(q);
   return 2;
