@@ -266,7 +266,7 @@ struct SlowCache {                       // 56 B
   uint32_t t_alloc, t_free, r_lo, shift, obj;
   uint32_t meta;                         // ts|w<<31 whose first/last/hit work is done
 };
-struct FastCache { uint64_t base, size, bm_word; uint32_t shift, meta; };
+struct FastCache { uint64_t base, size, bm_word; uint32_t shift, meta; bool sc; };   // sc: scratch_ok
 
 // per warp, shared memory: record counters of the slow paths and the tile
 // counts by path (diagnostics; shared-memory REDs keep them out of registers)
@@ -342,8 +342,10 @@ __device__ __forceinline__ WarpCounts* slow_counts() {
 }
 
 
+// small object: its whole bitmap fits the per-warp scratch (kScratchWords, below)
+__device__ __forceinline__ bool small_object(uint64_t size, uint32_t shift);
 __device__ __forceinline__ FastCache mirror(const SlowCache* c) {
-  return FastCache{c->base, c->size, c->bm_word, c->shift, c->meta};
+  return FastCache{c->base, c->size, c->bm_word, c->shift, c->meta, small_object(c->size, c->shift)};
 }
 
 __device__ __forceinline__ SegEntry ldg_seg(const SegEntry* e) {
@@ -567,20 +569,31 @@ __device__ __noinline__ void process_slow(const AttrParams& p, uint4 r, bool pre
 // OR the element range [e0, e1] (at most two words) of an object's bitmap.
 // OR is idempotent, so records sharing a word need no warp-level merge; the
 // L2 atomic units have the headroom (ncu: ~15% busy), the issue slots do not.
+// Elements [e0, e0 + len] (len < 32) as the masks of word e0 >> 5 (lo) and
+// of the next word (hi, 0 when the range stays in one word): len + 1 ones
+// shifted left by e0 % 32 across the 64-bit word pair (two funnel shifts,
+// which take the shift modulo 32).
+__device__ __forceinline__ void range_masks(uint32_t e0, uint32_t len, uint32_t& lo, uint32_t& hi) {
+  const uint32_t m = (2u << len) - 1u;   // len = 31: 2 << 31 = 0 in 32 bits -> all ones
+  lo = __funnelshift_l(0u, m, e0);
+  hi = __funnelshift_l(m, 0u, e0);
+}
+__device__ __forceinline__ void red_range(uint32_t* orw, uint64_t bm_word, uint32_t e0, uint32_t len) {
+  uint32_t lo, hi;
+  range_masks(e0, len, lo, hi);
+  uint32_t* a = orw + bm_word + (e0 >> 5);
+  red_or(a, lo);
+  if (hi) red_or(a + 1, hi);
+}
 __device__ __forceinline__ void red_record(uint32_t* orw, uint64_t bm_word, uint32_t e0, uint32_t e1) {
-  const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
-  if (w1 == w0) {
-    red_or(orw + bm_word + w0, bits_mask(e0 & 31, e1 & 31));
-  } else {
-    red_or(orw + bm_word + w0, 0xFFFFFFFFu << (e0 & 31));
-    red_or(orw + bm_word + w1, 0xFFFFFFFFu >> (31 - (e1 & 31)));
-  }
+  red_range(orw, bm_word, e0, e1 - e0);
 }
 
 // --- small-object scratch (warp-uniform calls)
-__device__ __forceinline__ bool scratch_ok(const FastCache& c) {
-  return kScratchWords > 0 && c.size <= (uint64_t(kScratchWords) * 32) << c.shift;
+__device__ __forceinline__ bool small_object(uint64_t size, uint32_t shift) {
+  return kScratchWords > 0 && size <= (uint64_t(kScratchWords) * 32) << shift;
 }
+__device__ __forceinline__ bool scratch_ok(const FastCache& c) { return c.sc; }
 __device__ __forceinline__ void red_shared_or(uint32_t a, uint32_t v) {
   asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
@@ -609,14 +622,15 @@ __device__ __forceinline__ void scratch_bind(uint32_t wsm, uint32_t* orw, uint64
   if (lane == 0) sts64(wsm + kOffScBase, bm_word);
   __syncwarp();
 }
+__device__ __forceinline__ void scratch_range(uint32_t wsm, uint32_t e0, uint32_t len) {
+  uint32_t lo, hi;
+  range_masks(e0, len, lo, hi);
+  const uint32_t a = wsm + kOffScratch + 4 * (e0 >> 5);
+  red_shared_or(a, lo);
+  if (hi) red_shared_or(a + 4, hi);
+}
 __device__ __forceinline__ void scratch_record(uint32_t wsm, uint32_t e0, uint32_t e1) {
-  const uint32_t w0 = e0 >> 5, w1 = e1 >> 5;
-  if (w1 == w0) {
-    red_shared_or(wsm + kOffScratch + 4 * w0, bits_mask(e0 & 31, e1 & 31));
-  } else {
-    red_shared_or(wsm + kOffScratch + 4 * w0, 0xFFFFFFFFu << (e0 & 31));
-    red_shared_or(wsm + kOffScratch + 4 * w1, 0xFFFFFFFFu >> (31 - (e1 & 31)));
-  }
+  scratch_range(wsm, e0, e1 - e0);
 }
 
 __device__ __forceinline__ void fast_or(uint32_t* orw, uint64_t bm_word, uint32_t e0, uint32_t e1, int lane) {
@@ -696,16 +710,19 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
   // mismatch bits of all four words of all records are ORed with 3-input
   // LOP3s (about 5 instructions per record)
   const uint32_t a0lo = __shfl_sync(FULL_MASK, r[0].x, 0);
-  const uint32_t a0hi = __shfl_sync(FULL_MASK, r[0].y, 0);
   const uint32_t st32 = __shfl_sync(FULL_MASK, r[0].x, 1) - a0lo;
-  const uint32_t sz = __shfl_sync(FULL_MASK, r[0].z, 0);
   uint32_t exp = a0lo + uint32_t(lane) * st32;
-  uint32_t bad = 0;
+  // the first tile's low address words first: most stages that are not
+  // affine (wrapping strided sweeps, gathers) fail here, before the rest
+  if (!__all_sync(FULL_MASK, r[0].x == exp)) return 0;
+  const uint32_t a0hi = __shfl_sync(FULL_MASK, r[0].y, 0);
+  const uint32_t sz = __shfl_sync(FULL_MASK, r[0].z, 0);
+  uint32_t bad = (r[0].y ^ a0hi) | (r[0].z ^ sz) | (r[0].w ^ c.meta);
 #pragma unroll
-  for (int k = 0; k < kTilesPerWarp; ++k) {
+  for (int k = 1; k < kTilesPerWarp; ++k) {
+    exp += 32u * st32;
     bad |= (r[k].x ^ exp) | (r[k].y ^ a0hi);
     bad |= (r[k].z ^ sz) | (r[k].w ^ c.meta);
-    exp += 32u * st32;
   }
   if (!__all_sync(FULL_MASK, bad == 0)) return 0;
   // uniform from here on: every lane holds the same values
@@ -746,7 +763,8 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
     }
     return 1;
   }
-  if (((sz - 1) >> c.shift) >= 32) return 0;   // records wider than a word: tile path
+  // records of up to 31 elements after the first (range_masks): wider ones take the tile path
+  if (((sz - 1) >> c.shift) >= 31) return 0;
   // not one range: every record ORs its own word(s) (offsets in 32 bits),
   // through the scratch for a small object
   uint32_t off = o0 + uint32_t(lane) * st32;
@@ -787,53 +805,56 @@ __device__ __forceinline__ int try_affine(const uint4 (&r)[kTilesPerWarp], const
 }
 
 // In-object tier: the warp's 128 records all carry the cached (API, rw) and
-// fall inside the cached object (< 4 GiB), unclipped, <= 2 words each, in any
+// start inside the cached object (< 4 GiB), <= 32 elements each after the
+// clip at the object's end, in any
 // order (random gathers, strided sweeps that wrap).  Each record ORs its own
 // word(s): no warp analysis, OR is idempotent.  Returns false without side
 // effects otherwise.
 __device__ __forceinline__ bool try_in_object(const uint4 (&r)[kTilesPerWarp], const FastCache& c,
                                               uint32_t* orw, uint32_t wsm, int lane) {
   const uint32_t osz = uint32_t(c.size);
-  uint32_t e0[kTilesPerWarp], e1[kTilesPerWarp];
+  uint32_t e0[kTilesPerWarp], ln[kTilesPerWarp];
   bool ok = true;
   uint32_t nclip = 0;
 #pragma unroll
   for (int k = 0; k < kTilesPerWarp; ++k) {
+    // off < c.size (< 2^32 here) also bounds the high word and off32 < osz
     const uint64_t off = ((uint64_t(r[k].y) << 32) | r[k].x) - c.base;
-    const uint32_t off32 = uint32_t(off), size = r[k].z, room = osz - off32;
-    const bool clip = size > room;   // runs past the object's end: clipped there (R3)
+    const uint32_t off32 = uint32_t(off), room = osz - off32;
+    const uint32_t sz = min(r[k].z, room);   // clipped at the object's end (R3)
+    nclip += r[k].z > room;
     e0[k] = off32 >> c.shift;
-    e1[k] = (off32 + (clip ? room : size) - 1) >> c.shift;
-    ok = ok && r[k].w == c.meta && (off >> 32) == 0 && off32 < osz && size != 0 &&
-         (e1[k] >> 5) - (e0[k] >> 5) < 2;
-    nclip += clip;
+    ln[k] = ((off32 + sz - 1) >> c.shift) - e0[k];
+    ok = ok && off < c.size && r[k].w == c.meta && r[k].z != 0 && ln[k] < 32;
   }
   if (!__all_sync(FULL_MASK, ok)) return false;
-  nclip = __reduce_add_sync(FULL_MASK, nclip);
-  if (nclip && lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, clip)>(wsm, nclip);
+  if (__any_sync(FULL_MASK, nclip != 0)) {
+    nclip = __reduce_add_sync(FULL_MASK, nclip);
+    if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, clip)>(wsm, nclip);
+  }
   if (scratch_ok(c)) {
     scratch_bind(wsm, orw, c.bm_word, lane);
 #pragma unroll
-    for (int k = 0; k < kTilesPerWarp; ++k) scratch_record(wsm, e0[k], e1[k]);
+    for (int k = 0; k < kTilesPerWarp; ++k) scratch_range(wsm, e0[k], ln[k]);
     return true;
   }
 #if DRGPUM_WINDOW
   {   // the 128 records of a large object within < 64 words: scratch window
-    uint32_t lo = e0[0], hi = e1[0];
+    uint32_t lo = e0[0], hi = e0[0] + ln[0];
 #pragma unroll
-    for (int k = 1; k < kTilesPerWarp; ++k) { lo = min(lo, e0[k]); hi = max(hi, e1[k]); }
+    for (int k = 1; k < kTilesPerWarp; ++k) { lo = min(lo, e0[k]); hi = max(hi, e0[k] + ln[k]); }
     const uint32_t lo_w = __reduce_min_sync(FULL_MASK, lo) >> 5, hi_w = __reduce_max_sync(FULL_MASK, hi) >> 5;
     if (kScratchWords >= 128 && hi_w - lo_w < 64) {
       const uint32_t wb = lo_w & ~63u;
       scratch_bind(wsm, orw, c.bm_word + wb, lane);
 #pragma unroll
-      for (int k = 0; k < kTilesPerWarp; ++k) scratch_record(wsm, e0[k] - 32 * wb, e1[k] - 32 * wb);
+      for (int k = 0; k < kTilesPerWarp; ++k) scratch_range(wsm, e0[k] - 32 * wb, ln[k]);
       return true;
     }
   }
 #endif
 #pragma unroll
-  for (int k = 0; k < kTilesPerWarp; ++k) red_record(orw, c.bm_word, e0[k], e1[k]);
+  for (int k = 0; k < kTilesPerWarp; ++k) red_range(orw, c.bm_word, e0[k], ln[k]);
   return true;
 }
 
@@ -863,7 +884,7 @@ __device__ __noinline__ bool try_uniform_slow(const AttrParams& p, uint4 r, bool
   const uint64_t off = addr - base;
   const uint32_t size = r.z;
   const uint32_t off32 = uint32_t(off), e0 = off32 >> d.w, e1 = (off32 + size - 1) >> d.w;
-  const bool ok = off < osz && size != 0 && size <= uint32_t(osz) - off32 && (e1 >> 5) - (e0 >> 5) < 2;
+  const bool ok = off < osz && size != 0 && size <= uint32_t(osz) - off32 && e1 - e0 < 32;
   if (!__all_sync(FULL_MASK, ok)) return false;
   c->base = base; c->size = osz;
   c->bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
@@ -1030,7 +1051,6 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
       }
       if (try_in_object(r4, c, p.orw, wsm, lane)) {
         fast_rec += kTilesPerWarp;
-        if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, fast)>(wsm, kTilesPerWarp);
         continue;
       }
     }
@@ -1048,13 +1068,12 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
         const uint32_t e0 = off32 >> c.shift;
         const uint32_t e1 = (off32 + (clip ? room : size) - 1) >> c.shift;
         const bool ok = present && r.w == c.meta && (off >> 32) == 0 && off32 < osz &&
-                        size != 0 && (e1 >> 5) - (e0 >> 5) < 2;
+                        size != 0 && e1 - e0 < 32;
         if (__all_sync(FULL_MASK, ok)) {
           const uint32_t nclip = __popc(__ballot_sync(FULL_MASK, clip));
           if (nclip && lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, clip)>(wsm, nclip);
           fast_or_c(wsm, p.orw, c, e0, e1, lane);
           ++fast_rec;
-          if (lane == 0) red_shared_add<kOffWc + offsetof(WarpCounts, fast)>(wsm, 1);
           continue;
         }
       }
@@ -1083,7 +1102,8 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
       if (v[i]) atomicAdd(&p.ctr[slot[i]], (unsigned long long)v[i]);
     atomicAdd(&p.ctr[C_TILES_AFFINE_UNION], (unsigned long long)wc->aff_u);
     atomicAdd(&p.ctr[C_TILES_AFFINE_WORDS], (unsigned long long)wc->aff_w);
-    atomicAdd(&p.ctr[C_TILES_FAST], (unsigned long long)wc->fast);
+    // fast tiles (in-object tier, tile fast path) = fast-path tiles - affine tiles
+    atomicAdd(&p.ctr[C_TILES_FAST], (unsigned long long)(fr / 32 - wc->aff_u - wc->aff_w));
     atomicAdd(&p.ctr[C_TILES_SLOW], (unsigned long long)wc->slow);
   }
 }

@@ -137,6 +137,8 @@ struct DigitHist {
 constexpr uint32_t kEvBuf = 256;
 __device__ __forceinline__ void ev_flush(const FreqParams& q, uint64_t* out, const uint64_t* buf, uint32_t cnt,
                                          int lane, DigitHist& dh) {
+  // per-lane shared atomics (aggregating a warp's uniform digits first, by a
+  // vote or by MATCH.ANY, measured slower: events 1.12 -> 1.6 / 2.05 ms on C2)
   if (DRGPUM_FQ_ONESWEEP)
     for (uint32_t j = lane; j < cnt; j += 32) dh.add(buf[j], q.n_digits);
   unsigned long long base = 0;
@@ -224,7 +226,11 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
 // ---------------------------------------------------------------- 2. radix sort
 // Lanes holding the same (kFreqRadixBits + 1)-bit value (the top bit = "no
 // key"): one ballot per bit.
+#ifndef DRGPUM_FQ_MATCH
+#define DRGPUM_FQ_MATCH 1   // peers by one MATCH.ANY (0: one ballot per bit; C2 pass 0.81 -> 0.73 ms)
+#endif
 __device__ __forceinline__ uint32_t peers_of(uint32_t v) {
+  if (DRGPUM_FQ_MATCH) return __match_any_sync(FULL_MASK, v);
   uint32_t m = FULL_MASK;
 #pragma unroll
   for (int b = 0; b <= int(kFreqRadixBits); ++b) {
@@ -495,6 +501,12 @@ __global__ void __launch_bounds__(kFT) freq_scatter_kernel(const __grid_constant
 // the previous tiles found by decoupled look-back (flag A: the tile's own
 // count, flag P: the inclusive prefix), so no per-pass histogram kernel and
 // no offset scan.
+// Look-back status per (tile, digit): flag A = the tile's own count, flag P =
+// inclusive prefix, 30-bit value.  Two status arrays alternate between the
+// passes (hist for even, offs for odd passes; offs is free in this form):
+// pass d clears, tile by tile, the rows pass d + 1 will use, so only the
+// first pass of a sort needs a memset (a u64 status tagged with a pass epoch
+// and no clearing measured slower: 0.73 -> 0.84 ms per pass on C2).
 constexpr uint32_t kFlagA = 1u << 30, kFlagP = 1u << 31, kValMask = kFlagA - 1;
 
 // skip flags of every pass (a pass whose digit is the same for every key)
@@ -508,14 +520,23 @@ __global__ void __launch_bounds__(kFT) freq_skip_kernel(const __grid_constant__ 
   }
 }
 
-__global__ void __launch_bounds__(kFT) freq_onesweep_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
+#ifndef DRGPUM_FQ_MINB
+#define DRGPUM_FQ_MINB 4   // blocks per SM of the one-sweep pass (register cap 64; C2: 0.755 -> 0.722 ms vs 3)
+#endif
+__global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
   __shared__ uint64_t s_keys[kFreqTileKeys];
   __shared__ uint16_t s_wc[kFT / 32][kBins];          // per-warp digit counts, then offsets (<= 4096)
   __shared__ uint32_t s_start[kBins], s_goff[kBins], s_gstart[kBins], s_w[kFT / 32];
   __shared__ uint32_t s_tile;
-  if (q.ctl[8 + d]) return;                          // every key has the same digit: pass skipped
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
+  volatile uint32_t* status = (d & 1) ? q.offs : q.hist;   // [tile][bin]
+  uint32_t* status_next = (d & 1) ? q.hist : q.offs;       // pass d + 1's, cleared here
+  if (q.ctl[8 + d]) {                                // every key has the same digit: pass skipped
+    for (uint64_t i = uint64_t(blockIdx.x) * kFT + threadIdx.x; i < ntiles * kBins; i += uint64_t(gridDim.x) * kFT)
+      status_next[i] = 0;
+    return;
+  }
   const uint32_t src_b = buf_before(q, d);
   const uint64_t* src = keys_buf(q, src_b);
   uint64_t* dst = keys_buf(q, src_b ^ 1u);
@@ -524,7 +545,6 @@ __global__ void __launch_bounds__(kFT) freq_onesweep_kernel(const __grid_constan
   const uint32_t lt = (1u << lane) - 1u;
   constexpr uint32_t kR = kFreqTileKeys / kFT;
   uint16_t* wc = s_wc[warp];
-  volatile uint32_t* status = q.hist;                // [tile][bin]
   {   // global digit starts of this pass (exclusive scan of the totals)
     const unsigned long long* tot = digit_totals(q, d);
     uint32_t c[kBPT], cs = 0;
@@ -586,6 +606,7 @@ __global__ void __launch_bounds__(kFT) freq_onesweep_kernel(const __grid_constan
       cnt[b] = run;
       csum += run;
       __stcg(const_cast<uint32_t*>(status) + tile * kBins + bin, (tile == 0 ? kFlagP : kFlagA) | run);
+      status_next[tile * kBins + bin] = 0;
     }
     uint32_t tsum;
     uint32_t st = block_excl_scan(csum, s_w, tsum);
@@ -781,11 +802,11 @@ static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& la
   const unsigned g = unsigned(num_sms) * DRGPUM_FQ_GRID;
 #if DRGPUM_FQ_ONESWEEP
   // digit totals: counted by the event kernel (and the previous call's carry)
-  cudaMemsetAsync(q.ctl + 8, 0, 8 * (kFreqCtlTot - 8), s);   // skip flags, tickets
+  cudaMemsetAsync(q.ctl + 8, 0, 8 * 16, s);   // skip flags, tickets
+  cudaMemsetAsync(q.hist, 0, 4ull * kBins * q.max_tiles, s);   // first pass's look-back status
   freq_skip_kernel<<<1, kFT, 0, s>>>(q);
   launches += 1;
   for (uint32_t d = 0; d < q.n_digits; ++d) {
-    cudaMemsetAsync(q.hist, 0, 4ull * kBins * q.max_tiles, s);   // look-back status
     freq_onesweep_kernel<<<g, kFT, 0, s>>>(q, d);
     launches += 1;
   }

@@ -129,7 +129,8 @@ struct FreqParams {
   uint32_t* state;               // [0] bit0 records out of order, bit1 event capacity exceeded;
                                  // [1] last timestamp of the previous call + 1 (0 = none)
   unsigned long long* ctl;       // [0] keys in the current buffer, [1] current buffer, [2] split,
-                                 // [8..16) skip flag per radix pass, [16..) digit totals
+                                 // [8..16) skip flag per radix pass, [16..24) tile tickets,
+                                 // [32..) digit totals
   uint64_t* keys0;               // event keys, ping-pong buffers of cap keys
   uint64_t* keys1;
   uint64_t cap;
