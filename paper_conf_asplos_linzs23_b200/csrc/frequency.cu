@@ -15,8 +15,10 @@
 //      [g0, g1] of global element indices it touches; consecutive records of
 //      a warp that touch adjacent, disjoint intervals of one object in one
 //      API (sequential sweeps) are merged into one interval first.  Each
-//      interval becomes two 64-bit keys (rank << pos_bits) | 2*g0 (start)
-//      and (rank << pos_bits) | 2*g1 + 1 (end); rank = access-API rank.
+//      interval becomes two 64-bit keys (rank << pos_bits) | 4*g0 (start)
+//      and (rank << pos_bits) | 4*g1 + 2 (end), a single-element interval
+//      ONE key (rank << pos_bits) | 4*g + 1 (point); rank = access-API rank
+//      (DRGPUM_FQ_POINTS=0: 2*g0 and 2*g1 + 1, no points).
 //   2. An LSD radix sort (8-bit digits, stable: tile histograms, a
 //      digit-major exclusive scan, a tile-local stable ranking through shared
 //      memory and coalesced stores) orders the keys by (API, element).
@@ -28,7 +30,8 @@
 //      (len, c*len, c*c*len) to (n, S1, S2) of its (object, API) slot
 //      (intervals never span objects or APIs, so runs with c > 0 do not
 //      either; every API's intervals are balanced, so no segmented scan is
-//      needed).
+//      needed).  Points do not change the count; the last of p equal point
+//      keys adds the p extra accesses of its element: (c == 0, p, 2cp + p^2).
 //   4. The call's last API may continue in the next call (records are in
 //      timestamp order across calls): its sorted keys are carried to the
 //      front of the other key buffer and sorted together with the next
@@ -137,8 +140,9 @@ struct DigitHist {
 constexpr uint32_t kEvBuf = 256;
 __device__ __forceinline__ void ev_flush(const FreqParams& q, uint64_t* out, const uint64_t* buf, uint32_t cnt,
                                          int lane, DigitHist& dh) {
-  // per-lane shared atomics (aggregating a warp's uniform digits first, by a
-  // vote or by MATCH.ANY, measured slower: events 1.12 -> 1.6 / 2.05 ms on C2)
+  // per-lane shared atomics: a warp vote (on every digit or only on the
+  // mostly uniform high digits) or a MATCH.ANY first measured slower --
+  // events 1.12 -> 1.6-2.05 ms on C2
   if (DRGPUM_FQ_ONESWEEP)
     for (uint32_t j = lane; j < cnt; j += 32) dh.add(buf[j], q.n_digits);
   unsigned long long base = 0;
@@ -200,7 +204,15 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
     const bool head = valid && !chain;
     const bool tail = valid && (lane == 31 || !((cb >> (lane + 1)) & 1u));
     const uint32_t hb = __ballot_sync(FULL_MASK, head), tb = __ballot_sync(FULL_MASK, tail);
-    const uint32_t cnt = __popc(hb) + __popc(tb);
+#if DRGPUM_FQ_POINTS
+    // a single-element interval is one point key: no end key
+    const bool pt = head && tail && g0 == g1;
+    const uint32_t eb_ = __ballot_sync(FULL_MASK, tail && !pt);
+#else
+    const bool pt = false;
+    const uint32_t eb_ = tb;
+#endif
+    const uint32_t cnt = __popc(hb) + __popc(eb_);
     if (!cnt) continue;
     if (nbuf + cnt > kEvBuf) {                       // warp-uniform
       __syncwarp();
@@ -210,8 +222,8 @@ __global__ void __launch_bounds__(kFT) freq_events_kernel(const __grid_constant_
     }
     const uint32_t lt = (1u << lane) - 1u;
     const uint64_t hi = uint64_t(rank) << q.pos_bits;
-    if (head) buf[nbuf + __popc(hb & lt)] = hi | (2 * g0);
-    if (tail) buf[nbuf + __popc(hb) + __popc(tb & lt)] = hi | (2 * g1 + 1);
+    if (head) buf[nbuf + __popc(hb & lt)] = hi | (kFreqPosMul * g0 + (pt ? 1 : 0));
+    if (tail && !pt) buf[nbuf + __popc(hb) + __popc(eb_ & lt)] = hi | (kFreqPosMul * g1 + kFreqPosMul / 2);
     nbuf += cnt;
   }
   __syncwarp();
@@ -520,6 +532,9 @@ __global__ void __launch_bounds__(kFT) freq_skip_kernel(const __grid_constant__ 
   }
 }
 
+#ifndef DRGPUM_FQ_ATOMRANK
+#define DRGPUM_FQ_ATOMRANK 1
+#endif
 #ifndef DRGPUM_FQ_MINB
 #define DRGPUM_FQ_MINB 4   // blocks per SM of the one-sweep pass (register cap 64; C2: 0.755 -> 0.722 ms vs 3)
 #endif
@@ -571,6 +586,26 @@ __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(cons
       kr[r] = idx < n ? __ldcs(src + idx) : ~0ull;
     }
     uint32_t rank[kR];
+#if DRGPUM_FQ_ATOMRANK
+    // each round's leader adds its peer count to the warp's digit counter with
+    // a returning shared atomic (two u16 counters per u32 word) and hands the
+    // old value to its peers: no read-modify-write chain through syncwarps,
+    // the rounds' atomics pipeline (same-address ones stay in program order)
+    uint32_t* wc32 = reinterpret_cast<uint32_t*>(wc);
+#pragma unroll
+    for (uint32_t r = 0; r < kR; ++r) {
+      const bool valid = kr[r] != ~0ull;
+      const uint32_t dg = valid ? uint32_t(kr[r] >> shift) & (kBins - 1) : kBins;
+      const uint32_t peers = peers_of(dg);
+      const int leader = __ffs(peers) - 1;
+      const uint32_t sh = (dg & 1u) * 16u;
+      uint32_t old = 0;
+      if (valid && leader == lane) old = atomicAdd(wc32 + (dg >> 1), uint32_t(__popc(peers)) << sh);
+      old = __shfl_sync(FULL_MASK, old, leader);
+      rank[r] = ((old >> sh) & 0xFFFFu) + __popc(peers & lt);
+    }
+    __syncwarp();
+#else
 #pragma unroll
     for (uint32_t r = 0; r < kR; ++r) {
       const bool valid = kr[r] != ~0ull;
@@ -590,6 +625,7 @@ __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(cons
       }
       __syncwarp();
     }
+#endif
     __syncthreads();
     // per digit: the tile's count, the warps' offsets, publish, look back
     uint32_t cnt[kBPT], csum = 0;
@@ -656,7 +692,16 @@ __global__ void freq_split_kernel(const __grid_constant__ FreqParams q, uint32_t
   q.ctl[2] = lo;
 }
 
-__device__ __forceinline__ int ev_sign(uint64_t key) { return (key & 1ull) ? -1 : 1; }
+// +1 start, -1 end, 0 point (the point's count is added at its element only)
+__device__ __forceinline__ int ev_sign(uint64_t key) {
+  return DRGPUM_FQ_POINTS ? 1 - int(key & 3u) : ((key & 1ull) ? -1 : 1);
+}
+// the element from which the count after this key applies: start g -> g,
+// point g -> g (no change there), end g -> g + 1
+__device__ __forceinline__ uint64_t ev_x(uint64_t pos) {
+  return DRGPUM_FQ_POINTS ? (pos + 2) >> 2 : (pos + 1) >> 1;
+}
+__device__ __forceinline__ bool ev_point(uint64_t key) { return DRGPUM_FQ_POINTS && (key & 3u) == 1; }
 
 // per chunk of kSweepChunk keys of [0, split): sum of the +1 / -1 events
 __global__ void __launch_bounds__(kFT) freq_sweep_sum_kernel(const __grid_constant__ FreqParams q) {
@@ -733,26 +778,47 @@ __global__ void __launch_bounds__(kFT) freq_sweep_kernel(const __grid_constant__
     for (uint32_t j = 0; j < kSweepItems; ++j) if (kk[j] != ~0ull) s += ev_sign(kk[j]);
     uint32_t total;
     int c = int(q.part[b]) + int(block_excl_scan(uint32_t(s), s_w, total));
+    auto locate = [&](uint64_t x0) {                 // object of element x0: shared sample, then global
+      if (x0 >= c_lo && x0 < c_hi) return;
+      uint32_t a = 0, bb = n_samp;
+      while (bb - a > 1) { const uint32_t m = (a + bb) >> 1; if (s_eb[m] <= x0) a = m; else bb = m; }
+      uint32_t lo = a * stride, hi = min(n_obj, lo + stride);
+      while (hi - lo > 1) { const uint32_t m = (lo + hi) >> 1; if (q.elem_base[m] <= x0) lo = m; else hi = m; }
+      const DevObj dv = q.a.objs[lo];
+      c_lo = q.elem_base[lo];
+      c_hi = c_lo + ((dv.end - dv.base) >> dv.shift);
+      c_sb = q.slot_base[lo];
+      c_rlo = dv.r_lo;
+    };
 #pragma unroll
     for (uint32_t j = 0; j < kSweepItems; ++j) {
       if (kk[j] == ~0ull) break;
       c += ev_sign(kk[j]);
+      if (ev_point(kk[j]) && kk[j + 1] != kk[j]) {
+        // last of a run of p equal point keys: element g has count c + p
+        // (c = the intervals covering it, already in its run): n + [c == 0],
+        // S1 + p, S2 + (c + p)^2 - c^2
+        // (the key before it from registers, earlier ones -- long runs -- from L2)
+        uint64_t p = 1;
+        const uint64_t gi = c0 + uint64_t(threadIdx.x) * kSweepItems + j;   // global index of key j
+        if (gi > 0 && (j > 0 ? kk[j - 1] : k[gi - 1]) == kk[j]) {
+          p = 2;
+          while (p <= gi && k[gi - p] == kk[j]) ++p;
+        }
+        const uint64_t g = (kk[j] & pmask) >> 2;
+        locate(g);
+        const uint64_t slot = c_sb + ((kk[j] >> q.pos_bits) - c_rlo);
+        if (slot != ss.slot) { ss.flush(acc); ss.slot = slot; }
+        const uint64_t cu = uint64_t(c);
+        ss.n += cu == 0 ? 1 : 0;
+        ss.s1 += p;
+        ss.s2 += 2 * cu * p + p * p;
+      }
       if (c <= 0 || kk[j + 1] == ~0ull) continue;   // c > 0: the next key belongs to the same API
-      const uint64_t p0 = kk[j] & pmask, p1 = kk[j + 1] & pmask;
-      const uint64_t x0 = (p0 + 1) >> 1, x1 = (p1 + 1) >> 1;
+      const uint64_t x0 = ev_x(kk[j] & pmask), x1 = ev_x(kk[j + 1] & pmask);
       if (x1 <= x0) continue;
       const uint64_t len = x1 - x0;
-      if (!(x0 >= c_lo && x0 < c_hi)) {             // object of element x0: shared sample, then global
-        uint32_t a = 0, bb = n_samp;
-        while (bb - a > 1) { const uint32_t m = (a + bb) >> 1; if (s_eb[m] <= x0) a = m; else bb = m; }
-        uint32_t lo = a * stride, hi = min(n_obj, lo + stride);
-        while (hi - lo > 1) { const uint32_t m = (lo + hi) >> 1; if (q.elem_base[m] <= x0) lo = m; else hi = m; }
-        const DevObj dv = q.a.objs[lo];
-        c_lo = q.elem_base[lo];
-        c_hi = c_lo + ((dv.end - dv.base) >> dv.shift);
-        c_sb = q.slot_base[lo];
-        c_rlo = dv.r_lo;
-      }
+      locate(x0);
       const uint64_t slot = c_sb + ((kk[j] >> q.pos_bits) - c_rlo);
       if (slot != ss.slot) { ss.flush(acc); ss.slot = slot; }
       const uint64_t cu = uint64_t(c);

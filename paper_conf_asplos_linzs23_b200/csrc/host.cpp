@@ -302,7 +302,7 @@ drgpum_status build_tables(drgpum_ctx* c) {
   uint64_t eb = 0;
   for (uint64_t i = 0; i < n; ++i) { c->elem_base[i] = eb; eb += c->objs[i].size / c->objs[i].elem_size; }
   c->n_elem_total = eb;
-  c->fq_pos_bits = std::max<uint32_t>(1, bits_for(2 * eb));        // NEXT-2 keys: 2*element (+1)
+  c->fq_pos_bits = std::max<uint32_t>(1, bits_for(kFreqPosMul * eb));   // NEXT-2 keys: 4*element + type
   c->fq_digits = (c->fq_pos_bits + bits_for(c->n_acc) + kFreqRadixBits - 1) / kFreqRadixBits;   // radix passes
   c->slot_base.assign(n, 0);
   uint64_t sb = 0;

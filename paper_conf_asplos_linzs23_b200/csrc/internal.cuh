@@ -100,7 +100,8 @@ struct SaParams {
 
 // NEXT-2 non-uniform access frequency pass (optional feature), sort-based:
 // every attributed record becomes the element interval it touches, as two
-// event keys (rank << pos_bits) | (2*g0) and (rank << pos_bits) | (2*g1+1)
+// event keys (rank << pos_bits) | (4*g0) and (rank << pos_bits) | (4*g1+2),
+// or one point key (rank << pos_bits) | (4*g+1) for a single element
 // (g = global element index, rank = access-API rank); adjacent disjoint
 // intervals of a warp's consecutive records are merged first.  An LSD radix
 // sort orders the keys by (API, element); a scan of the +1 / -1 events gives
@@ -109,6 +110,12 @@ struct SaParams {
 // API of the call's last records may continue in the next call: its events
 // are carried over, sorted, and swept when the next call (or a query)
 // completes it.
+// Single-element intervals (after merging) as ONE key: positions are
+// 4*g + type, type 0 = start, 1 = point, 2 = end (0: 2*g start, 2*g+1 end).
+#ifndef DRGPUM_FQ_POINTS
+#define DRGPUM_FQ_POINTS 1
+#endif
+constexpr uint64_t kFreqPosMul = DRGPUM_FQ_POINTS ? 4 : 2;
 #ifndef DRGPUM_FQ_TILE
 #define DRGPUM_FQ_TILE 4096
 #endif
