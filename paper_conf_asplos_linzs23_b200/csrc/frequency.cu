@@ -114,6 +114,15 @@ __device__ __forceinline__ uint64_t n_keys(const FreqParams& q) {
   return n < q.cap ? n : q.cap;
 }
 
+// Digit totals: the event and carry kernels count digit 0 only; one-sweep
+// pass d counts digit d + 1 of the keys it ranks (a skipped pass reads the
+// keys for it), so the event kernel -- issue-bound -- does one shared atomic
+// per key instead of one per pass (0: every digit in the event kernel).
+#ifndef DRGPUM_FQ_COUNT_NEXT
+#define DRGPUM_FQ_COUNT_NEXT 1
+#endif
+constexpr bool kFreqCountDigits = DRGPUM_FQ_ONESWEEP && DRGPUM_FQ_COUNT_NEXT;
+
 // ---------------------------------------------------------------- 1. events
 // Every pass's digit totals, counted where the keys are written (the event
 // kernel, and the carry kernel for the carried keys): per-block shared
@@ -144,7 +153,7 @@ __device__ __forceinline__ void ev_flush(const FreqParams& q, uint64_t* out, con
   // mostly uniform high digits) or a MATCH.ANY first measured slower --
   // events 1.12 -> 1.6-2.05 ms on C2
   if (DRGPUM_FQ_ONESWEEP)
-    for (uint32_t j = lane; j < cnt; j += 32) dh.add(buf[j], q.n_digits);
+    for (uint32_t j = lane; j < cnt; j += 32) dh.add(buf[j], kFreqCountDigits ? 1u : q.n_digits);
   unsigned long long base = 0;
   if (lane == 0 && cnt) base = atomicAdd(&q.ctl[0], (unsigned long long)cnt);
   base = __shfl_sync(FULL_MASK, base, 0);
@@ -541,18 +550,38 @@ __global__ void __launch_bounds__(kFT) freq_skip_kernel(const __grid_constant__ 
 __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(const __grid_constant__ FreqParams q, uint32_t d) {
   __shared__ uint64_t s_keys[kFreqTileKeys];
   __shared__ uint16_t s_wc[kFT / 32][kBins];          // per-warp digit counts, then offsets (<= 4096)
-  __shared__ uint32_t s_start[kBins], s_goff[kBins], s_gstart[kBins], s_w[kFT / 32];
+  __shared__ uint32_t s_start[kBins], s_goff[kBins], s_w[kFT / 32];
   __shared__ uint32_t s_tile;
+  __shared__ uint32_t s_nx[kBins];                   // digit d + 1 of this block's keys (kFreqCountDigits)
   const uint64_t n = n_keys(q);
   const uint64_t ntiles = (n + kFreqTileKeys - 1) / kFreqTileKeys;
   volatile uint32_t* status = (d & 1) ? q.offs : q.hist;   // [tile][bin]
   uint32_t* status_next = (d & 1) ? q.hist : q.offs;       // pass d + 1's, cleared here
-  if (q.ctl[8 + d]) {                                // every key has the same digit: pass skipped
-    for (uint64_t i = uint64_t(blockIdx.x) * kFT + threadIdx.x; i < ntiles * kBins; i += uint64_t(gridDim.x) * kFT)
-      status_next[i] = 0;
-    return;
+  const bool count_next = kFreqCountDigits && d + 1 < q.n_digits;
+  bool skip;
+  if (kFreqCountDigits) {   // every key has the same digit d (a total equals n): pass skipped
+    for (uint32_t k = threadIdx.x; k < kBins; k += kFT) s_nx[k] = 0;
+    bool hit = n == 0;
+    for (uint32_t k = threadIdx.x; k < kBins; k += kFT) hit |= digit_totals(q, d)[k] == n;
+    skip = __syncthreads_or(hit);
+    if (blockIdx.x == 0 && threadIdx.x == 0) q.ctl[8 + d] = skip ? 1ull : 0ull;
+  } else {
+    skip = q.ctl[8 + d] != 0;
   }
   const uint32_t src_b = buf_before(q, d);
+  if (skip) {
+    for (uint64_t i = uint64_t(blockIdx.x) * kFT + threadIdx.x; i < ntiles * kBins; i += uint64_t(gridDim.x) * kFT)
+      status_next[i] = 0;
+    if (count_next) {   // the next pass's digit totals from the unmoved keys
+      const uint64_t* kk = keys_buf(q, src_b);
+      for (uint64_t i = uint64_t(blockIdx.x) * kFT + threadIdx.x; i < n; i += uint64_t(gridDim.x) * kFT)
+        atomicAdd(&s_nx[uint32_t(kk[i] >> (kFreqRadixBits * (d + 1))) & (kBins - 1)], 1u);
+      __syncthreads();
+      for (uint32_t k = threadIdx.x; k < kBins; k += kFT)
+        if (s_nx[k]) atomicAdd(digit_totals(q, d + 1) + k, (unsigned long long)s_nx[k]);
+    }
+    return;
+  }
   const uint64_t* src = keys_buf(q, src_b);
   uint64_t* dst = keys_buf(q, src_b ^ 1u);
   const uint32_t shift = kFreqRadixBits * d;
@@ -560,7 +589,8 @@ __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(cons
   const uint32_t lt = (1u << lane) - 1u;
   constexpr uint32_t kR = kFreqTileKeys / kFT;
   uint16_t* wc = s_wc[warp];
-  {   // global digit starts of this pass (exclusive scan of the totals)
+  uint32_t gstart[kBPT];   // global digit starts of this thread's bins (exclusive scan of the totals)
+  {
     const unsigned long long* tot = digit_totals(q, d);
     uint32_t c[kBPT], cs = 0;
 #pragma unroll
@@ -568,7 +598,7 @@ __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(cons
     uint32_t all;
     uint32_t st = block_excl_scan(cs, s_w, all);
 #pragma unroll
-    for (uint32_t b = 0; b < kBPT; ++b) { s_gstart[threadIdx.x * kBPT + b] = st; st += c[b]; }
+    for (uint32_t b = 0; b < kBPT; ++b) { gstart[b] = st; st += c[b]; }
   }
   for (;;) {
     if (threadIdx.x == 0) s_tile = uint32_t(atomicAdd(&q.ctl[16 + d], 1ull));
@@ -584,6 +614,11 @@ __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(cons
     for (uint32_t r = 0; r < kR; ++r) {
       const uint64_t idx = w0 + r * 32 + lane;
       kr[r] = idx < n ? __ldcs(src + idx) : ~0ull;
+    }
+    if (count_next) {
+#pragma unroll
+      for (uint32_t r = 0; r < kR; ++r)
+        if (kr[r] != ~0ull) atomicAdd(&s_nx[uint32_t(kr[r] >> (shift + kFreqRadixBits)) & (kBins - 1)], 1u);
     }
     uint32_t rank[kR];
 #if DRGPUM_FQ_ATOMRANK
@@ -658,7 +693,7 @@ __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(cons
         if (v & kFlagA) { excl += v & kValMask; --pt; }
       }
       if (tile) __stcg(const_cast<uint32_t*>(status) + tile * kBins + bin, kFlagP | (excl + cnt[b]));
-      s_goff[bin] = s_gstart[bin] + excl;
+      s_goff[bin] = gstart[b] + excl;
     }
     __syncthreads();
 #pragma unroll
@@ -676,6 +711,9 @@ __global__ void __launch_bounds__(kFT, DRGPUM_FQ_MINB) freq_onesweep_kernel(cons
     }
     __syncthreads();
   }
+  if (count_next)   // (the loop's last __syncthreads: every count is in)
+    for (uint32_t k = threadIdx.x; k < kBins; k += kFT)
+      if (s_nx[k]) atomicAdd(digit_totals(q, d + 1) + k, (unsigned long long)s_nx[k]);
 }
 
 // ---------------------------------------------------------------- 3. sweep
@@ -843,7 +881,7 @@ __global__ void __launch_bounds__(kFT) freq_carry_kernel(const __grid_constant__
        i += uint64_t(gridDim.x) * blockDim.x) {
     const uint64_t key = src[i];
     dst[i - split] = key;
-    if (DRGPUM_FQ_ONESWEEP) s_dh.add(key, q.n_digits);
+    if (DRGPUM_FQ_ONESWEEP) s_dh.add(key, kFreqCountDigits ? 1u : q.n_digits);
   }
   if (DRGPUM_FQ_ONESWEEP) {
     __syncthreads();
@@ -870,8 +908,10 @@ static void radix_sort(const FreqParams& q, int num_sms, cudaStream_t s, int& la
   // digit totals: counted by the event kernel (and the previous call's carry)
   cudaMemsetAsync(q.ctl + 8, 0, 8 * 16, s);   // skip flags, tickets
   cudaMemsetAsync(q.hist, 0, 4ull * kBins * q.max_tiles, s);   // first pass's look-back status
-  freq_skip_kernel<<<1, kFT, 0, s>>>(q);
-  launches += 1;
+  if (!kFreqCountDigits) {   // skip flags from the totals (otherwise each pass decides its own)
+    freq_skip_kernel<<<1, kFT, 0, s>>>(q);
+    launches += 1;
+  }
   for (uint32_t d = 0; d < q.n_digits; ++d) {
     freq_onesweep_kernel<<<g, kFT, 0, s>>>(q, d);
     launches += 1;
