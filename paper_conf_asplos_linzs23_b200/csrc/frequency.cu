@@ -401,24 +401,28 @@ __global__ void __launch_bounds__(1024) freq_part_scan_kernel(const __grid_const
   } else {
     nb = (q.ctl[2] + kSweepChunk - 1) / kSweepChunk;
   }
+  // thread t scans a contiguous segment: its sum, one block scan of the
+  // sums, then the segment's exclusive prefixes (one round instead of
+  // nb / 1024 block-wide rounds)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  long long carry = 0;
-  for (uint64_t c0 = 0; c0 < nb; c0 += blockDim.x) {
-    const uint64_t i = c0 + threadIdx.x;
-    long long v = 0;
-    if (i < nb) v = mode == 0 ? (long long)q.part[i] : (long long)(int32_t)q.part[i];
-    long long x = v;
-    for (int o = 1; o < 32; o <<= 1) {
-      const long long y = __shfl_up_sync(FULL_MASK, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) s_w[w] = x;
-    __syncthreads();
-    long long before = 0, total = 0;
-    for (int k = 0; k < int(blockDim.x / 32); ++k) { before += k < w ? s_w[k] : 0; total += s_w[k]; }
-    __syncthreads();
-    if (i < nb) q.part[i] = uint32_t(carry + before + x - v);
-    carry += total;
+  const uint64_t seg = (nb + blockDim.x - 1) / blockDim.x;
+  const uint64_t i0 = min(nb, uint64_t(threadIdx.x) * seg), i1 = min(nb, i0 + seg);
+  auto val = [&](uint64_t i) { return mode == 0 ? (long long)q.part[i] : (long long)(int32_t)q.part[i]; };
+  long long v = 0;
+  for (uint64_t i = i0; i < i1; ++i) v += val(i);
+  long long x = v;
+  for (int o = 1; o < 32; o <<= 1) {
+    const long long y = __shfl_up_sync(FULL_MASK, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_w[w] = x;
+  __syncthreads();
+  long long run = x - v;
+  for (int k = 0; k < w; ++k) run += s_w[k];
+  for (uint64_t i = i0; i < i1; ++i) {
+    const long long e = val(i);
+    q.part[i] = uint32_t(run);
+    run += e;
   }
 }
 

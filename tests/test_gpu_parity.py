@@ -126,7 +126,13 @@ def c1():
 
 def test_c1_full(c1):
     p, r = c1
-    check_parity(p.objects, p.kinds, r)
+    s = check_parity(p.objects, p.kinds, r)
+    # diagnostics: every 32-record tile is counted on exactly one path (the
+    # fast-tile count is derived from the fast-record count in the kernel);
+    # chunks are multiples of 32 records except the launch's last one
+    paths = s.path_stats()
+    assert sum(paths.values()) == (len(r) + 31) // 32, paths
+    assert paths["affine_union"] > 0 and paths["tile_fast"] > 0, paths
 
 
 def test_c1_shuffled_and_chunked(c1):

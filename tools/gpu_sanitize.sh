@@ -14,7 +14,7 @@ SEL="tests/test_gpu_parity.py::test_golden_fixtures tests/test_gpu_parity.py::te
  tests/test_gpu_parity.py::test_uint32_size_boundary tests/test_gpu_parity.py::test_range_queue_overflow \
  tests/test_gpu_parity.py::test_range_queue_overflow_c1_and_tiny tests/test_gpu_parity.py::test_cuda_graph_replay \
  tests/test_gpu_merge_peers.py::test_owned_state_rules tests/test_gpu_structured.py::test_random_groups_tiny \
- tests/test_gpu_structured.py::test_gramschmidt_polybench_grouped tests/test_gpu_frequency.py::test_wide_record_queue_overflow \
+ tests/test_gpu_structured.py::test_gramschmidt_polybench_grouped tests/test_gpu_structured.py::test_wide_record_queue_overflow tests/test_gpu_frequency.py::test_sub_calls_and_carried_apis tests/test_gpu_frequency.py::test_c1 \
  tests/test_gpu_merge_peers.py::test_virtual_peers_c1 tests/test_gpu_merge_peers.py::test_virtual_peers_owned_c1 \
  tests/test_gpu_merge_peers.py::test_virtual_peers_owned_tiny_reuse \
  tests/test_gpu_frequency.py::test_tiny tests/test_gpu_frequency.py::test_dependency_chain \

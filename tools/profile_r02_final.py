@@ -1,9 +1,11 @@
-"""Summarise gpurun_out/<tag> of tools/gpu_final_r2.sh into profiles/r02_final.md (run here, no GPU)."""
-import csv, collections, json, subprocess, sys
+"""Summarise gpurun_out/<tag> of tools/gpu_final_r2.sh / gpu_final_r2b.sh into profiles/<out>.md (run here,
+no GPU).  usage: profile_r02_final.py [tag] [out-name]"""
+import csv, collections, json, os, subprocess, sys
 
 tag = sys.argv[1] if len(sys.argv) > 1 else "fin1"
+out = sys.argv[2] if len(sys.argv) > 2 else "r02_final"
 D = f"gpurun_out/{tag}"
-L = [f"# Round 2 final capture (`{D}`, `tools/gpu_final_r2.sh`)", ""]
+L = [f"# Round 2 final capture (`{D}`, `tools/gpu_final_r2.sh` / `tools/gpu_final_r2b.sh`)", ""]
 d = json.loads(open(f"{D}/bench.json").read().strip().splitlines()[-1])
 keep = {k: d[k] for k in ("value", "unit", "ms_per_step", "phases_ms", "roofline", "parity", "clocks", "e2e",
                           "cpu_baseline", "gpu_launches", "step_exec", "counters", "attribution_paths_tiles")}
@@ -36,7 +38,8 @@ mets = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 L += ["## ncu --set full captures", "", "| capture | kernel | " + " | ".join(m.split('.')[0] for m in mets) + " |",
       "|---|---|" + "---|" * len(mets)]
 traffic = {}
-for rep in ("attr_C5", "attr_C2", "fin_C5", "onesweep"):
+for rep in ("attr_C5", "attr_C2", "fin_C5", "onesweep", "freq_events_kernel", "freq_onesweep_kernel"):
+    if not os.path.exists(f"{D}/{rep}.ncu-rep"): continue
     txt = subprocess.run(["ncu", "-i", f"{D}/{rep}.ncu-rep", "--page", "raw", "--csv", "--metrics", ",".join(mets)],
                          capture_output=True, text=True).stdout
     r = list(csv.reader(txt.splitlines()))
@@ -51,11 +54,11 @@ for rep in ("attr_C5", "attr_C2", "fin_C5", "onesweep"):
             b = float(x["dram__bytes_read.sum"]) * sc.get(un["dram__bytes_read.sum"], 1) + \
                 float(x["dram__bytes_write.sum"]) * sc.get(un["dram__bytes_write.sum"], 1)
             traffic[rep[5:]] = int(b)
-open("profiles/r02_final.md", "w").write("\n".join(L) + "\n")
+open(f"profiles/{out}.md", "w").write("\n".join(L) + "\n")
 t = json.load(open("profiles/traffic.json"))
 recs = {"C5": 1 << 30, "C2": 100_000_000}
 for c, b in traffic.items():
     t[c] = {"bytes_per_launch": b, "records_per_launch": recs[c],
-            "source": f"profiles/r02_final.md: ncu --set full of attribute_kernel ({c}, {D}/attr_{c}.ncu-rep): dram read + write per launch"}
+            "source": f"profiles/{out}.md: ncu --set full of attribute_kernel ({c}, {D}/attr_{c}.ncu-rep): dram read + write per launch"}
 json.dump(t, open("profiles/traffic.json", "w"), indent=1)
-print("profiles/r02_final.md", traffic)
+print(f"profiles/{out}.md", traffic)
