@@ -388,8 +388,12 @@ __device__ __forceinline__ void reduce_one_tile(const uint32_t* __restrict__ orw
     }
 }
 
+#ifndef DRGPUM_FIN_UNTOUCHED
+#define DRGPUM_FIN_UNTOUCHED 1   // tiles / hit rows of objects with first[o] = NEVER: closed forms, no loads
+#endif
 __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(const uint32_t* __restrict__ orw,
-    const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr) {
+    const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr,
+    const uint32_t* __restrict__ first) {
   const int lane = threadIdx.x & 31;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctr[C_CONSISTENCY] = 0;   // counted by object_finalize_kernel
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
@@ -403,6 +407,16 @@ __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(cons
   uint4* buf = s_tile[threadIdx.x >> 5];
   for (uint64_t t = gwarp; t < n_tiles; t += nwarps) {
     const Tile tl = tiles[t];
+    if (DRGPUM_FIN_UNTOUCHED && __ldg(first + tl.obj) == kNever) {
+      // an object no record reached: its words are all zero (every
+      // attributed record folds first[], the invariant the sparse reset uses
+      // too) -- the all-zeros monoid of the tile's view, as the loads would give
+      if (lane == 0) {
+        const uint64_t L = (DRGPUM_TR_SMALL && tl.n_words <= 128) ? 4096u : 32768u, nb = tl.n_bits;
+        out[t] = nb == L ? BitMonoid{L, 0, kNoPos, kNoPos, L, L, L} : BitMonoid{L, 0, kNoPos, kNoPos, nb, 0, nb};
+      }
+      continue;
+    }
 #if DRGPUM_TR_SMALL
     if (tl.n_words <= 128) { reduce_one_tile<4>(orw, tl, t, out, buf, lane); continue; }
 #endif
@@ -627,7 +641,8 @@ __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const Fina
         const DevObj ob = p.objs[ol];
         const BitMonoid bm = t1 > t0 ? p.group_part[t0] : bm_identity();
         HitFold f;
-        f.words(p.orw + ob.hit_word, 0, nw, ob.r_lo, acc_ts, acc_cs, p.ti_min_idle);
+        if (!DRGPUM_FIN_UNTOUCHED || p.first[ol] != kNever)   // untouched: an all-zero hit row
+          f.words(p.orw + ob.hit_word, 0, nw, ob.r_lo, acc_ts, acc_cs, p.ti_min_idle);
         HitM hm = hit_identity();
         if (f.cnt) hm = HitM{f.cnt, f.f_ts, f.l_ts, 0, f.ti_cnt, f.ti_max, f.dw, f.ti_sum};
         emit_object(p, ol, ob, bm, hm);
@@ -658,7 +673,7 @@ __global__ void __launch_bounds__(kFinThreads) object_finalize_kernel(const Fina
       // previous non-empty lane's last one (one indexed shuffle), and warp
       // sums / maxima.
       const DevObj ob = p.objs[o];
-      const uint32_t nwords = (2 * p.n_hit[o] + 31) / 32;
+      const uint32_t nwords = (DRGPUM_FIN_UNTOUCHED && p.first[o] == kNever) ? 0u : (2 * p.n_hit[o] + 31) / 32;
       const uint32_t per = (nwords + 31) / 32;
       const uint32_t wlo = min(nwords, lane * per), whi = min(nwords, wlo + per);
       HitFold f;
@@ -696,7 +711,7 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   const uint64_t tb = (nt + 7) / 8;
   const uint64_t cap1 = uint64_t(num_sms) * DRGPUM_TR_GRID_PER_SM;
   const unsigned g1 = (unsigned)(tb < cap1 ? tb : cap1);
-  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles + p.t_lo, nt, p.tile_part + p.t_lo, p.ctr);
+  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles + p.t_lo, nt, p.tile_part + p.t_lo, p.ctr, p.first);
   // mostly single-tile groups (many small objects, C5): 32 groups per warp,
   // single-tile ones copied lane-parallel (C5 finalize 2.77 -> 2.37 ms);
   // otherwise one warp per group (C2: the batched form 83 vs 58 us)
