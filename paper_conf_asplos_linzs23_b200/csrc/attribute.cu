@@ -75,9 +75,6 @@ constexpr int kWarpRecords = kTilesPerWarp * 32;             // 128 records = 2 
 #ifndef DRGPUM_FETCH_V2
 #define DRGPUM_FETCH_V2 1   // per-stage fetch bookkeeping as records-left + next address (A/B macro)
 #endif
-#ifndef DRGPUM_L2PF
-#define DRGPUM_L2PF 0   // stages ahead of the ring prefetched into L2 per fetch (0: none)
-#endif
 #ifndef DRGPUM_TAIL
 #define DRGPUM_TAIL 1   // guided tail (below): C2 0.389 -> 0.381 ms with kBigPct 85; C3 within noise
 #endif
@@ -138,10 +135,6 @@ __device__ __forceinline__ void tma_load_1d(uint32_t dst, const void* gsrc, uint
   asm volatile(
       "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
       ::"r"(dst), "l"(gsrc), "r"(bytes), "r"(bar), "l"(policy) : "memory");
-}
-// L2 prefetch of a bulk range (no shared memory, no completion tracking)
-__device__ __forceinline__ void prefetch_l2(uint64_t gsrc, uint32_t bytes) {
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(gsrc), "r"(bytes) : "memory");
 }
 __device__ __forceinline__ uint64_t evict_first_policy() {
   uint64_t p;
@@ -954,16 +947,6 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
                   evict_first_policy());
       sts64(wsm + kOffSrc, src + 16ull * cnt);
       left -= cnt;
-#if DRGPUM_L2PF
-      // the stage DRGPUM_L2PF stages after this one (inside the chunk) into
-      // L2 now: its TMA, issued that many stages later, then waits for an L2
-      // hit instead of HBM -- the ring's depth without its shared memory
-      if (left > (DRGPUM_L2PF - 1) * kWarpRecords) {
-        const uint32_t rem = left - (DRGPUM_L2PF - 1) * kWarpRecords;
-        prefetch_l2(src + 16ull * (cnt + (DRGPUM_L2PF - 1) * kWarpRecords),
-                    16u * (rem < kWarpRecords ? rem : kWarpRecords));
-      }
-#endif
       sts32(wsm + kOffLeft, left);
       // the next chunk's ticket is taken when this one has at most two stages
       // left: its latency hides behind them, and no warp holds a reservation
