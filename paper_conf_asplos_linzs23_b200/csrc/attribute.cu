@@ -75,32 +75,57 @@ constexpr int kWarpRecords = kTilesPerWarp * 32;             // 128 records = 2 
 #ifndef DRGPUM_FETCH_V2
 #define DRGPUM_FETCH_V2 1   // per-stage fetch bookkeeping as records-left + next address (A/B macro)
 #endif
+#ifndef DRGPUM_TICKET_AHEAD
+#define DRGPUM_TICKET_AHEAD 2   // stages before a chunk's end at which the next chunk's ticket is taken
+#endif
 #ifndef DRGPUM_TAIL
 #define DRGPUM_TAIL 1   // guided tail (below): C2 0.389 -> 0.381 ms with kBigPct 85; C3 within noise
 #endif
 constexpr uint64_t kChunkBig = DRGPUM_CHUNK_BIG, kChunkSmall = DRGPUM_CHUNK_SMALL;
 constexpr uint64_t kBigPct = DRGPUM_BIG_PCT;
 constexpr bool kStatic = DRGPUM_STATIC != 0;
-__device__ __forceinline__ uint64_t chunk_start(uint64_t k, uint64_t n, uint32_t n_warps) {
+// Big chunks grow with the records per warp (launch_attribute: 2^chunk_shift
+// records, 8192 up to kChunkMax while every warp still gets at least
+// kChunksPerWarp of them): each chunk start costs a cold lane cache -- a
+// dependent-load search of the segment index, DRAM misses on C5's 16-MB
+// index -- so long launches take long chunks.  A/B on one box: C5 (302k
+// records per warp and launch) 8192 -> 32768 records: attribution 47.35 ->
+// 42.75 ms; C2 (28k per warp) keeps 8192 (32768: 0.385 -> 0.51 ms).
+#ifndef DRGPUM_CHUNK_MAX_SHIFT
+#define DRGPUM_CHUNK_MAX_SHIFT 13
+#endif
+#ifndef DRGPUM_CHUNKS_PER_WARP
+#define DRGPUM_CHUNKS_PER_WARP 8
+#endif
+static_assert((kChunkBig & (kChunkBig - 1)) == 0, "big chunks are powers of two");
+uint32_t attribute_chunk_shift(uint64_t n, uint64_t n_warps) {
+  uint32_t shift = 0;
+  for (uint64_t c = kChunkBig; (c >> 1) != 0; c >>= 1) ++shift;   // log2(kChunkBig)
+  const uint64_t per = n_warps ? n / n_warps : n;
+  while (shift < DRGPUM_CHUNK_MAX_SHIFT && per >= (2ull << shift) * DRGPUM_CHUNKS_PER_WARP) ++shift;
+  return shift;
+}
+__device__ __forceinline__ uint64_t chunk_start(uint64_t k, uint64_t n, uint32_t n_warps, uint32_t cs) {
+  const uint64_t cb = 1ull << cs;   // big chunk
   if (kStatic) {
     const uint64_t per = n / 100 * kBigPct / n_warps;
     return k <= n_warps ? k * per : n_warps * per + (k - n_warps) * kChunkSmall;
   }
 #if DRGPUM_TAIL
-  // guided tail: 8192-record chunks for the first kBigPct%, then 4096 up to
-  // 95%, 2048 up to 98.5%, 1024 to the end (smaller pieces where the last
-  // warps finish, big ones where chunk-start warm-ups would dominate)
-  const uint64_t b1 = (n / 100 * kBigPct) / kChunkBig * kChunkBig;
+  // guided tail: big chunks for the first kBigPct%, then 4096 up to 95%, 2048
+  // up to 98.5%, 1024 to the end (smaller pieces where the last warps finish,
+  // big ones where chunk-start warm-ups would dominate)
+  const uint64_t b1 = ((n / 100 * kBigPct) >> cs) << cs;
   const uint64_t b2 = b1 + (n / 1000 * 950 - min(n / 1000 * 950, b1)) / 4096 * 4096;
   const uint64_t b3 = b2 + (n / 1000 * 985 - min(n / 1000 * 985, b2)) / 2048 * 2048;
-  const uint64_t k1 = b1 / kChunkBig, k2 = k1 + (b2 - b1) / 4096, k3 = k2 + (b3 - b2) / 2048;
-  if (k <= k1) return k * kChunkBig;
+  const uint64_t k1 = b1 >> cs, k2 = k1 + (b2 - b1) / 4096, k3 = k2 + (b3 - b2) / 2048;
+  if (k <= k1) return k * cb;
   if (k <= k2) return b1 + (k - k1) * 4096;
   if (k <= k3) return b2 + (k - k2) * 2048;
   return b3 + (k - k3) * 1024;
 #else
-  const uint64_t k_big = (n / 100 * kBigPct) / kChunkBig;
-  return k <= k_big ? k * kChunkBig : k_big * kChunkBig + (k - k_big) * kChunkSmall;
+  const uint64_t k_big = (n / 100 * kBigPct) >> cs;
+  return k <= k_big ? k * cb : k_big * cb + (k - k_big) * kChunkSmall;
 #endif
 }
 
@@ -121,13 +146,22 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t byt
 }
 // bar + OFF: the constant offset stays an immediate of the instruction (no
 // hoisted, register-resident base per field)
+#ifndef DRGPUM_MBAR_TEST
+#define DRGPUM_MBAR_TEST 0   // A/B: spin on the non-blocking test_wait instead of try_wait
+#endif
 template <uint32_t OFF>
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   uint32_t done;
   do {
+#if DRGPUM_MBAR_TEST
+    asm volatile(
+        "{ .reg .pred p; mbarrier.test_wait.parity.shared::cta.b64 p, [%1+%3], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done) : "r"(bar), "r"(parity), "n"(OFF) : "memory");
+#else
     asm volatile(
         "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1+%3], %2; selp.u32 %0, 1, 0, p; }"
         : "=r"(done) : "r"(bar), "r"(parity), "n"(OFF) : "memory");
+#endif
   } while (!done);
 }
 __device__ __forceinline__ void tma_load_1d(uint32_t dst, const void* gsrc, uint32_t bytes, uint32_t bar,
@@ -303,6 +337,7 @@ constexpr uint64_t kNoScratch = ~0ull;
 
 struct alignas(16) WarpSmem {
   uint4 ring[kStages][kWarpRecords];   // 3 x 2 KB stages
+  uint4 hint[kStages][4];              // chunk-start hint of the stage (ChunkHint), when flagged
   uint32_t scratch[kScratchWords > 0 ? kScratchWords : 4];   // small-object bitmap copy
   uint64_t sc_base;                    // global word of scratch[0], kNoScratch if unbound
   uint64_t full[kStages];              // one mbarrier per stage
@@ -310,13 +345,16 @@ struct alignas(16) WarpSmem {
   uint32_t f_left, f_last;             // lane 0: records left in the chunk; 1 if it ends the launch
   uint32_t cnt[kStages];               // records in each stage (0 = end of work)
   uint32_t pad;
+  uint32_t rk_meta, rk_rank;           // one-entry (meta -> access rank) cache, filled from chunk hints
   WarpCounts wc;
 };
 constexpr uint32_t kOffFull = offsetof(WarpSmem, full), kOffSrc = offsetof(WarpSmem, f_src),
                    kOffLeft = offsetof(WarpSmem, f_left), kOffLast = offsetof(WarpSmem, f_last),
                    kOffCnt = offsetof(WarpSmem, cnt),
                    kOffWc = offsetof(WarpSmem, wc), kOffScratch = offsetof(WarpSmem, scratch),
-                   kOffScBase = offsetof(WarpSmem, sc_base);
+                   kOffScBase = offsetof(WarpSmem, sc_base), kOffHint = offsetof(WarpSmem, hint),
+                   kOffRk = offsetof(WarpSmem, rk_meta);
+constexpr uint32_t kHintFlag = 0x80000000u;   // in cnt[s]: the stage starts a chunk and carries its hint
 static_assert(offsetof(WarpCounts, aff_w) == offsetof(WarpCounts, aff_u) + 4, "aff_u / aff_w adjacent");
 // block layout: 8 x WarpSmem | level-1 keys (4 KB) | 256 x 56-B lane caches
 // = ~66 KB: three blocks (24 warps) per SM with ~26 KB of L1
@@ -348,8 +386,39 @@ __device__ __forceinline__ FastCache mirror(const SlowCache* c) {
   return FastCache{c->base, c->size, c->bm_word, c->shift, c->meta, small_object(c->size, c->shift)};
 }
 
+// Index loads (segment entries, candidates, object rows, rank table) with an
+// L2 evict-last policy: the record stream is evict-first and the bitmap REDs
+// evict-normal, so the lookups at chunk and burst starts keep finding the
+// index in L2 instead of HBM (C5's index is 32 MB next to 1.25 GiB of shadow).
+#ifndef DRGPUM_INDEX_KEEP
+#define DRGPUM_INDEX_KEEP 1
+#endif
+__device__ __forceinline__ uint64_t evict_last_policy() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint4 ldg_keep4(const void* a) {
+#if DRGPUM_INDEX_KEEP
+  uint4 r;
+  asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(a), "l"(evict_last_policy()));
+  return r;
+#else
+  return __ldg(reinterpret_cast<const uint4*>(a));
+#endif
+}
+__device__ __forceinline__ uint32_t ldg_keep(const uint32_t* a) {
+#if DRGPUM_INDEX_KEEP
+  uint32_t r;
+  asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(a), "l"(evict_last_policy()));
+  return r;
+#else
+  return __ldg(a);
+#endif
+}
 __device__ __forceinline__ SegEntry ldg_seg(const SegEntry* e) {
-  const uint4 v = __ldg(reinterpret_cast<const uint4*>(e));
+  const uint4 v = ldg_keep4(e);
   return SegEntry{(uint64_t(v.y) << 32) | v.x, v.z, v.w};
 }
 
@@ -364,9 +433,9 @@ __device__ __forceinline__ uint32_t resolve_seg(const AttrParams& p, uint32_t re
   const uint2* cand = reinterpret_cast<const uint2*>(p.cand);
   while (l < h) {
     const uint32_t mid = (l + h) >> 1;
-    if (__ldg(&cand[mid].y) < ts) l = mid + 1; else h = mid;
+    if (ldg_keep(&cand[mid].y) < ts) l = mid + 1; else h = mid;
   }
-  return l == c0 ? kNone : __ldg(&cand[l - 1].x);
+  return l == c0 ? kNone : ldg_keep(&cand[l - 1].x);
 }
 
 // Per-lane lookup (A2): level-1 keys (every l1_stride-th segment start) in
@@ -431,11 +500,11 @@ __device__ __forceinline__ uint32_t find_object_warp(const AttrParams& p, const 
   uint32_t hit = kNone;
   for (uint32_t b0 = 0; b0 < aux; b0 += 32) {
     const uint32_t i = b0 + uint32_t(lane);
-    const uint32_t ok = __ballot_sync(FULL_MASK, i < aux && __ldg(&cand[c0 + i].y) < ts);
+    const uint32_t ok = __ballot_sync(FULL_MASK, i < aux && ldg_keep(&cand[c0 + i].y) < ts);
     if (ok) hit = c0 + b0 + uint32_t(31 - __clz(ok));
     if (ok != FULL_MASK) break;   // sorted by t_alloc: the rest are later
   }
-  return hit == kNone ? kNone : __ldg(&cand[hit].x);
+  return hit == kNone ? kNone : ldg_keep(&cand[hit].x);
 }
 
 __device__ __noinline__ void enqueue_range(RangeEntry* rq, uint32_t rq_cap, unsigned long long* ctr,
@@ -489,7 +558,7 @@ __device__ __noinline__ void process_slow(const AttrParams& p, uint4 r, bool pre
   const uint32_t is_w = r.w >> 31;
   // ---- A1: validity (footnote 2: ALLOC/FREE timestamps access nothing)
   bool ok = present && size != 0 && ts < p.n_api && addr <= ~0ull - size;
-  const uint32_t rank = ok ? __ldg(p.acc_rank + ts) : kNone;
+  const uint32_t rank = ok ? ldg_keep(p.acc_rank + ts) : kNone;
   ok = ok && rank != kNone;
   // ---- A2: object lookup
   bool att = false;
@@ -500,7 +569,7 @@ __device__ __noinline__ void process_slow(const AttrParams& p, uint4 r, bool pre
       const uint32_t o = find_object(p, s_l1, addr, ts);
       if (o != kNone) {
         const uint4* q = reinterpret_cast<const uint4*>(p.objs + o);
-        const uint4 a = __ldg(q), b = __ldg(q + 1), d = __ldg(q + 2);
+        const uint4 a = ldg_keep4(q), b = ldg_keep4(q + 1), d = ldg_keep4(q + 2);
         if (ts < d.y) {
           c->base = (uint64_t(a.y) << 32) | a.x;
           c->size = ((uint64_t(a.w) << 32) | a.z) - c->base;
@@ -871,28 +940,45 @@ __device__ __noinline__ bool try_uniform_slow(const AttrParams& p, uint4 r, bool
   if (!__all_sync(FULL_MASK, present && meta == meta0)) return false;
   const uint32_t ts = meta & 0x7FFFFFFFu, is_w = meta >> 31;
   if (ts >= p.n_api) return false;
-  const uint32_t rank = __ldg(p.acc_rank + ts);   // checked after the search: its latency overlaps it
+  // the access rank: from the warp's one-entry cache (a chunk hint's first
+  // record) or loaded; checked after the search, whose latency it overlaps
+  const uint32_t wsm = smem_u32(attr_smem()) + (threadIdx.x >> 5) * uint32_t(sizeof(WarpSmem));
+  const uint32_t rank = lds32<kOffRk>(wsm) == meta ? lds32<kOffRk + 4>(wsm) : ldg_keep(p.acc_rank + ts);
   const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
-  const uint32_t o = find_object_warp(p, s_l1, __shfl_sync(FULL_MASK, addr, 0), ts, lane);
-  if (rank == kNone || o == kNone) return false;
-  const uint4* q = reinterpret_cast<const uint4*>(p.objs + o);
-  const uint4 a = __ldg(q), b = __ldg(q + 1), d = __ldg(q + 2);
-  if (ts >= d.y) return false;
-  const uint64_t base = (uint64_t(a.y) << 32) | a.x;
-  const uint64_t osz = ((uint64_t(a.w) << 32) | a.z) - base;
+  const uint64_t addr0 = __shfl_sync(FULL_MASK, addr, 0);
+  uint64_t base, osz, bm_word, hit_word;
+  uint32_t o, t_alloc, t_free, r_lo, shift;
+  if (__all_sync(FULL_MASK, addr0 - c->base < c->size && ts > c->t_alloc && ts < c->t_free)) {
+    // every lane's cached object contains addr0 and is live at ts: it is THE
+    // object (R5: live objects never overlap) -- no search (chunk starts
+    // with a hint, a new API on the same object)
+    base = c->base; osz = c->size; bm_word = c->bm_word; hit_word = c->hit_word;
+    o = c->obj; t_alloc = c->t_alloc; t_free = c->t_free; r_lo = c->r_lo; shift = c->shift;
+  } else {
+    o = find_object_warp(p, s_l1, addr0, ts, lane);
+    if (o == kNone) return false;
+    const uint4* q = reinterpret_cast<const uint4*>(p.objs + o);
+    const uint4 a = ldg_keep4(q), b = ldg_keep4(q + 1), d = ldg_keep4(q + 2);
+    base = (uint64_t(a.y) << 32) | a.x;
+    osz = ((uint64_t(a.w) << 32) | a.z) - base;
+    bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
+    hit_word = (uint64_t(b.w) << 32) | b.z;
+    t_alloc = d.x; t_free = d.y; r_lo = d.z; shift = d.w;
+  }
+  if (rank == kNone || ts >= t_free) return false;
   if (osz > 0xFFFFFFFFull) return false;
   const uint64_t off = addr - base;
   const uint32_t size = r.z;
-  const uint32_t off32 = uint32_t(off), e0 = off32 >> d.w, e1 = (off32 + size - 1) >> d.w;
+  const uint32_t off32 = uint32_t(off), e0 = off32 >> shift, e1 = (off32 + size - 1) >> shift;
   const bool ok = off < osz && size != 0 && size <= uint32_t(osz) - off32 && e1 - e0 < 32;
   if (!__all_sync(FULL_MASK, ok)) return false;
   c->base = base; c->size = osz;
-  c->bm_word = ((uint64_t(b.y) << 32) | b.x) >> 5;
-  c->hit_word = (uint64_t(b.w) << 32) | b.z;
-  c->t_alloc = d.x; c->t_free = d.y; c->r_lo = d.z; c->shift = d.w; c->obj = o;
+  c->bm_word = bm_word;
+  c->hit_word = hit_word;
+  c->t_alloc = t_alloc; c->t_free = t_free; c->r_lo = r_lo; c->shift = shift; c->obj = o;
   c->meta = meta;
   if (lane == 0) {
-    const uint32_t hb = 2 * (rank - d.z) + is_w;
+    const uint32_t hb = 2 * (rank - r_lo) + is_w;
     red_min(p.first + o, ts);
     red_max(p.last + o, ts);
     red_or(p.orw + c->hit_word + (hb >> 5), 1u << (hb & 31));
@@ -923,13 +1009,15 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
     // a new chunk only every 64 stages; no 64-bit position arithmetic
     uint32_t left = lds32<kOffLeft>(wsm);
     uint64_t src;
+    uint32_t hk = kNone;   // the chunk whose first stage this is (hint index)
     if (left == 0) {
       uint64_t lo, hi;
       do {   // skip empty chunks (only possible at the end or in a tiny static part)
         const uint32_t kc = f_next == kNone ? ticket() : f_next;
+        hk = kc;
         f_next = kNone;
-        lo = min(chunk_start(kc, p.n, n_warps), p.n);
-        hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps), p.n);
+        lo = min(chunk_start(kc, p.n, n_warps, p.chunk_shift), p.n);
+        hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps, p.chunk_shift), p.n);
       } while (lo == hi && lo < p.n);
       if (lo >= p.n) lo = hi = p.n;
       left = uint32_t(hi - lo);
@@ -939,19 +1027,23 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
       src = lds64(wsm + kOffSrc);
     }
     const uint32_t cnt = min(uint32_t(kWarpRecords), left);
-    sts32(wsm + kOffCnt + 4 * s, cnt);
+    const bool hinted = cnt && hk < p.hint_cap;
+    sts32(wsm + kOffCnt + 4 * s, cnt | (hinted ? kHintFlag : 0u));
     const uint32_t bar = wsm + kOffFull + 8 * s;
     if (cnt) {
-      mbar_arrive_expect_tx(bar, cnt * 16);
+      mbar_arrive_expect_tx(bar, cnt * 16 + (hinted ? uint32_t(sizeof(ChunkHint)) : 0u));
       tma_load_1d(wsm + s * (kWarpRecords * 16), reinterpret_cast<const void*>(src), cnt * 16, bar,
                   evict_first_policy());
+      if (hinted)   // the chunk's hint rides on the same barrier
+        tma_load_1d(wsm + kOffHint + s * uint32_t(sizeof(ChunkHint)), p.hints + hk, uint32_t(sizeof(ChunkHint)), bar,
+                    evict_first_policy());
       sts64(wsm + kOffSrc, src + 16ull * cnt);
       left -= cnt;
       sts32(wsm + kOffLeft, left);
       // the next chunk's ticket is taken when this one has at most two stages
       // left: its latency hides behind them, and no warp holds a reservation
       // long enough to unbalance the end of the launch
-      if (left <= 2 * kWarpRecords && f_next == kNone && !lds32<kOffLast>(wsm))
+      if (left <= DRGPUM_TICKET_AHEAD * kWarpRecords && f_next == kNone && !lds32<kOffLast>(wsm))
         f_next = ticket();
     } else {
       mbar_arrive(bar);   // end of work: complete the phase with cnt = 0
@@ -966,8 +1058,8 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
       do {   // skip empty chunks (only possible at the end or in a tiny static part)
         const uint32_t kc = f_next == kNone ? ticket() : f_next;
         f_next = kNone;
-        f_pos = min(chunk_start(kc, p.n, n_warps), p.n);
-        f_hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps), p.n);
+        f_pos = min(chunk_start(kc, p.n, n_warps, p.chunk_shift), p.n);
+        f_hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps, p.chunk_shift), p.n);
       } while (f_pos == f_hi && f_pos < p.n);
       if (f_pos >= p.n) f_pos = f_hi = p.n;
       sts64(wsm + kOffLeft, f_hi);
@@ -1001,6 +1093,7 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
     sts32(wsm + kOffLeft, 0);
     sts32(wsm + kOffLast, 0);
     sts64(wsm + kOffScBase, kNoScratch);
+    sts32(wsm + kOffRk, kNever);
     for (int s = 0; s < kStages; ++s) mbar_init(wsm + kOffFull + 8 * s, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     for (int s = 0; s < kStages; ++s) fetch(s);
@@ -1017,8 +1110,29 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
   for (uint32_t st = 0;; ++st) {
     const int s = int(st % kStages);
     mbar_wait<kOffFull>(wsm + 8 * s, (st / kStages) & 1);
-    const uint32_t cnt = lds32<kOffCnt>(wsm + 4 * s);
+    uint32_t cnt = lds32<kOffCnt>(wsm + 4 * s);
     if (cnt == 0) break;                                   // warp-uniform
+    if (cnt & kHintFlag) {
+      // a new chunk: every lane's cache takes the object of its first record
+      // (resolved by chunk_hint_kernel), with no API folded yet (meta =
+      // NEVER), so the first tile's uniform slow path finds the object in the
+      // cache instead of searching the index
+      cnt &= ~kHintFlag;
+      const uint32_t hb = wsm + kOffHint + s * uint32_t(sizeof(ChunkHint));
+      const uint4 h0 = lds128(hb), h1 = lds128(hb + 16), h2 = lds128(hb + 32), h3 = lds128(hb + 48);
+      if (h3.x != kNone) {
+        SlowCache* my = slow_cache();
+        my->base = (uint64_t(h0.y) << 32) | h0.x;
+        my->size = ((uint64_t(h0.w) << 32) | h0.z) - my->base;
+        my->bm_word = ((uint64_t(h1.y) << 32) | h1.x) >> 5;
+        my->hit_word = (uint64_t(h1.w) << 32) | h1.z;
+        my->t_alloc = h2.x; my->t_free = h2.y; my->r_lo = h2.z; my->shift = h2.w; my->obj = h3.x;
+        my->meta = kNever;
+        c = mirror(my);
+        uni = false;
+        if (lane == 0) { sts32(wsm + kOffRk, h3.y); sts32(wsm + kOffRk + 4, h3.z); }
+      }
+    }
     const int ntiles = int((cnt + 31) / 32);
     // copy the stage to registers (lane l: records l, 32+l, 64+l, 96+l) and refill the slot
     const uint32_t sbuf = wsm + s * (kWarpRecords * 16) + lane * 16;
@@ -1149,6 +1263,45 @@ __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
   }
 }
 
+// Chunk-start hints: thread k resolves the first record of work chunk k (the
+// same chunk_start as the attribution launch that follows) with the per-lane
+// search.  All chunks' lookups run in parallel here, so their dependent
+// index loads overlap, instead of stalling one warp per chunk start inside
+// the attribution (C5: ~10% of the attribution's stall samples were those
+// searches).  The hint is only a candidate: the attribution re-checks that
+// the object contains the record and is live at its timestamp (R5 makes such
+// an object unique), else it searches as before.
+#ifndef DRGPUM_HINT_MIN
+#define DRGPUM_HINT_MIN 0   // launches with fewer records get no hints
+#endif
+__global__ void __launch_bounds__(256) chunk_hint_kernel(const __grid_constant__ AttrParams p, uint32_t n_warps) {
+  __shared__ uint64_t s_l1[kL1MaxKeys];
+  for (uint32_t i = threadIdx.x; i < p.n_l1; i += blockDim.x) s_l1[i] = p.l1[i];
+  __syncthreads();
+  ChunkHint* hints = const_cast<ChunkHint*>(p.hints);
+  for (uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; k < p.hint_cap;
+       k += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t i = chunk_start(k, p.n, n_warps, p.chunk_shift);
+    if (i >= p.n) break;                               // chunk starts grow with k
+    const uint4 r = __ldg(p.recs + i);
+    const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
+    const uint32_t ts = r.w & 0x7FFFFFFFu;
+    uint32_t o = kNone, rank = kNone;
+    DevObj d{};
+    if (ts < p.n_api) rank = __ldg(p.acc_rank + ts);
+    if (r.z != 0 && ts < p.n_api && addr <= ~0ull - r.z && rank != kNone) {
+      o = find_object(p, s_l1, addr, ts);
+      if (o != kNone) {
+        d = p.objs[o];
+        if (ts >= d.t_free) o = kNone;
+      }
+    }
+    ChunkHint h;
+    h.o = d; h.obj = o; h.pad[0] = r.w; h.pad[1] = rank; h.pad[2] = 0;   // pad: the first record's meta, its rank
+    hints[k] = h;
+  }
+}
+
 int attribute_occupancy() {
   int occ = 0;
   cudaFuncSetAttribute(attribute_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kAttrSmem));
@@ -1165,9 +1318,20 @@ int launch_attribute(const AttrParams& p, int num_sms, int occ, cudaStream_t s) 
   const uint64_t full = uint64_t(num_sms) * occ;
   if (blocks > full) blocks = full;
   if (blocks < 1) blocks = 1;
-  attribute_kernel<<<(unsigned)blocks, kAttrThreads, kAttrSmem, s>>>(p);
+  AttrParams q = p;
+  q.chunk_shift = attribute_chunk_shift(p.n, blocks * kConsumerWarps);
+  int launches = 2;
+  if (q.hint_cap && p.n >= DRGPUM_HINT_MIN) {
+    const uint64_t kmax = p.n / 1024 + 2;              // chunks have >= 1024 records but the last
+    q.hint_cap = uint32_t(kmax < q.hint_cap ? kmax : q.hint_cap);
+    chunk_hint_kernel<<<(q.hint_cap + 255) / 256, 256, 0, s>>>(q, uint32_t(blocks * kConsumerWarps));
+    ++launches;
+  } else {
+    q.hint_cap = 0;
+  }
+  attribute_kernel<<<(unsigned)blocks, kAttrThreads, kAttrSmem, s>>>(q);
   range_expand_kernel<<<num_sms * 4, 256, 0, s>>>(p.rq, p.ctr, p.rq_slot, p.rq_cap, p.orw);
-  return 2;
+  return launches;
 }
 
 }  // namespace drgpum

@@ -37,7 +37,7 @@ struct Layout {
   uint64_t dyn_end;
   uint64_t objs, seg_start, seg_cand_off, seg, cand, l1, acc_rank, acc_ts, acc_cs, n_hit;
   uint64_t rfull;                 // per object: a whole-object range was queued in this trace
-  uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage;
+  uint64_t tiles, tile_part, groups, group_off, group_part, stats, reports, rq, stage, hints;
   // NEXT-3 structured access (feature): owner[sum n_elem], overlap[n_obj], elem_base, queue
   uint64_t sa_owner, sa_overlap, sa_elem_base, sa_q, sa_qcount, sa_end, sa_group;
   // NEXT-2 frequency (feature): cells[sum n_elem], acc[n_slots][3], state, queue, outputs
@@ -347,6 +347,7 @@ drgpum_status compute_layout(drgpum_ctx* c) {
   L.stats = put(sizeof(drgpum_object_stats_t) * n);
   L.reports = put(sizeof(drgpum_pattern_report_t) * n);
   L.rq = put(sizeof(RangeEntry) * c->rq_cap);
+  L.hints = put(sizeof(ChunkHint) * kHintCap);
   L.stage = put(2 * kStageRecords * sizeof(drgpum_record_t));
   L.sa_owner = L.sa_overlap = L.sa_elem_base = L.sa_q = L.sa_qcount = L.sa_end = L.sa_group = off;
   if (c->features & (DRGPUM_FEATURE_STRUCTURED | DRGPUM_FEATURE_FREQUENCY)) {
@@ -460,7 +461,10 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   p.rfull = at<uint32_t>(c, c->L.rfull);
   p.rq = at<RangeEntry>(c, c->L.rq);
   p.rq_cap = c->rq_cap;
+  p.hints = at<ChunkHint>(c, c->L.hints);
+  p.hint_cap = kHintCap;
   p.rq_slot = (c->attr_calls & 1) ? C_RQ_COUNT_ALT : C_RQ_COUNT;
+  p.chunk_shift = 13;   // launch_attribute sets the attribution's own
   return p;
 }
 

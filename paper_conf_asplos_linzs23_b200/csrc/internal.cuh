@@ -39,6 +39,13 @@ constexpr uint32_t kMultiBit = 0x80000000u;
 struct alignas(16) SegEntry { uint64_t start; uint32_t ref, aux; };
 static_assert(sizeof(SegEntry) == 16, "SegEntry layout");
 
+// Chunk-start hint (64 B): the object of the first record of an attribution
+// work chunk, resolved for all chunks of a launch at once by
+// chunk_hint_kernel (obj = kNone: no live object / invalid record).
+struct alignas(16) ChunkHint { DevObj o; uint32_t obj; uint32_t pad[3]; };
+static_assert(sizeof(ChunkHint) == 64, "ChunkHint layout");
+constexpr uint32_t kHintCap = 1u << 20;          // chunks per launch that get a hint (64 MB)
+
 // Range-expansion queue entry: inclusive global bit range, <= kRangeChunkWords words.
 struct RangeEntry { uint64_t bit_lo, bit_hi; };
 
@@ -83,6 +90,9 @@ struct AttrParams {
   RangeEntry* rq;
   uint32_t rq_cap;
   uint32_t rq_slot;          // counter slot of this call's range-queue count (C_RQ_COUNT / _ALT)
+  uint32_t chunk_shift;      // log2 of the attribution's big work chunk (set by launch_attribute)
+  const ChunkHint* hints;    // [hint_cap] chunk-start hints (launch_attribute fills them)
+  uint32_t hint_cap;         // chunks with a hint in this launch (0: none)
 };
 
 // NEXT-3 structured access pass (optional feature).
