@@ -85,12 +85,13 @@ constexpr uint64_t kChunkBig = DRGPUM_CHUNK_BIG, kChunkSmall = DRGPUM_CHUNK_SMAL
 constexpr uint64_t kBigPct = DRGPUM_BIG_PCT;
 constexpr bool kStatic = DRGPUM_STATIC != 0;
 // Big chunks grow with the records per warp (launch_attribute: 2^chunk_shift
-// records, 8192 up to kChunkMax while every warp still gets at least
-// kChunksPerWarp of them): each chunk start costs a cold lane cache -- a
-// dependent-load search of the segment index, DRAM misses on C5's 16-MB
-// index -- so long launches take long chunks.  A/B on one box: C5 (302k
-// records per warp and launch) 8192 -> 32768 records: attribution 47.35 ->
-// 42.75 ms; C2 (28k per warp) keeps 8192 (32768: 0.385 -> 0.51 ms).
+// records, from 8192 while every warp still gets at least kChunksPerWarp of
+// them, up to AttrParams::chunk_max_shift: 2^15 when most bitmap tiles are
+// small -- the per-warp scratch path, C5 -- else 2^13).  A/B on one box
+// (DESIGN.md section 6): 8192 -> 16384 -> 32768 records per chunk take C5
+// (302k records per warp and launch) from 47.6 to 44.3 to 42.9 ms and C4
+// from 10.54 to 10.29 to 10.21 ms, but C3 from 2.86 to 3.52 to 4.10 ms; C2
+// (28k per warp) keeps 8192 either way.
 #ifndef DRGPUM_CHUNK_MAX_SHIFT
 #define DRGPUM_CHUNK_MAX_SHIFT 13
 #endif
@@ -98,34 +99,42 @@ constexpr bool kStatic = DRGPUM_STATIC != 0;
 #define DRGPUM_CHUNKS_PER_WARP 8
 #endif
 static_assert((kChunkBig & (kChunkBig - 1)) == 0, "big chunks are powers of two");
-uint32_t attribute_chunk_shift(uint64_t n, uint64_t n_warps) {
+uint32_t attribute_chunk_shift(uint64_t n, uint64_t n_warps, uint32_t max_shift) {
   uint32_t shift = 0;
   for (uint64_t c = kChunkBig; (c >> 1) != 0; c >>= 1) ++shift;   // log2(kChunkBig)
+  const uint32_t cap = max_shift > DRGPUM_CHUNK_MAX_SHIFT ? max_shift : DRGPUM_CHUNK_MAX_SHIFT;
   const uint64_t per = n_warps ? n / n_warps : n;
-  while (shift < DRGPUM_CHUNK_MAX_SHIFT && per >= (2ull << shift) * DRGPUM_CHUNKS_PER_WARP) ++shift;
+  while (shift < cap && per >= (2ull << shift) * DRGPUM_CHUNKS_PER_WARP) ++shift;
   return shift;
 }
-__device__ __forceinline__ uint64_t chunk_start(uint64_t k, uint64_t n, uint32_t n_warps, uint32_t cs) {
-  const uint64_t cb = 1ull << cs;   // big chunk
+// guided tail: big chunks for the first kBigPct%, then 4096 up to 95%, 2048
+// up to 98.5%, 1024 to the end (smaller pieces where the last warps finish,
+// big ones where chunk-start warm-ups would dominate).  The boundaries are
+// computed once per launch on the host (chunk_bounds): a chunk start in the
+// kernel is a few compares and one multiply-add (the in-kernel 64-bit
+// divisions by 100 / 1000 were a dependent chain on lane 0 at every chunk).
+void chunk_bounds(AttrParams& p) {
+  const uint64_t n = p.n;
+  const uint32_t cs = p.chunk_shift;
+  const uint64_t b1 = ((n / 100 * kBigPct) >> cs) << cs;
+  const uint64_t e2 = n / 1000 * 950, e3 = n / 1000 * 985;
+  const uint64_t b2 = b1 + (e2 - (e2 < b1 ? e2 : b1)) / 4096 * 4096;
+  const uint64_t b3 = b2 + (e3 - (e3 < b2 ? e3 : b2)) / 2048 * 2048;
+  p.cb1 = b1; p.cb2 = b2; p.cb3 = b3;
+  p.ck1 = b1 >> cs; p.ck2 = p.ck1 + (b2 - b1) / 4096; p.ck3 = p.ck2 + (b3 - b2) / 2048;
+}
+__device__ __forceinline__ uint64_t chunk_start(uint64_t k, const AttrParams& p, uint32_t n_warps) {
   if (kStatic) {
-    const uint64_t per = n / 100 * kBigPct / n_warps;
+    const uint64_t per = p.n / 100 * kBigPct / n_warps;
     return k <= n_warps ? k * per : n_warps * per + (k - n_warps) * kChunkSmall;
   }
 #if DRGPUM_TAIL
-  // guided tail: big chunks for the first kBigPct%, then 4096 up to 95%, 2048
-  // up to 98.5%, 1024 to the end (smaller pieces where the last warps finish,
-  // big ones where chunk-start warm-ups would dominate)
-  const uint64_t b1 = ((n / 100 * kBigPct) >> cs) << cs;
-  const uint64_t b2 = b1 + (n / 1000 * 950 - min(n / 1000 * 950, b1)) / 4096 * 4096;
-  const uint64_t b3 = b2 + (n / 1000 * 985 - min(n / 1000 * 985, b2)) / 2048 * 2048;
-  const uint64_t k1 = b1 >> cs, k2 = k1 + (b2 - b1) / 4096, k3 = k2 + (b3 - b2) / 2048;
-  if (k <= k1) return k * cb;
-  if (k <= k2) return b1 + (k - k1) * 4096;
-  if (k <= k3) return b2 + (k - k2) * 2048;
-  return b3 + (k - k3) * 1024;
+  if (k <= p.ck1) return k << p.chunk_shift;
+  if (k <= p.ck2) return p.cb1 + (k - p.ck1) * 4096;
+  if (k <= p.ck3) return p.cb2 + (k - p.ck2) * 2048;
+  return p.cb3 + (k - p.ck3) * 1024;
 #else
-  const uint64_t k_big = (n / 100 * kBigPct) >> cs;
-  return k <= k_big ? k * cb : k_big * cb + (k - k_big) * kChunkSmall;
+  return k <= p.ck1 ? k << p.chunk_shift : (p.ck1 << p.chunk_shift) + (k - p.ck1) * kChunkSmall;
 #endif
 }
 
@@ -1016,8 +1025,8 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
         const uint32_t kc = f_next == kNone ? ticket() : f_next;
         hk = kc;
         f_next = kNone;
-        lo = min(chunk_start(kc, p.n, n_warps, p.chunk_shift), p.n);
-        hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps, p.chunk_shift), p.n);
+        lo = min(chunk_start(kc, p, n_warps), p.n);
+        hi = min(chunk_start(uint64_t(kc) + 1, p, n_warps), p.n);
       } while (lo == hi && lo < p.n);
       if (lo >= p.n) lo = hi = p.n;
       left = uint32_t(hi - lo);
@@ -1058,8 +1067,8 @@ __global__ void __launch_bounds__(kAttrThreads, DRGPUM_MINBLOCKS) attribute_kern
       do {   // skip empty chunks (only possible at the end or in a tiny static part)
         const uint32_t kc = f_next == kNone ? ticket() : f_next;
         f_next = kNone;
-        f_pos = min(chunk_start(kc, p.n, n_warps, p.chunk_shift), p.n);
-        f_hi = min(chunk_start(uint64_t(kc) + 1, p.n, n_warps, p.chunk_shift), p.n);
+        f_pos = min(chunk_start(kc, p, n_warps), p.n);
+        f_hi = min(chunk_start(uint64_t(kc) + 1, p, n_warps), p.n);
       } while (f_pos == f_hi && f_pos < p.n);
       if (f_pos >= p.n) f_pos = f_hi = p.n;
       sts64(wsm + kOffLeft, f_hi);
@@ -1272,7 +1281,7 @@ __global__ void __launch_bounds__(256) range_expand_kernel(const RangeEntry* rq,
 // the object contains the record and is live at its timestamp (R5 makes such
 // an object unique), else it searches as before.
 #ifndef DRGPUM_HINT_MIN
-#define DRGPUM_HINT_MIN 0   // launches with fewer records get no hints
+#define DRGPUM_HINT_MIN (1ull << 28)   // launches with fewer records get no hints (C2, 1e8 records: the hint pass cost 2%)
 #endif
 __global__ void __launch_bounds__(256) chunk_hint_kernel(const __grid_constant__ AttrParams p, uint32_t n_warps) {
   __shared__ uint64_t s_l1[kL1MaxKeys];
@@ -1281,7 +1290,7 @@ __global__ void __launch_bounds__(256) chunk_hint_kernel(const __grid_constant__
   ChunkHint* hints = const_cast<ChunkHint*>(p.hints);
   for (uint64_t k = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; k < p.hint_cap;
        k += uint64_t(gridDim.x) * blockDim.x) {
-    const uint64_t i = chunk_start(k, p.n, n_warps, p.chunk_shift);
+    const uint64_t i = chunk_start(k, p, n_warps);
     if (i >= p.n) break;                               // chunk starts grow with k
     const uint4 r = __ldg(p.recs + i);
     const uint64_t addr = (uint64_t(r.y) << 32) | r.x;
@@ -1319,7 +1328,8 @@ int launch_attribute(const AttrParams& p, int num_sms, int occ, cudaStream_t s) 
   if (blocks > full) blocks = full;
   if (blocks < 1) blocks = 1;
   AttrParams q = p;
-  q.chunk_shift = attribute_chunk_shift(p.n, blocks * kConsumerWarps);
+  q.chunk_shift = attribute_chunk_shift(p.n, blocks * kConsumerWarps, p.chunk_max_shift);
+  chunk_bounds(q);
   int launches = 2;
   if (q.hint_cap && p.n >= DRGPUM_HINT_MIN) {
     const uint64_t kmax = p.n / 1024 + 2;              // chunks have >= 1024 records but the last

@@ -465,6 +465,10 @@ AttrParams attr_params(drgpum_ctx* c, const drgpum_record_t* recs, uint64_t n) {
   p.hint_cap = kHintCap;
   p.rq_slot = (c->attr_calls & 1) ? C_RQ_COUNT_ALT : C_RQ_COUNT;
   p.chunk_shift = 13;   // launch_attribute sets the attribution's own
+  // work chunks may grow to 32768 records when most bitmap tiles are small
+  // (objects of <= 4096 elements: the per-warp scratch path, C5); A/B in
+  // DESIGN.md section 6 (C5 / C4 faster with larger chunks, C3 slower)
+  p.chunk_max_shift = 2 * c->n_small_tiles > c->tiles.size() ? kChunkMaxShiftSmall : 13;
   return p;
 }
 

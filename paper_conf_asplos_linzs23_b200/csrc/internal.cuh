@@ -44,6 +44,10 @@ static_assert(sizeof(SegEntry) == 16, "SegEntry layout");
 // chunk_hint_kernel (obj = kNone: no live object / invalid record).
 struct alignas(16) ChunkHint { DevObj o; uint32_t obj; uint32_t pad[3]; };
 static_assert(sizeof(ChunkHint) == 64, "ChunkHint layout");
+#ifndef DRGPUM_CHUNK_MAX_SHIFT_SMALL
+#define DRGPUM_CHUNK_MAX_SHIFT_SMALL 15
+#endif
+constexpr uint32_t kChunkMaxShiftSmall = DRGPUM_CHUNK_MAX_SHIFT_SMALL;   // big-chunk bound, small-object traces
 constexpr uint32_t kHintCap = 1u << 20;          // chunks per launch that get a hint (64 MB)
 
 // Range-expansion queue entry: inclusive global bit range, <= kRangeChunkWords words.
@@ -91,6 +95,10 @@ struct AttrParams {
   uint32_t rq_cap;
   uint32_t rq_slot;          // counter slot of this call's range-queue count (C_RQ_COUNT / _ALT)
   uint32_t chunk_shift;      // log2 of the attribution's big work chunk (set by launch_attribute)
+  uint32_t chunk_max_shift;  // its upper bound (objects_load: larger when small objects dominate)
+  // guided-tail boundaries of the launch's chunks (records b1 < b2 < b3, chunk
+  // indices k1 < k2 < k3; launch_attribute computes them once per launch)
+  uint64_t cb1, cb2, cb3, ck1, ck2, ck3;
   const ChunkHint* hints;    // [hint_cap] chunk-start hints (launch_attribute fills them)
   uint32_t hint_cap;         // chunks with a hint in this launch (0: none)
 };
