@@ -32,4 +32,4 @@ for k in freq_events_kernel freq_onesweep_kernel; do
     python tools/nuaf_prof.py C2 134217728 > $OUT/ncu_$k.log 2>&1; echo "ncu $k rc=$?"
 done
 timeout 300 python tools/nuaf_prof.py C2 134217728 > $OUT/nuaf_prof.txt 2>&1; grep -v -i warn $OUT/nuaf_prof.txt | head -12
-bash tools/gpu_sanitize.sh $TAG/san
+if [ -n "$SAN" ]; then bash tools/gpu_sanitize.sh $TAG/san; fi   # (compute-sanitizer is closed on the current pool)
