@@ -58,6 +58,7 @@ WORKLOADS = {
 # traces above RESIDENT_BYTES per rank are streamed in GEN_CHUNK chunks
 GEN_CHUNK = 1 << 30
 RESIDENT_BYTES = 96 << 30
+CONSUME = False   # reduce-and-clear in Workload steps (main() turns it on unless --no-consume)
 FALLBACK_HBM_GBS = 6650.0
 GOLDEN_DIR = os.path.join(ROOT, "tests", "golden", "digests")
 
@@ -81,6 +82,8 @@ def args_():
                          "merge_or + all-gather")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-next", action="store_true", help="skip the SURVEY §8(f) NEXT-row timings")
+    ap.add_argument("--no-consume", action="store_true",
+                    help="finalize keeps the bitmaps (no reduce-and-clear; the next reset clears them)")
     ap.add_argument("--no-graph", action="store_true",
                     help="time eager launches instead of CUDA-graph replays of the step")
     ap.add_argument("--no-parity", action="store_true", help="skip the golden-digest check")
@@ -310,6 +313,21 @@ class Workload:
         self.owned = self.sm is not None and merge == "owned"
         self.stream = torch.cuda.current_stream()
         self.graph = None
+        # reduce-and-clear: the step's finalize zeroes the bitmap words it
+        # reduces, so the next step's reset skips them (one shadow pass per
+        # step instead of two; no effect after an owned merge)
+        self.consume = CONSUME
+        self.s.set_finalize_consume(self.consume)
+
+    def keep_shadow(self):
+        """One more (untimed) step without reduce-and-clear, so that the
+        shadow holds the trace's bitmaps for the touched-word count and the
+        parity digests read after the timed region (collective at N > 1)."""
+        if self.consume:
+            self.s.set_finalize_consume(False)
+            self.consume = False
+            self.step()
+            self.torch.cuda.synchronize()
 
     # -- the step ------------------------------------------------------------
     def do_merge(self):
@@ -653,6 +671,7 @@ def other_config(cfg, a, hbm, hbm_src):
     w = Workload(cfg)
     steps = max(3, min(a.steps, 10))
     m = measure(w, a, steps, max(2, min(a.warmup, 3)), use_graph=not a.no_graph)
+    w.keep_shadow()
     touched = touched_words(w)
     out = {"workload": WORKLOADS[cfg], "records": w.N, "value": w.N / (m["ms_step"] / 1e3),
            "unit": "records/s", "ms_per_step": m["ms_step"], "steps": steps,
@@ -670,7 +689,9 @@ def other_config(cfg, a, hbm, hbm_src):
 
 
 def main():
+    global CONSUME
     a = args_()
+    CONSUME = not a.no_consume
     world, rank, local = world_env()
     if a.gpus > 1 and "WORLD_SIZE" not in os.environ and a.impl == "ours":
         sys.exit(relaunch(a))
@@ -696,6 +717,7 @@ def main():
         ranks["symmetric_memory_peers"] = len(w.sm.peer_ptrs())
     m = measure(w, a, a.steps, a.warmup, clocks=True, use_graph=not a.no_graph)
     value = w.N / (m["ms_step"] / 1e3)
+    w.keep_shadow()
     touched = touched_words(w)
     parity = None if a.no_parity else parity_check(w, full=(world == 1))
     if world > 1:   # every rank's verdict: all must hold the whole-trace results
@@ -721,7 +743,12 @@ def main():
                                  f"steps' reset + attribute + merge + finalize events)") if w.chunked
                    else "resident in HBM for the whole timed region",
                    "l2": f"inputs larger than L2 ({16 * w.n_local / 2**30:.2f} GiB of records per rank per step)",
-                   "shadow_words": int(w.s.view.or_words), "touched_words": touched},
+                   "shadow_words": int(w.s.view.or_words), "touched_words": touched,
+                   "finalize": ("reduce-and-clear (drgpum_set_finalize_consume): the step's finalize zeroes "
+                                "the bitmap words it reduces and the next step's reset skips them; one "
+                                "untimed plain step after the timed region restores the bitmaps for the "
+                                "touched-word count and the parity digests") if CONSUME and not w.owned
+                               else "plain (the reset clears the touched bitmaps)"},
         "phases_ms": dict(zip(("reset", "attribute", "merge", "finalize"), map(float, m["phases"]))),
         "roofline": rl,
         "parity": parity,

@@ -343,6 +343,19 @@ DRGPUM_API drgpum_status drgpum_merge_peers_owned_nvls(drgpum_ctx *ctx, void *co
 DRGPUM_API drgpum_status drgpum_gather_peers(drgpum_ctx *ctx, void *const *h_peer_ws,
     uint32_t n_peers, uint32_t rank, void *stream);
 
+/* Reduce-and-clear (default off).  While on, drgpum_finalize zeroes every
+ * bitmap word it reduces (the per-object reductions of PAPER.md §5.2 l.268
+ * read each word once), so the next drgpum_reset skips the bitmap tiles: one
+ * pass over the shadow per trace instead of two.  After such a finalize the
+ * bitmaps are CONSUMED: the shadow's bitmap words read back as zero,
+ * drgpum_trace_attribute(_host) and the merge calls return DRGPUM_ESTATE
+ * until drgpum_reset, while object_stats / patterns stay valid (other
+ * thresholds re-run only the classification: the tile reductions are kept).
+ * Hit rows, first / last and counters are untouched.  No effect after
+ * drgpum_merge_peers_owned (the other ranks' objects are not finalized here).
+ * Any time after create; on != 0 enables. */
+DRGPUM_API drgpum_status drgpum_set_finalize_consume(drgpum_ctx *ctx, int on);
+
 /* Enqueue the per-object reductions and the pattern classification on the
  * device (thresholds NULL = defaults).  Asynchronous; the results stay on
  * the device until object_stats / patterns copy them out. */

@@ -60,7 +60,7 @@ class DrgpumError(RuntimeError):
         self.status = status
 
 
-EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_set_features", "drgpum_set_queue_capacity", "drgpum_set_api_group", "drgpum_slice_frequency", "drgpum_set_frequency_capacity", "drgpum_structured",
+EXPORTS = ["drgpum_create", "drgpum_objects_load", "drgpum_set_features", "drgpum_set_finalize_consume", "drgpum_set_queue_capacity", "drgpum_set_api_group", "drgpum_slice_frequency", "drgpum_set_frequency_capacity", "drgpum_structured",
            "drgpum_frequency", "drgpum_frequency_slots",
            "drgpum_workspace_size",
            "drgpum_workspace_bind", "drgpum_reset", "drgpum_trace_attribute",
@@ -106,6 +106,7 @@ def load():
         "drgpum_consistency_errors": ([P, ctypes.POINTER(U64), P], I),
         "drgpum_path_stats": ([P, P, P], I),
         "drgpum_set_features": ([P, U32], I),
+        "drgpum_set_finalize_consume": ([P, ctypes.c_int], I),
         "drgpum_set_queue_capacity": ([P, U32, U32], I),
         "drgpum_set_api_group": ([P, P, P], I),
         "drgpum_set_frequency_capacity": ([P, U64], I),

@@ -163,8 +163,8 @@ __device__ __noinline__ uint32_t interior_zero_run(uint32_t u) {
 // The run-view length of a 4-word-lane tile is 4096 bits; such tiles are
 // always an object's last, so the length only has to cover its real bits.
 template <uint32_t kLaneWords>
-__device__ __forceinline__ void reduce_one_tile(const uint32_t* __restrict__ orw, const Tile& tl, uint64_t t,
-                                                BitMonoid* __restrict__ out, uint4* buf, int lane) {
+__device__ __forceinline__ void reduce_one_tile(uint32_t* __restrict__ orw, const Tile& tl, uint64_t t,
+                                                BitMonoid* __restrict__ out, uint4* buf, int lane, bool consume) {
   constexpr uint32_t kLaneBits = kLaneWords * 32;
   static_assert(kLaneWords == 32 || kLaneWords == 4, "lane widths");
     const uint32_t nbits = uint32_t(tl.n_bits);
@@ -173,8 +173,15 @@ __device__ __forceinline__ void reduce_one_tile(const uint32_t* __restrict__ orw
 #pragma unroll
     for (int b = 0; b < int(kLaneWords / 4); ++b) {
       const uint32_t w = 128 * b + 4 * lane;
-      v[b] = w < tl.n_words ? __ldg(reinterpret_cast<const uint4*>(orw + tl.word_lo + w))
-                            : make_uint4(0, 0, 0, 0);
+      const uint4* a = reinterpret_cast<const uint4*>(orw + tl.word_lo + w);
+      v[b] = w < tl.n_words ? (consume ? *a : __ldg(a)) : make_uint4(0, 0, 0, 0);   // (no .nc path for words it rewrites)
+    }
+    if (consume) {   // reduce-and-clear: every word read is zeroed (the next reset skips the tiles)
+#pragma unroll
+      for (int b = 0; b < int(kLaneWords / 4); ++b) {
+        const uint32_t w = 128 * b + 4 * lane;
+        if (w < tl.n_words) *reinterpret_cast<uint4*>(orw + tl.word_lo + w) = make_uint4(0, 0, 0, 0);
+      }
     }
 #if DRGPUM_TR_UNIFORM
     // whole tiles that are all ones (dense sweeps) or all zeros (untouched
@@ -391,9 +398,9 @@ __device__ __forceinline__ void reduce_one_tile(const uint32_t* __restrict__ orw
 #ifndef DRGPUM_FIN_UNTOUCHED
 #define DRGPUM_FIN_UNTOUCHED 1   // tiles / hit rows of objects with first[o] = NEVER: closed forms, no loads
 #endif
-__global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(const uint32_t* __restrict__ orw,
+__global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(uint32_t* __restrict__ orw,
     const Tile* __restrict__ tiles, uint64_t n_tiles, BitMonoid* __restrict__ out, unsigned long long* ctr,
-    const uint32_t* __restrict__ first) {
+    const uint32_t* __restrict__ first, bool consume) {
   const int lane = threadIdx.x & 31;
   if (blockIdx.x == 0 && threadIdx.x == 0) ctr[C_CONSISTENCY] = 0;   // counted by object_finalize_kernel
   const uint64_t gwarp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
@@ -418,9 +425,9 @@ __global__ void __launch_bounds__(256, DRGPUM_TR_BLOCKS) tile_reduce_kernel(cons
       continue;
     }
 #if DRGPUM_TR_SMALL
-    if (tl.n_words <= 128) { reduce_one_tile<4>(orw, tl, t, out, buf, lane); continue; }
+    if (tl.n_words <= 128) { reduce_one_tile<4>(orw, tl, t, out, buf, lane, consume); continue; }
 #endif
-    reduce_one_tile<32>(orw, tl, t, out, buf, lane);
+    reduce_one_tile<32>(orw, tl, t, out, buf, lane, consume);
   }
 }
 
@@ -711,7 +718,11 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
   const uint64_t tb = (nt + 7) / 8;
   const uint64_t cap1 = uint64_t(num_sms) * DRGPUM_TR_GRID_PER_SM;
   const unsigned g1 = (unsigned)(tb < cap1 ? tb : cap1);
-  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(p.orw, p.tiles + p.t_lo, nt, p.tile_part + p.t_lo, p.ctr, p.first);
+  if (p.skip_tiles) {   // consumed bitmaps: the monoids are in place; the consistency count restarts
+    cudaMemsetAsync(p.ctr + C_CONSISTENCY, 0, sizeof(unsigned long long), s);
+  } else {
+  tile_reduce_kernel<<<g1 ? g1 : 1, 256, 0, s>>>(const_cast<uint32_t*>(p.orw), p.tiles + p.t_lo, nt,
+                                                 p.tile_part + p.t_lo, p.ctr, p.first, p.consume);
   // mostly single-tile groups (many small objects, C5): 32 groups per warp,
   // single-tile ones copied lane-parallel (C5 finalize 2.77 -> 2.37 ms);
   // otherwise one warp per group (C2: the batched form 83 vs 58 us)
@@ -722,6 +733,7 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
     group_reduce_kernel<true><<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
   else
     group_reduce_kernel<false><<<g3 ? g3 : 1, 256, 0, s>>>(p.groups + p.g_lo, ng, p.tile_part, p.group_part + p.g_lo);
+  }
   // lane-parallel small objects when they are the majority (host count,
   // FinalParams::n_small), else one object per warp
   // (only with enough objects to give every SM's warps 32 each: C5's 10^6;
@@ -739,7 +751,7 @@ int launch_finalize(const FinalParams& p, int num_sms, cudaStream_t s) {
     if (lane) object_finalize_kernel<false, true><<<g2, kFinThreads, 0, s>>>(p);
     else object_finalize_kernel<false, false><<<g2, kFinThreads, 0, s>>>(p);
   }
-  return 3;
+  return p.skip_tiles ? 1 : 3;
 }
 
 // ---------------------------------------------------------------- utilities

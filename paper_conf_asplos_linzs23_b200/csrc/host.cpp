@@ -97,6 +97,10 @@ struct drgpum_ctx {
   drgpum_thresholds_t final_th{2, 80, 80};
   // owned merge: this rank holds the merged shadow of objects [own_lo, own_hi) only
   bool owned = false, gathered = false;
+  // reduce-and-clear (drgpum_set_finalize_consume): finalize zeroes the
+  // bitmap words it reduces; consumed = they are zero and the tile monoids
+  // are authoritative until the next reset
+  bool fin_consume = false, consumed = false;
   uint64_t own_lo = 0, own_hi = 0;
   uint32_t own_P = 0, own_rank = 0;
   // host ingest
@@ -419,10 +423,13 @@ drgpum_status enqueue_reset(drgpum_ctx* ctx, cudaStream_t s, bool dense) {
   // later reset): only the touched objects' bitmap tiles and hit rows -- the
   // OR words of an object are nonzero only if its first[] is not NEVER --,
   // then the small sections from first[] on.
+  const bool consumed = ctx->consumed;   // bitmaps already zeroed by a consuming finalize
+  ctx->consumed = false;
   if (dense || !DRGPUM_SPARSE_RESET) {
     ctx->launches += launch_reset(ctx->ws, ctx->L.dyn_end, ctx->L.first, 4 * ctx->n_obj, ctx->num_sms, s);
   } else {
     ctx->launches += launch_reset_touched(at<uint32_t>(ctx, ctx->L.orw), at<Tile>(ctx, ctx->L.tiles),
+                                          consumed ? 0 :
                                           ctx->tiles.size(), at<DevObj>(ctx, ctx->L.objs),
                                           at<uint32_t>(ctx, ctx->L.n_hit), at<uint32_t>(ctx, ctx->L.first),
                                           ctx->n_obj, 2 * ctx->n_small_tiles > ctx->tiles.size(),
@@ -566,6 +573,12 @@ DRGPUM_API drgpum_status drgpum_objects_load(drgpum_ctx* ctx, const drgpum_objec
   ctx->ws_bytes = 0;
   ctx->state = S_LOADED;
   ctx->final_valid = false;
+  return DRGPUM_OK;
+}
+
+DRGPUM_API drgpum_status drgpum_set_finalize_consume(drgpum_ctx* ctx, int on) {
+  if (!ctx) return DRGPUM_EINVAL;
+  ctx->fin_consume = on != 0;
   return DRGPUM_OK;
 }
 
@@ -823,6 +836,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute(drgpum_ctx* ctx, const drgpum_re
   if (n == 0) return DRGPUM_OK;
   if (!d_recs || reinterpret_cast<uintptr_t>(d_recs) % 16)
     return fail(ctx, DRGPUM_EINVAL, "records must be non-NULL and 16-B aligned");
+  if (ctx->consumed) return fail(ctx, DRGPUM_ESTATE, "trace_attribute after a consuming finalize: reset first");
   AttrParams p = attr_params(ctx, d_recs, n);
   ctx->launches += launch_attribute(p, ctx->num_sms, ctx->attr_occ, as_stream(stream));
   ctx->attr_calls++;
@@ -842,6 +856,7 @@ DRGPUM_API drgpum_status drgpum_trace_attribute_host(drgpum_ctx* ctx, const drgp
   if (drgpum_status _d = set_device(ctx)) return _d;
   if (n == 0) return DRGPUM_OK;
   if (!h_recs) return fail(ctx, DRGPUM_EINVAL, "records is NULL");
+  if (ctx->consumed) return fail(ctx, DRGPUM_ESTATE, "trace_attribute_host after a consuming finalize: reset first");
   cudaStream_t st = as_stream(stream);
   if (!ctx->copy_stream) {
     CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking));
@@ -905,6 +920,7 @@ DRGPUM_API drgpum_status drgpum_merge_or(drgpum_ctx* ctx, const uint32_t* d_in, 
                                          uint64_t word_hi, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_or before workspace_bind");
+  if (ctx->consumed) return fail(ctx, DRGPUM_ESTATE, "merge_or after a consuming finalize: reset first");
   if (drgpum_status _d = set_device(ctx)) return _d;
   const uint64_t total = ctx->bitmap_words + ctx->hit_words;
   ctx->final_valid = false;  // the caller is merging state into this shadow
@@ -956,6 +972,7 @@ DRGPUM_API drgpum_status drgpum_merge_peers(drgpum_ctx* ctx, void* const* h_peer
                                             uint32_t rank, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers before workspace_bind");
+  if (ctx->consumed) return fail(ctx, DRGPUM_ESTATE, "merge_peers after a consuming finalize: reset first");
   if (drgpum_status _d = set_device(ctx)) return _d;
   MergePeersParams q{};
   if (drgpum_status e = check_peers(ctx, "merge_peers", h_peer_ws, n_peers, rank, q.peer)) return e;
@@ -1001,6 +1018,7 @@ static drgpum_status merge_owned_impl(drgpum_ctx* ctx, void* const* h_peer_ws, u
                                       uint32_t rank, void* d_mc, void* stream) {
   if (!ctx) return DRGPUM_EINVAL;
   if (ctx->state < S_BOUND) return fail(ctx, DRGPUM_ESTATE, "merge_peers_owned before workspace_bind");
+  if (ctx->consumed) return fail(ctx, DRGPUM_ESTATE, "merge_peers_owned after a consuming finalize: reset first");
   if (drgpum_status _d = set_device(ctx)) return _d;
   MergeOwnedParams q{};
   if (drgpum_status e = check_peers(ctx, "merge_peers_owned", h_peer_ws, n_peers, rank, q.peer)) return e;
@@ -1107,7 +1125,12 @@ DRGPUM_API drgpum_status drgpum_finalize(drgpum_ctx* ctx, const drgpum_threshold
           (ctx->group_off[o + 1] - ctx->group_off[o] <= 1 && (2ull * ctx->n_hit[o] + 31) / 32 <= kLaneHitWords);
   }
   p.n_small = ctx->small_prefix[p.o_hi] - ctx->small_prefix[p.o_lo];
+  // consumed bitmaps: the tile / group monoids of the consuming finalize are
+  // still in place, only the classification runs again
+  p.skip_tiles = ctx->consumed;
+  p.consume = ctx->fin_consume && !ctx->owned && !ctx->consumed;
   ctx->launches += launch_finalize(p, ctx->num_sms, st);
+  if (p.consume) ctx->consumed = true;
   ctx->gathered = false;
   CK(cudaGetLastError());
   ctx->final_valid = true;

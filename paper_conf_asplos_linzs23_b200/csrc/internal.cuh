@@ -203,6 +203,8 @@ struct FinalParams {
   // narrowed it) and their tiles / groups
   uint64_t o_lo, o_hi, t_lo, t_hi, g_lo, g_hi;
   uint64_t n_small;          // objects in [o_lo, o_hi) with one bitmap group and <= kLaneHitWords hit words
+  bool consume;              // tile_reduce zeroes the bitmap words it reads (reduce-and-clear)
+  bool skip_tiles;           // bitmaps consumed earlier: tile / group monoids are already in place
 };
 constexpr uint32_t kLaneHitWords = 128;   // hit rows a single lane folds in object_finalize (<= 2048 APIs)
 

@@ -137,6 +137,12 @@ class Session:
                                                           _stream_handle(stream)))
 
     # ------------------------------------------------------------ results
+    def set_finalize_consume(self, on=True):
+        """drgpum_set_finalize_consume: reduce-and-clear -- finalize zeroes the
+        bitmap words it reduces (bitmaps read back as zero afterwards; stats
+        and patterns stay valid; attribute / merges need a reset first)."""
+        check(self._h, self.L.drgpum_set_finalize_consume(self._h, 1 if on else 0))
+
     def finalize(self, thresholds=None, stream=None):
         th = _thresholds(thresholds)
         check(self._h, self.L.drgpum_finalize(self._h, ctypes.byref(th), _stream_handle(stream)))

@@ -390,3 +390,55 @@ def test_sparse_reset_between_traces():
     assert np.array_equal(s.or_words().cpu().numpy().view(np.uint32),
                           expected_or_words(s, orc, p.objects, p.kinds))
     del orc_any
+
+
+# ---------------------------------------------------------------- reduce-and-clear
+@pytest.mark.parametrize("cfg", ["C1", "tiny"])
+def test_finalize_consume(cfg, c1):
+    """drgpum_set_finalize_consume: finalize zeroes the bitmap words it
+    reduces; stats / reports equal the oracle's (also at other thresholds:
+    only the classification re-runs), the bitmap part of the shadow reads
+    back zero while the hit rows stay, attribution is refused until a reset,
+    and the next trace (sparse reset skipping the consumed tiles) is exact."""
+    from paper_conf_asplos_linzs23_b200 import DrgpumError
+    if cfg == "C1":
+        p, r = c1
+        objs, kinds, recs = p.objects, p.kinds, r
+    else:
+        p = build_tiny(7)
+        objs, kinds, recs = p.objects, p.kinds, gen_all_records(p)
+    orc = Oracle(objs, kinds)
+    orc.attribute(recs)
+    ost, octr = orc.stats()
+    ths = [(2, 80, 80), (5, 50, 90)]
+    oreps = [orc.patterns(th) for th in ths]
+    s = _session(objs, kinds)
+    s.set_finalize_consume(True)
+    d = torch.from_numpy(np.ascontiguousarray(recs).view(np.uint8)).cuda()
+    for rnd in range(3):
+        s.reset()
+        s.attribute(d)
+        s.finalize(ths[0])
+        st, ctr = s.object_stats()
+        for name in octr.dtype.names:
+            assert int(ctr[name]) == int(octr[name]), (rnd, name)
+        for name in ost.dtype.names:
+            if name != "_pad":
+                assert np.array_equal(st[name], ost[name]), (rnd, name)
+        for th, orep in zip(ths, oreps):
+            rep = s.patterns(th)
+            for name in orep.dtype.names:
+                assert np.array_equal(rep[name], orep[name]), (rnd, th, name)
+        assert s.consistency_errors() == 0
+        orw = s.or_words().cpu().numpy().view(np.uint32)
+        nb = int(s.view.bitmap_words)
+        assert not orw[:nb].any(), "bitmap words survived a consuming finalize"
+        exp = expected_or_words(s, orc, objs, kinds)
+        assert np.array_equal(orw[nb:], exp[nb:]), "hit rows changed"
+        with pytest.raises(DrgpumError):
+            s.attribute(d)
+    s.set_finalize_consume(False)   # back to a plain trace: bitmaps kept
+    s.reset()
+    s.attribute(d)
+    s.finalize()
+    assert np.array_equal(s.or_words().cpu().numpy().view(np.uint32), expected_or_words(s, orc, objs, kinds))
