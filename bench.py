@@ -58,7 +58,7 @@ WORKLOADS = {
 # traces above RESIDENT_BYTES per rank are streamed in GEN_CHUNK chunks
 GEN_CHUNK = 1 << 30
 RESIDENT_BYTES = 96 << 30
-CONSUME = False   # reduce-and-clear in Workload steps (main() turns it on unless --no-consume)
+CONSUME = False   # reduce-and-clear in Workload steps (main(): --consume)
 FALLBACK_HBM_GBS = 6650.0
 GOLDEN_DIR = os.path.join(ROOT, "tests", "golden", "digests")
 
@@ -82,8 +82,9 @@ def args_():
                          "merge_or + all-gather")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-next", action="store_true", help="skip the SURVEY §8(f) NEXT-row timings")
-    ap.add_argument("--no-consume", action="store_true",
-                    help="finalize keeps the bitmaps (no reduce-and-clear; the next reset clears them)")
+    ap.add_argument("--consume", action="store_true",
+                    help="reduce-and-clear: finalize zeroes the bitmaps it reduces, the next reset skips them "
+                         "(measured slower than the separate sparse reset: DESIGN.md section 6)")
     ap.add_argument("--no-graph", action="store_true",
                     help="time eager launches instead of CUDA-graph replays of the step")
     ap.add_argument("--no-parity", action="store_true", help="skip the golden-digest check")
@@ -691,7 +692,7 @@ def other_config(cfg, a, hbm, hbm_src):
 def main():
     global CONSUME
     a = args_()
-    CONSUME = not a.no_consume
+    CONSUME = a.consume
     world, rank, local = world_env()
     if a.gpus > 1 and "WORLD_SIZE" not in os.environ and a.impl == "ours":
         sys.exit(relaunch(a))
