@@ -91,7 +91,10 @@ constexpr bool kStatic = DRGPUM_STATIC != 0;
 // (DESIGN.md section 6): 8192 -> 16384 -> 32768 records per chunk take C5
 // (302k records per warp and launch) from 47.6 to 44.3 to 42.9 ms and C4
 // from 10.54 to 10.29 to 10.21 ms, but C3 from 2.86 to 3.52 to 4.10 ms; C2
-// (28k per warp) keeps 8192 either way.
+// (28k per warp) keeps 8192 either way.  C3's loss is one straggler chunk of slow tiles
+// (DESIGN.md section 6), so for any trace a big chunk may also grow while it
+// stays within a quarter of the tail every warp gets (DRGPUM_TAIL_GUARD):
+// C4 (1.13M records per warp) 10.58 -> 10.25 ms, C3 unchanged.
 #ifndef DRGPUM_CHUNK_MAX_SHIFT
 #define DRGPUM_CHUNK_MAX_SHIFT 13
 #endif
@@ -99,12 +102,21 @@ constexpr bool kStatic = DRGPUM_STATIC != 0;
 #define DRGPUM_CHUNKS_PER_WARP 8
 #endif
 static_assert((kChunkBig & (kChunkBig - 1)) == 0, "big chunks are powers of two");
+#ifndef DRGPUM_TAIL_GUARD
+#define DRGPUM_TAIL_GUARD 4   // big chunks <= (tail records per warp) / this, whatever the objects (0: off)
+#endif
 uint32_t attribute_chunk_shift(uint64_t n, uint64_t n_warps, uint32_t max_shift) {
   uint32_t shift = 0;
   for (uint64_t c = kChunkBig; (c >> 1) != 0; c >>= 1) ++shift;   // log2(kChunkBig)
   const uint32_t cap = max_shift > DRGPUM_CHUNK_MAX_SHIFT ? max_shift : DRGPUM_CHUNK_MAX_SHIFT;
   const uint64_t per = n_warps ? n / n_warps : n;
   while (shift < cap && per >= (2ull << shift) * DRGPUM_CHUNKS_PER_WARP) ++shift;
+  // any trace: a big chunk may grow while it stays within a quarter of the
+  // small-chunk tail every warp gets ((100 - kBigPct)% of its records), so
+  // one chunk of slow tiles (C3's straggler) is absorbed by the tail
+  if (DRGPUM_TAIL_GUARD)
+    while (shift < kChunkMaxShiftSmall &&
+           (2ull << shift) * DRGPUM_TAIL_GUARD <= per / 100 * (100 - kBigPct)) ++shift;
   return shift;
 }
 // guided tail: big chunks for the first kBigPct%, then 4096 up to 95%, 2048
